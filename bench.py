@@ -1,0 +1,418 @@
+#!/usr/bin/env python
+"""bench.py -- EST-gradient GB/s reduced (bit-exact across G), % of roofline.
+
+One STEP = one global step of EasyScale's data-parallel hot path over one
+batch of synthetic gradients: for every local EST
+a context switch (k_swap over the Philox record + BN payload) and a stash of
+each bucket (k_stash; the last local EST is borrowed),
+then es_allreduce of every bucket (exchange + canonical fold + 1/N + gather).
+value = N * sum_b L_b * bytes / step time (whole job; inputs resident in HBM).
+
+  python bench.py [--gpus N --steps K --warmup W] [--config resnet50] [--impl reference]
+  (N > 1: torchrun --nproc-per-node N ... bench.py --gpus N ...; NCCL transport)
+
+Prints ONE JSON line on rank 0.  See DESIGN.md "Measurement".
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "EST-gradient GB/s reduced (bit-exact across G) at 1/2/4/8 B200; % of roofline"
+L2_BYTES = 126 * 1024 * 1024
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=50)
+    p.add_argument("--warmup", type=int, default=5)
+    p.add_argument("--impl", default="es200", choices=["es200", "reference"])
+    p.add_argument("--config", default="resnet50",
+                   choices=["tiny", "resnet50", "vgg19", "bert_base", "swin_b"])
+    p.add_argument("--mapping", default="contiguous", choices=["contiguous", "round_robin", "random"])
+    p.add_argument("--sched", default="auto", choices=["auto", "direct", "chain"])
+    p.add_argument("--no-graph", action="store_true", help="eager launches instead of one CUDA graph per step")
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    p.add_argument("--cpu-seconds", type=float, default=10.0)
+    return p.parse_args()
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy read+write)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def cores_used():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count()
+
+
+# ---- clocks sampler ------------------------------------------------------------------------
+
+class Clocks:
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "50"],
+                                         stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+        self.t0 = time.time()
+
+    def mark(self):
+        return time.time()
+
+    def stop(self, t_start, t_end):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.15)
+        self.proc.terminate()
+        self.proc.wait()
+        self.f.flush()
+        rows = []
+        with open(self.f.name) as f:
+            for line in f:
+                parts = [x.strip() for x in line.split(",")]
+                if len(parts) >= 9:
+                    rows.append(parts)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        # samples are ~50 ms apart; keep the ones during the timed window (+1 sample on each side)
+        n = len(rows)
+        total = max(time.time() - self.t0, 1e-3)
+        lo = int(max(0, (t_start - self.t0) / total * n - 1))
+        hi = int(min(n, (t_end - self.t0) / total * n + 2))
+        win = rows[lo:hi] or rows
+        sm = [float(r[1]) for r in win if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in win if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in win for i in range(4) if r[5 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(win)}
+
+
+# ---- oracle legs (cpu_baseline / --impl reference) -----------------------------------------
+
+def oracle_windows(name, fetch, budget_s, seed=0):
+    """Times the oracle, as it stands (single thread), on windows of every
+    bucket until ~budget_s of CPU work.  fetch(k, b, s, n) -> EST k's bucket b
+    elements [s, s+n) as numpy.  Returns (GB/s, sample text, [(b, s, n, out)])."""
+    import numpy as np
+    import oracle
+    from paper_conf_sc_lixyszrljlllq23_b200 import workloads
+    cfg = workloads.config(name)
+    N = cfg["N"]
+    esz = 2 if cfg["dtype"] == "bf16" else 4
+    rng = np.random.default_rng(seed)
+    done_bytes, t_oracle, windows = 0, 0.0, []
+    win = 1 << 18
+    t_begin = time.time()
+    while t_oracle < budget_s and time.time() - t_begin < 3 * budget_s:
+        for b, (L, d) in enumerate(cfg["buckets"]):
+            n = min(win, L)
+            s = int(rng.integers(0, L - n + 1))
+            xs = [fetch(k, b, s, n) for k in range(N)]
+            t0 = time.perf_counter()
+            out = oracle.reduce(xs, d, L=L, first=s)
+            t_oracle += time.perf_counter() - t0
+            done_bytes += N * n * esz
+            windows.append((b, s, n, out))
+            if t_oracle >= budget_s:
+                break
+    gbs = done_bytes / t_oracle / 1e9
+    sample = (f"{len(windows)} windows of <= {win} elements x {N} ESTs across the {len(cfg['buckets'])} buckets "
+              f"({done_bytes / 1e6:.1f} MB of EST gradients, {t_oracle:.1f} s single-thread C oracle)")
+    return gbs, sample, windows
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    from paper_conf_sc_lixyszrljlllq23_b200 import workloads
+    name = args.config
+    cfg = workloads.config(name)
+    cache = {}
+
+    def fetch(k, b, s, n):
+        if (k, b) not in cache:
+            t = workloads.est_bucket(name, k, b, device="cpu")
+            cache[(k, b)] = t.numpy() if cfg["dtype"] == "f32" else t.view(__import__("torch").int16).numpy().view("uint16")
+        return cache[(k, b)][s:s + n]
+
+    # one "step" = one bounded sample of the workload; K timed samples after W warm-ups
+    budget = max(0.5, min(args.cpu_seconds, 60.0 / max(1, args.steps + args.warmup)))
+    for _ in range(args.warmup):
+        oracle_windows(name, fetch, budget * 0.2, seed=1)
+    rates, sample = [], ""
+    for i in range(args.steps):
+        gbs, sample, _ = oracle_windows(name, fetch, budget, seed=100 + i)
+        rates.append(gbs)
+    value = statistics.median(rates)
+    payload = workloads.payload_bytes(name)
+    ms = payload / (value * 1e9) * 1e3
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GB/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 3), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": cfg["dtype"], "data": "synthetic",
+        "config": {"workload": name, "N": cfg["N"], "G": world, "desc": cfg["desc"]},
+        "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                         "sample": sample + "; ms_per_step extrapolates the full step"},
+        "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ---- the GPU arm ------------------------------------------------------------------------------
+
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_lixyszrljlllq23_b200 import es, workloads
+    from paper_conf_sc_lixyszrljlllq23_b200.aggregator import Aggregator, nccl_comm_ptr
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    comm = None
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+        t = torch.ones(1, device=dev)
+        dist.all_reduce(t)                       # create the NCCL communicator
+        torch.cuda.synchronize()
+        comm = nccl_comm_ptr()
+    name = args.config
+    cfg = workloads.config(name)
+    N, G = cfg["N"], world
+    mapping = workloads.mapping(N, G, args.mapping)
+    local = [k for k in range(N) if mapping[k] == rank]
+    buckets = cfg["buckets"]
+    B = len(buckets)
+    sched = {"auto": es.ES_SCHED_AUTO, "direct": es.ES_SCHED_DIRECT, "chain": es.ES_SCHED_CHAIN}[args.sched]
+    snb = workloads.state_nbytes()
+    agg = Aggregator(N, G, rank, mapping, buckets, state_nbytes=snb,
+                     transport=es.ES_TRANSPORT_NONE if G == 1 else es.ES_TRANSPORT_NCCL, comm=comm, sched=sched,
+                     device=dev)
+    live = [torch.zeros(n, dtype=torch.uint8, device=dev) for n in snb]
+    agg.register_state(live)
+    for k in local:
+        for i, blob in enumerate(workloads.est_state(name, k)):
+            agg.init_state(k, i, blob)
+    grads = {k: [workloads.est_bucket(name, k, b, device=dev) for b in range(B)] for k in local}
+    outs = [agg.new_out(b) for b in range(B)]
+    esz = 2 if cfg["dtype"] == "bf16" else 4
+    in_bytes = len(local) * sum(n for n, _ in buckets) * esz
+    flush = None if in_bytes > 2 * L2_BYTES else torch.empty(4 * L2_BYTES, dtype=torch.uint8, device=dev)
+    torch.cuda.synchronize()
+
+    def step():
+        for i, k in enumerate(local):
+            agg.switch(k)
+            for b in range(B):
+                agg.stash(k, b, grads[k][b], es.ES_STASH_BORROW if i == len(local) - 1 else es.ES_STASH_COPY)
+        for b in range(B):
+            agg.allreduce(b, outs[b])
+
+    use_graph = not args.no_graph
+    stream = torch.cuda.Stream(device=dev)
+    for _ in range(max(args.warmup, 3) if not use_graph else 2):
+        with torch.cuda.stream(stream):
+            step()
+    torch.cuda.synchronize()
+    graph = None
+    agg.profile(True)
+    agg.profile_reset()
+    if use_graph:
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph, stream=stream):
+            step()
+        torch.cuda.synchronize()
+        for _ in range(max(args.warmup, 3)):
+            with torch.cuda.stream(stream):
+                graph.replay()
+        torch.cuda.synchronize()
+    else:
+        for _ in range(max(args.warmup, 3) - 2):
+            with torch.cuda.stream(stream):
+                step()
+        torch.cuda.synchronize()
+        agg.profile_reset()
+
+    clocks = Clocks(local_rank)
+    clocks.start()
+    time.sleep(0.3)
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t_start = time.time()
+    with torch.cuda.stream(stream):
+        for i in range(args.steps):
+            if flush is not None:
+                flush.zero_()                     # L2 flush between timed steps (untimed)
+            starts[i].record(stream)
+            if graph is not None:
+                graph.replay()
+            else:
+                step()
+            ends[i].record(stream)
+    torch.cuda.synchronize()
+    t_end = time.time()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop(t_start, t_end)
+    step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
+    ms = sum(step_ms) / len(step_ms)
+    if world > 1:
+        t = torch.tensor([ms], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+
+    kinds = {"stash": es.ES_KERNEL_STASH, "fold": es.ES_KERNEL_FOLD, "swap": es.ES_KERNEL_SWAP}
+    prof = {k: agg.profile_query(v) for k, v in kinds.items()}   # (launches, ms, bytes)
+    agg.profile(False)
+    steps_profiled = 1 if graph is not None else args.steps
+    launches_per_step = sum(p[0] for p in prof.values()) / (1 if graph is not None else args.steps)
+    fl_n, fl_ms, fl_bytes = prof["fold"]
+    payload = workloads.payload_bytes(name)
+    value = payload / (ms / 1e3) / 1e9
+    peak, peak_src = peaks()
+    achieved = fl_bytes / (fl_ms / 1e3) / 1e9 if fl_ms > 0 else None
+    per_launch = fl_bytes / max(fl_n, 1)
+    traffic = None
+    tfile = os.path.join(ROOT, "profiles", f"traffic_{name}_g{G}.json")
+    if os.path.exists(tfile):
+        with open(tfile) as f:
+            traffic = json.load(f).get("fold_dram_bytes_per_launch")
+
+    line = {
+        "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": cfg["dtype"], "data": "synthetic",
+        "config": {"workload": name, "N": N, "G": G, "mapping": args.mapping, "sched": args.sched,
+                   "buckets": B, "elements": sum(n for n, _ in buckets), "graph": graph is not None,
+                   "l2": ("inputs larger than L2 (%.1f MB of EST gradients per GPU per step)" % (in_bytes / 1e6))
+                   if flush is None else "L2 flushed between timed steps (512 MB write)",
+                   "desc": cfg["desc"]},
+        "roofline": {"bound": "hbm", "kernel": "k_fold", "achieved": round(achieved, 1) if achieved else None,
+                     "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4) if achieved else None,
+                     "traffic": traffic, "algorithmic_bytes_per_launch": int(per_launch),
+                     "launches_per_step": int(fl_n / steps_profiled),
+                     "avg_launch_us": round(fl_ms / max(fl_n, 1) * 1e3, 2), "peak_source": peak_src},
+        "breakdown_ms_per_step": {k: round(v[1] / steps_profiled, 4) for k, v in prof.items()},
+        "gpu_launches": int(round(launches_per_step * args.steps)),
+        "clocks": clk,
+    }
+
+    # ---- parity of the timed outputs against the oracle on sampled windows (+ cpu_baseline) ----
+    if rank == 0:
+        import oracle  # test infrastructure: the cpu_baseline leg and parity check only
+        gen_cache = {}
+
+        def fetch(k, b, s, n):
+            if k in grads:
+                t = grads[k][b][s:s + n]
+            else:                                   # remote EST: regenerate its seeded input
+                if (k, b) not in gen_cache:
+                    gen_cache[(k, b)] = workloads.est_bucket(name, k, b, device=dev)
+                t = gen_cache[(k, b)][s:s + n]
+            t = t.cpu()
+            return t.numpy() if t.dtype == torch.float32 else t.view(torch.int16).numpy().view(np.uint16)
+
+        budget = args.cpu_seconds if (world == 1 and not args.no_cpu) else 1.0
+        gbs, sample, windows = oracle_windows(name, fetch, budget)
+        mism = 0
+        checked = 0
+        for b, s, n, want in windows:
+            got = outs[b][s:s + n].cpu()
+            got = got.numpy() if got.dtype == torch.float32 else got.view(torch.int16).numpy().view(np.uint16)
+            w = want.view(np.uint32 if want.dtype == np.float32 else np.uint16)
+            g_ = got.view(w.dtype)
+            mism += int((w != g_).sum())
+            checked += n
+        line["parity"] = {"checked_elements": checked, "mismatched_words": mism, "vs": "CPU oracle, bit-exact"}
+        if world == 1 and not args.no_cpu:
+            line["cpu_baseline"] = {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                                    "sample": sample, "host_cores_available": cores_used()}
+
+    # ---- e2e: public API with host buffers (pinned H2D in, D2H out, inside the timed region) ----
+    if not args.no_e2e:
+        host = {k: [g.cpu().pin_memory() for g in grads[k]] for k in local}
+        live_grad = [torch.empty_like(grads[local[0]][b]) for b in range(B)]
+        host_out = [torch.empty(o.shape, dtype=o.dtype).pin_memory() for o in outs]
+        h2d = len(local) * sum(n for n, _ in buckets) * esz
+        d2h = sum(n for n, _ in buckets) * esz
+
+        def e2e_step():
+            for i, k in enumerate(local):
+                for b in range(B):
+                    live_grad[b].copy_(host[k][b], non_blocking=True)     # "backward" lands in the live buffer
+                agg.switch(k)
+                for b in range(B):
+                    agg.stash(k, b, live_grad[b], es.ES_STASH_BORROW if i == len(local) - 1 else es.ES_STASH_COPY)
+            for b in range(B):
+                agg.allreduce(b, outs[b])
+                host_out[b].copy_(outs[b], non_blocking=True)
+
+        k_e2e = max(3, min(args.steps, 10))
+        with torch.cuda.stream(stream):
+            e2e_step()
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with torch.cuda.stream(stream):
+            e0.record(stream)
+            for _ in range(k_e2e):
+                e2e_step()
+            e1.record(stream)
+        torch.cuda.synchronize()
+        ems = e0.elapsed_time(e1) / k_e2e
+        if world > 1:
+            t = torch.tensor([ems], device=dev, dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ems = float(t.item())
+        line["e2e"] = {"value": round(payload / (ems / 1e3) / 1e9, 3), "unit": "GB/s", "h2d_bytes_per_step": h2d,
+                       "d2h_bytes_per_step": d2h, "ms_per_step": round(ems, 3), "steps": k_e2e}
+    agg.sync()
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

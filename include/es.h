@@ -1,0 +1,263 @@
+/*
+ * es.h -- C ABI of libes, the B200-native placement-invariant EST gradient
+ * aggregator (EasyScale, SC '23; PAPER.md = arXiv 2208.14228v3 text).
+ *
+ * "P:n" cites line n of PAPER.md; "Rn" cites a reading in DESIGN.md
+ * ("Readings of the paper"), which fixes what the paper leaves unstated.
+ *
+ * The hot path (PAPER.md 3.2 "EasyScaleThread", and 3.3 "D1
+ * elastic determinism"):
+ *
+ *   N logical EasyScaleThreads (ESTs) -- DDP workers with constant virtual
+ *   ranks 0..N-1 -- are time-sliced onto G GPUs.
+ *   At each EST's context switch its gradient buckets are stashed
+ *   (es_stash_grad) and its RNG / BatchNorm context is swapped
+ *   (es_switch_context).  After the last local EST the
+ *   buckets are aggregated across all N ESTs (es_allreduce, P:526-532,
+ *   P:963-967) in ONE canonical order that depends only on N, the persisted
+ *   bucket layout and the chunk alignment A -- never on G or on the
+ *   EST->GPU mapping -- so the result is bitwise identical for any placement
+ *   (D1; readings R1-R6, R13):
+ *
+ *     C = A*ceil(ceil(L/N)/A);  element i lies in chunk c = floor(i/C);
+ *     s = x[(c+1)%N][i];  for j = 2..N: s = fl32(s + x[(c+j)%N][i]);
+ *     out[i] = round_to_bucket_dtype(fl32(s * fl32(1/N))).
+ *
+ * Conventions for every function:
+ *   - extern "C", never throws, returns es_status (ES_OK == 0).
+ *   - Pointers named *_dev / grad / out / workspace are CUDA device pointers
+ *     (cudaMalloc / torch CUDA storage) on the calling thread's current
+ *     device; host_* pointers are ordinary host memory.
+ *   - Argument errors (ES_EINVAL) are detected synchronously and have no
+ *     side effects.  Protocol errors return ES_ESTATE.  A CUDA / NCCL error
+ *     at enqueue time returns ES_ECUDA / ES_ENCCL and poisons the handle:
+ *     every later call on it returns the same status (sticky).
+ *     Asynchronous device faults surface at es_sync().
+ *   - es_last_error() returns a thread-local human-readable detail string
+ *     for the most recent failing call on this thread.
+ *   - A handle is not thread-safe; use one handle per thread (one per GPU
+ *     rank).  Different handles may be used concurrently.
+ */
+#ifndef ES_H
+#define ES_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define ES_ABI_VERSION 1
+
+typedef struct es_ctx *es_handle;        /* opaque; one per rank (= per GPU) */
+typedef struct CUstream_st *es_stream;   /* identical to cudaStream_t; NULL = legacy default stream */
+
+typedef enum {
+  ES_OK = 0,
+  ES_EINVAL = 1,        /* bad argument (synchronous, no side effects)            */
+  ES_ESTATE = 2,        /* protocol violation (missing stash, non-local EST, ...)  */
+  ES_ENOMEM = 3,        /* workspace too small                                     */
+  ES_ECUDA = 4,         /* CUDA runtime error (sticky)                             */
+  ES_ENCCL = 5,         /* NCCL error / NCCL library not loadable (sticky)         */
+  ES_EUNSUPPORTED = 6   /* feature not available in this build / on this device   */
+} es_status;
+
+/* Element types.  A bucket's dtype is the dtype of its slots and of the
+ * aggregated output; accumulation is always fp32 (R4). */
+typedef enum { ES_F32 = 0, ES_BF16 = 1 } es_dtype;
+
+/* ES_STASH_COPY copies (or casts) the gradient into the EST's slot in the
+ * workspace; the caller may overwrite `grad` once `stream` has passed the
+ * call.  ES_STASH_BORROW records the pointer only -- the paper's last local
+ * EST, whose gradients are synchronised in place; the buffer
+ * must stay unchanged until es_allreduce of that bucket has completed on
+ * its stream, and must already hold the bucket dtype. */
+typedef enum { ES_STASH_COPY = 0, ES_STASH_BORROW = 1 } es_stash_mode;
+
+/* Exchange schedule for G > 1.  Both produce the
+ * same bits; they differ only in NVLink bytes.
+ *   DIRECT: GPU g owns element shard S_g, receives the N - n_g remote
+ *           contributions for it, folds all N in canonical order, then the
+ *           shards are all-gathered.
+ *   CHAIN:  chunk c's unrounded fp32 partial walks the GPUs in canonical
+ *           EST order; each GPU folds its consecutive local ESTs; the GPU of
+ *           EST c scales, rounds and owns chunk c; then all-gather.
+ *   AUTO:   per bucket, the one with fewer max-per-GPU received bytes
+ *           (ties -> DIRECT).  The choice is identical on every rank. */
+typedef enum { ES_SCHED_AUTO = 0, ES_SCHED_DIRECT = 1, ES_SCHED_CHAIN = 2 } es_sched;
+
+/* How ranks exchange bytes when G > 1.
+ *   NONE:     G == 1 only.
+ *   NCCL:     `comm` is a borrowed ncclComm_t over exactly the G ranks
+ *             (e.g. torch ProcessGroupNCCL._comm_ptr()).  Only point-to-point
+ *             ncclSend/ncclRecv inside ncclGroupStart/End are used -- never an
+ *             NCCL reduction, whose order is not the canonical one.  libnccl is
+ *             resolved at es_init from the copy already loaded in the process
+ *             (dlopen RTLD_NOLOAD "libnccl.so.2"), else dlopen'ed by name.
+ *   LOOPBACK: `comm` is an es_loopback world (es_loopback_create); all G ranks
+ *             live in ONE process, each driven by its own host thread, all
+ *             on the same device; bytes move with cudaMemcpyAsync.  Test
+ *             transport that lets a single GPU run every G and mapping. */
+typedef enum { ES_TRANSPORT_NONE = 0, ES_TRANSPORT_NCCL = 1, ES_TRANSPORT_LOOPBACK = 2 } es_transport;
+
+/* One DDP gradient bucket; its index in the array is the bucket id.  The
+ * bucket layout is persisted state and part of the canonical definition
+ * (R8, R9). */
+typedef struct {
+  uint64_t numel;       /* elements, < 2^31 */
+  es_dtype dtype;
+} es_bucket_desc;
+
+typedef struct {
+  int32_t N;                      /* logical ESTs, 1..1024                         */
+  int32_t G;                      /* GPUs (ranks), 1..64, G <= N                               */
+  int32_t rank;                   /* this process's GPU rank, 0..G-1                           */
+  const int32_t *est_to_gpu;      /* host [N]: GPU of each EST; every GPU owns >= 1 EST (R10);
+                                     identical on all ranks                                    */
+  const es_bucket_desc *buckets;  /* host [n_buckets]: persisted layout (D1)                   */
+  int32_t n_buckets;              /* 1..4096                                                   */
+  uint32_t chunk_align;           /* A in elements; 0 => 16; must be a multiple of 8 (R1)      */
+  int32_t n_state;                /* registered per-EST context buffers (Philox record, BN
+                                     running stats), 0..4096            */
+  const uint64_t *state_nbytes;   /* host [n_state]: bytes of each context buffer              */
+  es_transport transport;
+  void *comm;                     /* ncclComm_t (NCCL), es_loopback world (LOOPBACK), NULL (NONE) */
+  es_sched sched;
+} es_config;
+
+/* ---- sizing / lifetime --------------------------------------------------- */
+
+/* Bytes of device workspace es_init needs for `cfg` (per-EST gradient and
+ * context slots for the local ESTs, exchange staging, chain partials,
+ * tables).  Host-only; no CUDA call.  ES_EINVAL on an invalid config. */
+es_status es_workspace_bytes(const es_config *cfg, size_t *bytes);
+
+/* Creates a handle.  `workspace` is caller-owned device memory of at least
+ * es_workspace_bytes() bytes, 256-byte aligned, outliving the handle; the
+ * library never calls cudaMalloc (PyTorch stays the only device allocator)
+ * and owns only host metadata, CUDA events and, for G > 1, its planner
+ * tables.  The bucket plan (chunk table, shards, schedule, exchange ops) is
+ * computed here once and never rebuilt (D1).  Elastic change of
+ * G or of the mapping = es_destroy + es_init with the same N, layout and A
+ * (P:619-624).  cfg and its arrays are copied. */
+es_status es_init(const es_config *cfg, void *workspace, size_t workspace_bytes, es_handle *out);
+
+/* Releases host resources.  Does not synchronise; the caller must not
+ * destroy a handle with work still in flight (call es_sync first). */
+es_status es_destroy(es_handle h);
+
+/* Waits for all work this handle enqueued and reports asynchronous faults
+ * (ES_ECUDA, sticky). */
+es_status es_sync(es_handle h);
+
+/* ---- EST context: stash + state swap ----------------------------------- */
+
+/* Binds the live copies of the n == cfg.n_state context buffers (device
+ * pointers, 16-byte aligned, sizes as in cfg.state_nbytes).  Must precede
+ * es_switch_context when n_state > 0. */
+es_status es_register_state(es_handle h, int32_t n, void *const *live_dev_ptrs);
+
+/* Synchronously writes the saved copy of context buffer `idx` of local EST
+ * `est` from host memory (state_nbytes[idx] bytes).  Used to seed each
+ * EST's Philox record / BN statistics (D0: fixed seeds). */
+es_status es_init_state(es_handle h, int32_t est, int32_t idx, const void *host_src);
+
+/* Synchronously reads the saved copy of context buffer `idx` of local EST
+ * `est` into host memory.  (The live copy belongs to the running EST.) */
+es_status es_read_state(es_handle h, int32_t est, int32_t idx, void *host_dst);
+
+/* Context switch to local EST `est` at a mini-batch boundary:
+ * one kernel saves every live context buffer into the current EST's slot
+ * and loads `est`'s slot into the live buffers.  The first switch only
+ * loads.  Switching to the current EST is a no-op.  ES_ESTATE if `est` is
+ * not mapped to this rank. */
+es_status es_switch_context(es_handle h, int32_t est, es_stream stream);
+
+/* Stashes local EST `est`'s gradient for `bucket`.
+ * grad: device pointer, 16-byte aligned, `numel` elements of grad_dtype.
+ * COPY: one vectorised kernel copies/casts into the EST's slot (RNE when
+ * narrowing fp32->bf16, exact when widening).  BORROW: grad_dtype must
+ * equal the bucket dtype; the pointer is recorded.  Either way an event on
+ * `stream` orders the stash before the bucket's next es_allreduce.
+ * ES_ESTATE if `est` is not mapped to this rank. */
+es_status es_stash_grad(es_handle h, int32_t est, int32_t bucket, const void *grad,
+                        es_dtype grad_dtype, es_stash_mode mode, es_stream stream);
+
+/* ---- aggregation ---------------------------------------------------------- */
+
+/* Collective over the G ranks: every rank calls it for the same bucket
+ * sequence.  Requires every local EST to have stashed `bucket` since the
+ * bucket's previous es_allreduce (ES_ESTATE otherwise).  Writes the
+ * canonical average of all N ESTs' contributions (header comment) to
+ * `out` (device, 16-byte aligned, numel elements of the bucket dtype) on
+ * every rank.  `out` may alias a BORROWed gradient of this bucket; it may
+ * not overlap the workspace.  Enqueued on `stream`; no host sync. */
+es_status es_allreduce(es_handle h, int32_t bucket, void *out, es_stream stream);
+
+/* ---- planner introspection (host-only, no CUDA) -------------------------- */
+
+/* R1 chunk size C = A*ceil(ceil(L/N)/A) (A = 0 means 16). */
+uint64_t es_chunk_elems(uint64_t L, int32_t N, uint32_t A);
+
+/* Op-list export of the plan rank cfg->rank executes for `bucket`, so that
+ * a host simulator can replay exactly what the GPU path does.  Each op is
+ * ES_OP_FIELDS int64 values (layout below).  Writes up to cap_ops ops and
+ * the total count to *n_ops; *sched_out gets the chosen es_sched (1/2; 0
+ * when G == 1). */
+#define ES_OP_FIELDS 10
+enum {
+  ES_OP_FOLD = 1,        /* [1]=lo [2]=hi [3]=e0 (-1: per-element rotation (c+1)%N) [4]=m (#ESTs)
+                            [5]=in_kind (0 none / ES_BUF_PART) [6]=in_id
+                            [7]=out_kind (ES_BUF_PART: unscaled fp32 partial /
+                                          ES_BUF_OUT: scaled, rounded) [8]=out_id              */
+  ES_OP_SEND = 2,        /* [1]=lo [2]=hi [3]=peer [4]=buf_kind [5]=buf_id                      */
+  ES_OP_RECV = 3,        /* same fields as SEND                                                 */
+  ES_OP_GROUP_BEGIN = 4,
+  ES_OP_GROUP_END = 5
+};
+enum {
+  ES_BUF_NONE = 0,
+  ES_BUF_SRC = 1,        /* local EST buf_id's contribution (slot or borrowed), bucket dtype   */
+  ES_BUF_STAGE = 2,      /* staging for remote EST buf_id's contribution, bucket dtype         */
+  ES_BUF_PART = 3,       /* fp32 partial buffer buf_id                                         */
+  ES_BUF_OUT = 4         /* the caller's output, bucket dtype                                  */
+};
+/* All [lo, hi) ranges are in bucket element coordinates. */
+es_status es_plan_ops(const es_config *cfg, int32_t bucket, int64_t *ops, size_t cap_ops,
+                      size_t *n_ops, int32_t *sched_out);
+
+/* ---- loopback transport (testing; see es_transport) ---------------------- */
+
+es_status es_loopback_create(int32_t G, void **world);
+es_status es_loopback_destroy(void *world);
+
+/* ---- instrumentation ------------------------------------------------------ */
+
+typedef enum { ES_KERNEL_STASH = 0, ES_KERNEL_FOLD = 1, ES_KERNEL_SWAP = 2, ES_KERNEL_KINDS = 3 } es_kernel_kind;
+
+/* When enabled, every kernel launch of this handle is bracketed by CUDA
+ * events on its own stream.  es_profile_query synchronises on those events
+ * and returns, per kind since the last reset: launches, summed device ms,
+ * and algorithmic bytes (reads + writes the method needs, DESIGN.md
+ * "Roofline").  Launch counts are kept even when timing is off. */
+es_status es_profile_enable(es_handle h, int32_t on);
+es_status es_profile_reset(es_handle h);
+es_status es_profile_query(es_handle h, es_kernel_kind kind, uint64_t *launches, double *ms,
+                           uint64_t *bytes);
+
+/* Test hook (T4, launch-config invariance): force the
+ * fold/stash grid size and block size; 0 restores the defaults.  Results
+ * must not change. */
+es_status es_set_launch_override(es_handle h, int32_t blocks, int32_t threads);
+
+/* ---- errors --------------------------------------------------------------- */
+
+const char *es_status_string(es_status s);
+const char *es_last_error(void);
+int32_t es_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ES_H */

@@ -1,0 +1,129 @@
+"""Torch-facing wrapper of the libes C ABI (marshalling only).
+
+``Aggregator`` is one rank's handle: it allocates the workspace with
+PyTorch's allocator (the library never calls cudaMalloc), passes tensor
+pointers and the current CUDA stream through, and keeps the host-side
+mirror of torch's Philox generator state per EST (reading R12).
+"""
+import torch
+
+from . import es
+
+DTYPES = {torch.float32: es.ES_F32, torch.bfloat16: es.ES_BF16, "f32": es.ES_F32, "bf16": es.ES_BF16,
+          es.ES_F32: es.ES_F32, es.ES_BF16: es.ES_BF16}
+TORCH_DTYPES = {es.ES_F32: torch.float32, es.ES_BF16: torch.bfloat16}
+
+
+def _stream(stream):
+    if stream is None:
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, torch.cuda.Stream):
+        return stream.cuda_stream
+    return int(stream)
+
+
+def nccl_comm_ptr(group=None):
+    """ncclComm_t of a torch ProcessGroupNCCL (after at least one collective)."""
+    import torch.distributed as dist
+    group = group or dist.group.WORLD
+    backend = group._get_backend(torch.device("cuda"))
+    return int(backend._comm_ptr())
+
+
+class Aggregator:
+    """One rank of the placement-invariant EST gradient aggregator.
+
+    buckets: list of (numel, dtype) with dtype torch.float32/bfloat16 or 'f32'/'bf16'.
+    """
+
+    def __init__(self, N, G, rank, est_to_gpu, buckets, chunk_align=16, state_nbytes=(),
+                 transport=None, comm=None, sched=es.ES_SCHED_AUTO, device=None):
+        if transport is None:
+            transport = es.ES_TRANSPORT_NONE if G == 1 else es.ES_TRANSPORT_NCCL
+        self.buckets = [(int(n), DTYPES[d]) for n, d in buckets]
+        self.cfg = es.Config(N, G, rank, est_to_gpu, self.buckets, chunk_align, tuple(state_nbytes),
+                             transport, comm, sched)
+        self.N, self.G, self.rank = N, G, rank
+        self.local_ests = [e for e in range(N) if est_to_gpu[e] == rank]
+        self.device = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+        self.ws_bytes = es.es_workspace_bytes(self.cfg)
+        self.workspace = torch.empty(max(self.ws_bytes, 256), dtype=torch.uint8, device=self.device)
+        if self.workspace.data_ptr() % 256:
+            raise RuntimeError("workspace not 256-byte aligned")
+        with torch.cuda.device(self.device):
+            self.h = es.es_init(self.cfg, self.workspace.data_ptr(), self.workspace.numel())
+        self._live = None
+        self._gen = None
+        self._philox = {}
+        self._cur = None
+
+    # ---- context state -------------------------------------------------------------
+    def register_state(self, tensors):
+        """Live per-EST context buffers (Philox record, BN running stats), in
+        the order of state_nbytes."""
+        self._live = list(tensors)
+        es.es_register_state(self.h, [t.data_ptr() for t in self._live])
+
+    def init_state(self, est, idx, data):
+        if isinstance(data, torch.Tensor):
+            data = data.detach().cpu().contiguous().view(torch.uint8).numpy().tobytes()
+        es.es_init_state(self.h, est, idx, data)
+
+    def read_state(self, est, idx):
+        return es.es_read_state(self.h, est, idx, self.cfg.state_nbytes[idx])
+
+    def attach_generator(self, gen, seeds):
+        """Keep torch generator `gen` in step with the running EST: EST k
+        starts from manual_seed(seeds[k]) with offset 0 (D0 fixed seeds,
+        PAPER.md:751-757)."""
+        self._gen = gen
+        self._philox = {k: (int(seeds[k]), 0) for k in self.local_ests}
+
+    def switch(self, est, stream=None):
+        es.es_switch_context(self.h, est, _stream(stream))
+        if self._gen is not None and est != self._cur:
+            if self._cur is not None:
+                self._philox[self._cur] = (self._gen.initial_seed(), self._gen.get_offset())
+            seed, off = self._philox[est]
+            self._gen.manual_seed(seed)
+            self._gen.set_offset(off)
+        self._cur = est
+
+    # ---- stash / aggregate ------------------------------------------------------------
+    def stash(self, est, bucket, grad, mode=es.ES_STASH_COPY, stream=None):
+        es.es_stash_grad(self.h, est, bucket, grad.data_ptr(), DTYPES[grad.dtype], mode, _stream(stream))
+
+    def allreduce(self, bucket, out, stream=None):
+        es.es_allreduce(self.h, bucket, out.data_ptr(), _stream(stream))
+        return out
+
+    def new_out(self, bucket):
+        n, d = self.buckets[bucket]
+        return torch.empty(n, dtype=TORCH_DTYPES[d], device=self.device)
+
+    def sync(self):
+        es.es_sync(self.h)
+
+    # ---- instrumentation -------------------------------------------------------------
+    def profile(self, on=True):
+        es.es_profile_enable(self.h, on)
+
+    def profile_reset(self):
+        es.es_profile_reset(self.h)
+
+    def profile_query(self, kind):
+        return es.es_profile_query(self.h, kind)
+
+    def set_launch_override(self, blocks, threads):
+        es.es_set_launch_override(self.h, blocks, threads)
+
+    def close(self):
+        if getattr(self, "h", None) is not None:
+            es.es_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

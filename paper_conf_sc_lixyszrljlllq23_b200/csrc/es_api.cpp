@@ -1,0 +1,548 @@
+// es_api.cpp -- the C ABI of libes (include/es.h): argument checking, the
+// per-rank handle, stash bookkeeping, and the executor that walks the
+// planner's op list (plan.cpp) launching kernels (kernels.cu) and transport
+// groups (transport_*.cpp) on the caller's stream.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "../../include/es.h"
+#include "kernels.h"
+#include "plan.h"
+#include "transport.h"
+
+namespace {
+
+thread_local std::string g_err;
+
+es_status set_err(es_status s, const std::string &msg) {
+  g_err = msg;
+  return s;
+}
+
+bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+// CUDA-graph support: the id of the capture `s` is part of, 0 when eager.
+// Events recorded in one capture (or eagerly) are only waited on from the
+// same capture (or eagerly): a graph cannot depend on work outside it, and
+// replays of a graph on one stream are ordered anyway.
+unsigned long long capture_id(cudaStream_t s) {
+  cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+  unsigned long long id = 0;
+  if (cudaStreamGetCaptureInfo(s, &st, &id) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  return st == cudaStreamCaptureStatusActive ? id : 0;
+}
+
+}  // namespace
+
+struct es_ctx {
+  es::Plan plan;
+  unsigned char *ws = nullptr;
+  size_t ws_bytes = 0;
+  std::unique_ptr<es::Transport> tp;
+  int device = 0;
+  int32_t B = 0, n_local = 0;
+
+  // stash bookkeeping, [local EST index * B + bucket]
+  std::vector<uint8_t> stashed;
+  std::vector<const void *> borrowed;
+  std::vector<cudaEvent_t> stash_ev;
+  std::vector<unsigned long long> stash_cap;
+  std::vector<cudaEvent_t> ar_ev;       // [B]: last es_allreduce of the bucket
+  std::vector<unsigned long long> ar_cap;
+  std::vector<uint8_t> ar_recorded;
+  cudaEvent_t last_ar = nullptr;        // orders staging / partial reuse across buckets
+  unsigned long long last_ar_cap = 0;
+
+  // context state
+  bool state_registered = false;
+  uint64_t max_state = 0;
+  int32_t cur_local = -1;
+
+  es_status sticky = ES_OK;
+  std::string sticky_msg;
+
+  // instrumentation
+  bool prof = false;
+  struct Rec {
+    int kind;
+    cudaEvent_t a, b;
+    bool captured;       // recorded by a CUDA-graph node: never recycled
+  };
+  std::vector<Rec> recs;
+  std::vector<cudaEvent_t> pool;
+  std::vector<cudaEvent_t> graph_events;
+  uint64_t launches[ES_KERNEL_KINDS] = {0, 0, 0};
+  uint64_t bytes[ES_KERNEL_KINDS] = {0, 0, 0};
+  double ms[ES_KERNEL_KINDS] = {0, 0, 0};
+  int blocks_ov = 0, threads_ov = 0;
+
+  ~es_ctx() {
+    for (auto e : stash_ev) if (e) cudaEventDestroy(e);
+    for (auto e : ar_ev) if (e) cudaEventDestroy(e);
+    for (auto &r : recs) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
+    for (auto e : pool) cudaEventDestroy(e);
+    for (auto e : graph_events) cudaEventDestroy(e);
+  }
+  cudaEvent_t ev() {
+    if (!pool.empty()) {
+      cudaEvent_t e = pool.back();
+      pool.pop_back();
+      return e;
+    }
+    cudaEvent_t e = nullptr;
+    cudaEventCreate(&e);
+    return e;
+  }
+  es_status poison(es_status s, const std::string &msg) {
+    if (sticky == ES_OK) {
+      sticky = s;
+      sticky_msg = msg;
+    }
+    return set_err(s, msg);
+  }
+  es_status check_sticky() {
+    if (sticky != ES_OK) return set_err(sticky, "handle poisoned by an earlier error: " + sticky_msg);
+    return ES_OK;
+  }
+  // Runs `launch` bracketed by timing events when profiling is on.
+  template <typename F>
+  es_status timed(int kind, uint64_t nbytes, cudaStream_t s, F launch) {
+    cudaEvent_t a = nullptr, b = nullptr;
+    // Inside a graph capture the timing events become event-record nodes.
+    const bool cap = capture_id(s) != 0;
+    const unsigned int flags = cap ? cudaEventRecordExternal : cudaEventRecordDefault;
+    if (prof) {
+      a = ev();
+      b = ev();
+      cudaEventRecordWithFlags(a, s, flags);
+    }
+    cudaError_t e = launch();
+    if (e != cudaSuccess) return poison(ES_ECUDA, std::string("kernel launch: ") + cudaGetErrorString(e));
+    if (prof) {
+      cudaEventRecordWithFlags(b, s, flags);
+      recs.push_back({kind, a, b, cap});
+    }
+    launches[kind]++;
+    bytes[kind] += nbytes;
+    return ES_OK;
+  }
+};
+
+namespace {
+
+es_status check_handle(es_handle h) {
+  if (!h) return set_err(ES_EINVAL, "handle is NULL");
+  return h->check_sticky();
+}
+
+}  // namespace
+
+extern "C" {
+
+int32_t es_abi_version(void) { return ES_ABI_VERSION; }
+
+const char *es_status_string(es_status s) {
+  switch (s) {
+    case ES_OK: return "ES_OK";
+    case ES_EINVAL: return "ES_EINVAL: invalid argument";
+    case ES_ESTATE: return "ES_ESTATE: protocol violation";
+    case ES_ENOMEM: return "ES_ENOMEM: workspace too small";
+    case ES_ECUDA: return "ES_ECUDA: CUDA error";
+    case ES_ENCCL: return "ES_ENCCL: NCCL error";
+    case ES_EUNSUPPORTED: return "ES_EUNSUPPORTED: unsupported";
+  }
+  return "unknown es_status";
+}
+
+const char *es_last_error(void) { return g_err.c_str(); }
+
+uint64_t es_chunk_elems(uint64_t L, int32_t N, uint32_t A) { return es::chunk_elems(L, N, A ? A : 16); }
+
+es_status es_workspace_bytes(const es_config *cfg, size_t *bytes) {
+  if (!bytes) return set_err(ES_EINVAL, "bytes is NULL");
+  es::Plan p;
+  std::string err;
+  es_status s = es::build_plan(cfg, &p, &err, false);
+  if (s != ES_OK) return set_err(s, err);
+  *bytes = p.total;
+  return ES_OK;
+}
+
+es_status es_plan_ops(const es_config *cfg, int32_t bucket, int64_t *ops, size_t cap_ops, size_t *n_ops,
+                      int32_t *sched_out) {
+  if (!n_ops) return set_err(ES_EINVAL, "n_ops is NULL");
+  es::Plan p;
+  std::string err;
+  es_status s = es::build_plan(cfg, &p, &err, false);
+  if (s != ES_OK) return set_err(s, err);
+  if (bucket < 0 || bucket >= (int32_t)p.bp.size()) return set_err(ES_EINVAL, "bucket out of range");
+  const es::BucketPlan &b = p.bp[bucket];
+  *n_ops = b.ops.size();
+  if (sched_out) *sched_out = b.sched;
+  if (ops)
+    for (size_t i = 0; i < b.ops.size() && i < cap_ops; ++i)
+      std::memcpy(ops + i * ES_OP_FIELDS, b.ops[i].f, sizeof(int64_t) * ES_OP_FIELDS);
+  return ES_OK;
+}
+
+es_status es_init(const es_config *cfg, void *workspace, size_t workspace_bytes, es_handle *out) {
+  if (!out) return set_err(ES_EINVAL, "out is NULL");
+  *out = nullptr;
+  std::unique_ptr<es_ctx> h(new es_ctx());
+  std::string err;
+  es_status s = es::build_plan(cfg, &h->plan, &err);
+  if (s != ES_OK) return set_err(s, err);
+  if (!workspace || (reinterpret_cast<uintptr_t>(workspace) & 255u))
+    return set_err(ES_EINVAL, "workspace must be a non-NULL 256-byte aligned device pointer");
+  if (workspace_bytes < h->plan.total)
+    return set_err(ES_ENOMEM, "workspace smaller than es_workspace_bytes()");
+  cudaPointerAttributes attr;
+  if (cudaPointerGetAttributes(&attr, workspace) != cudaSuccess || attr.type != cudaMemoryTypeDevice) {
+    cudaGetLastError();
+    return set_err(ES_EINVAL, "workspace is not device memory");
+  }
+  if (cudaGetDevice(&h->device) != cudaSuccess) return set_err(ES_ECUDA, "cudaGetDevice failed");
+  h->ws = reinterpret_cast<unsigned char *>(workspace);
+  h->ws_bytes = workspace_bytes;
+  h->B = (int32_t)h->plan.bp.size();
+  h->n_local = (int32_t)h->plan.local_ests.size();
+  const size_t nslot = (size_t)h->B * h->n_local;
+  h->stashed.assign(nslot, 0);
+  h->borrowed.assign(nslot, nullptr);
+  h->stash_ev.assign(nslot, nullptr);
+  h->stash_cap.assign(nslot, 0);
+  h->ar_ev.assign(h->B, nullptr);
+  h->ar_cap.assign(h->B, 0);
+  h->ar_recorded.assign(h->B, 0);
+  for (auto &e : h->stash_ev)
+    if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
+      return set_err(ES_ECUDA, "cudaEventCreate failed");
+  for (auto &e : h->ar_ev)
+    if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
+      return set_err(ES_ECUDA, "cudaEventCreate failed");
+  for (uint64_t n : h->plan.state_nbytes) h->max_state = std::max<uint64_t>(h->max_state, n);
+  if (h->plan.G > 1) {
+    es::Transport *t = h->plan.transport == ES_TRANSPORT_NCCL
+                           ? es::make_nccl_transport(h->plan.comm, h->plan.G, h->plan.rank, &err)
+                           : es::make_loopback_transport(h->plan.comm, h->plan.G, h->plan.rank, &err);
+    if (!t) return set_err(h->plan.transport == ES_TRANSPORT_NCCL ? ES_ENCCL : ES_EINVAL, err);
+    h->tp.reset(t);
+  }
+  *out = h.release();
+  return ES_OK;
+}
+
+es_status es_destroy(es_handle h) {
+  if (!h) return set_err(ES_EINVAL, "handle is NULL");
+  delete h;
+  return ES_OK;
+}
+
+es_status es_sync(es_handle h) {
+  if (!h) return set_err(ES_EINVAL, "handle is NULL");
+  es_status s = h->check_sticky();
+  if (s != ES_OK) return s;
+  cudaError_t e = cudaDeviceSynchronize();
+  if (e == cudaSuccess) e = cudaGetLastError();
+  if (e != cudaSuccess) return h->poison(ES_ECUDA, std::string("asynchronous CUDA error: ") + cudaGetErrorString(e));
+  return ES_OK;
+}
+
+// ---- context state ----------------------------------------------------------
+
+es_status es_register_state(es_handle h, int32_t n, void *const *live) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  const es::Plan &p = h->plan;
+  if (n != (int32_t)p.state_nbytes.size()) return set_err(ES_EINVAL, "n must equal cfg.n_state");
+  if (n > 0 && !live) return set_err(ES_EINVAL, "live_dev_ptrs is NULL");
+  std::vector<es::SwapEntry> tab(n);
+  for (int32_t i = 0; i < n; ++i) {
+    if (!live[i] || !aligned16(live[i])) return set_err(ES_EINVAL, "live state pointers must be 16-byte aligned");
+    tab[i].live = reinterpret_cast<unsigned char *>(live[i]);
+    tab[i].slot0 = h->ws + p.state_area_off + p.state_off[i];
+    tab[i].stride = p.state_block;
+    tab[i].nbytes = p.state_nbytes[i];
+  }
+  if (n > 0 && cudaMemcpy(h->ws + p.table_off, tab.data(), sizeof(es::SwapEntry) * n, cudaMemcpyHostToDevice) !=
+                   cudaSuccess)
+    return h->poison(ES_ECUDA, "cudaMemcpy of the swap table failed");
+  h->state_registered = true;
+  return ES_OK;
+}
+
+static es_status state_slot(es_handle h, int32_t est, int32_t idx, unsigned char **ptr, uint64_t *nbytes) {
+  const es::Plan &p = h->plan;
+  if (est < 0 || est >= p.N) return set_err(ES_EINVAL, "est out of range");
+  if (idx < 0 || idx >= (int32_t)p.state_nbytes.size()) return set_err(ES_EINVAL, "state idx out of range");
+  int32_t li = p.local_index[est];
+  if (li < 0) return set_err(ES_ESTATE, "est is not mapped to this rank");
+  *ptr = h->ws + p.state_area_off + (uint64_t)li * p.state_block + p.state_off[idx];
+  *nbytes = p.state_nbytes[idx];
+  return ES_OK;
+}
+
+es_status es_init_state(es_handle h, int32_t est, int32_t idx, const void *host_src) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  if (!host_src) return set_err(ES_EINVAL, "host_src is NULL");
+  unsigned char *d;
+  uint64_t nb;
+  if ((s = state_slot(h, est, idx, &d, &nb)) != ES_OK) return s;
+  if (cudaMemcpy(d, host_src, nb, cudaMemcpyHostToDevice) != cudaSuccess)
+    return h->poison(ES_ECUDA, "cudaMemcpy H2D of EST state failed");
+  return ES_OK;
+}
+
+es_status es_read_state(es_handle h, int32_t est, int32_t idx, void *host_dst) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  if (!host_dst) return set_err(ES_EINVAL, "host_dst is NULL");
+  unsigned char *d;
+  uint64_t nb;
+  if ((s = state_slot(h, est, idx, &d, &nb)) != ES_OK) return s;
+  if (cudaMemcpy(host_dst, d, nb, cudaMemcpyDeviceToHost) != cudaSuccess)
+    return h->poison(ES_ECUDA, "cudaMemcpy D2H of EST state failed");
+  return ES_OK;
+}
+
+es_status es_switch_context(es_handle h, int32_t est, es_stream stream) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  const es::Plan &p = h->plan;
+  if (est < 0 || est >= p.N) return set_err(ES_EINVAL, "est out of range");
+  int32_t li = p.local_index[est];
+  if (li < 0) return set_err(ES_ESTATE, "est is not mapped to this rank");
+  const int32_t n = (int32_t)p.state_nbytes.size();
+  if (n > 0 && !h->state_registered) return set_err(ES_ESTATE, "es_register_state has not been called");
+  if (li == h->cur_local) return ES_OK;
+  if (n > 0) {
+    uint64_t tot = 0;
+    for (uint64_t b : p.state_nbytes) tot += b;
+    cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
+    const int32_t cur = h->cur_local;
+    const auto *tab = reinterpret_cast<const es::SwapEntry *>(h->ws + p.table_off);
+    s = h->timed(ES_KERNEL_SWAP, (cur >= 0 ? 4 : 2) * tot, cs,
+                 [&] { return es::launch_swap(tab, n, h->max_state, cur, li, cs); });
+    if (s != ES_OK) return s;
+  }
+  h->cur_local = li;
+  return ES_OK;
+}
+
+// ---- stash ----------------------------------------------------------------------
+
+es_status es_stash_grad(es_handle h, int32_t est, int32_t bucket, const void *grad, es_dtype gdt, es_stash_mode mode,
+                        es_stream stream) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  const es::Plan &p = h->plan;
+  if (est < 0 || est >= p.N) return set_err(ES_EINVAL, "est out of range");
+  if (bucket < 0 || bucket >= h->B) return set_err(ES_EINVAL, "bucket out of range");
+  if (gdt != ES_F32 && gdt != ES_BF16) return set_err(ES_EINVAL, "bad grad dtype");
+  if (mode != ES_STASH_COPY && mode != ES_STASH_BORROW) return set_err(ES_EINVAL, "bad stash mode");
+  const es::BucketPlan &b = p.bp[bucket];
+  if (b.L > 0 && (!grad || !aligned16(grad))) return set_err(ES_EINVAL, "grad must be a 16-byte aligned device pointer");
+  if (mode == ES_STASH_BORROW && gdt != b.dtype) return set_err(ES_EINVAL, "BORROW needs grad dtype == bucket dtype");
+  int32_t li = p.local_index[est];
+  if (li < 0) return set_err(ES_ESTATE, "est is not mapped to this rank");
+  cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
+  const size_t k = (size_t)li * h->B + bucket;
+  if (mode == ES_STASH_COPY) {
+    unsigned char *slot = h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[bucket];
+    if (h->ar_recorded[bucket] && h->ar_cap[bucket] == capture_id(cs) &&
+        cudaStreamWaitEvent(cs, h->ar_ev[bucket], 0) != cudaSuccess)
+      return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
+    const uint64_t nbytes = b.L * (es::dtype_size(gdt) + b.esize);
+    s = h->timed(ES_KERNEL_STASH, nbytes, cs, [&] {
+      return es::launch_stash(grad, gdt, slot, b.dtype, (int64_t)b.L, cs, h->blocks_ov, h->threads_ov);
+    });
+    if (s != ES_OK) return s;
+    h->borrowed[k] = nullptr;
+  } else {
+    h->borrowed[k] = grad;
+  }
+  if (cudaEventRecord(h->stash_ev[k], cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaEventRecord failed");
+  h->stash_cap[k] = capture_id(cs);
+  h->stashed[k] = 1;
+  return ES_OK;
+}
+
+// ---- aggregation --------------------------------------------------------------------
+
+es_status es_allreduce(es_handle h, int32_t bucket, void *out, es_stream stream) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  const es::Plan &p = h->plan;
+  if (bucket < 0 || bucket >= h->B) return set_err(ES_EINVAL, "bucket out of range");
+  const es::BucketPlan &b = p.bp[bucket];
+  const uint64_t out_bytes = b.L * b.esize;
+  if (b.L > 0) {
+    if (!out || !aligned16(out)) return set_err(ES_EINVAL, "out must be a 16-byte aligned device pointer");
+    const unsigned char *o = reinterpret_cast<const unsigned char *>(out);
+    if (o < h->ws + h->ws_bytes && h->ws < o + out_bytes) return set_err(ES_EINVAL, "out overlaps the workspace");
+  }
+  for (int32_t li = 0; li < h->n_local; ++li)
+    if (!h->stashed[(size_t)li * h->B + bucket])
+      return set_err(ES_ESTATE, "es_allreduce before every local EST stashed this bucket");
+  cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
+  const unsigned long long cap = capture_id(cs);
+  for (int32_t li = 0; li < h->n_local; ++li) {
+    const size_t k = (size_t)li * h->B + bucket;
+    if (h->stash_cap[k] == cap && cudaStreamWaitEvent(cs, h->stash_ev[k], 0) != cudaSuccess)
+      return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
+  }
+  if (h->last_ar && h->last_ar_cap == cap && cudaStreamWaitEvent(cs, h->last_ar, 0) != cudaSuccess)
+    return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
+
+  const uint32_t es_ = b.esize;
+  auto src_base = [&](int32_t e) -> unsigned char * {   // element 0 of EST e's contribution
+    int32_t li = p.local_index[e];
+    const void *bw = h->borrowed[(size_t)li * h->B + bucket];
+    if (bw) return reinterpret_cast<unsigned char *>(const_cast<void *>(bw));
+    return h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[bucket];
+  };
+  auto contrib_at = [&](int32_t e, int64_t lo) -> unsigned char * {
+    if (p.local_index[e] >= 0) return src_base(e) + (uint64_t)lo * es_;
+    return h->ws + p.stage_off + (uint64_t)b.stage_index[e] * b.stage_stride + (uint64_t)(lo - b.shard_lo) * es_;
+  };
+  auto part_at = [&](int64_t id, int64_t lo) -> unsigned char * {
+    const es::Part &pt = b.parts[id];
+    return h->ws + p.parts_off + pt.off + (uint64_t)(lo - pt.lo) * 4;
+  };
+  unsigned char *outp = reinterpret_cast<unsigned char *>(out);
+  const float r = 1.0f / (float)p.N;   // R5: fl32(1/N), correctly rounded fp32 division
+  std::vector<const void *> srcs(p.N);
+
+  for (const es::Op &op : b.ops) {
+    const int64_t *f = op.f;
+    switch (f[0]) {
+      case ES_OP_FOLD: {
+        const int64_t lo = f[1], hi = f[2];
+        es::FoldDesc d;
+        d.lo = lo;
+        d.n = hi - lo;
+        d.N = p.N;
+        d.C = (uint32_t)b.C;
+        d.r = r;
+        int nsrc;
+        if (f[3] < 0) {
+          d.rot = true;
+          nsrc = p.N;
+          for (int32_t e = 0; e < p.N; ++e) srcs[e] = contrib_at(e, lo);
+        } else {
+          d.rot = false;
+          d.m = (int32_t)f[4];
+          nsrc = d.m;
+          for (int32_t t = 0; t < d.m; ++t) srcs[t] = contrib_at((int32_t)((f[3] + t) % p.N), lo);
+        }
+        d.part_in = f[5] == ES_BUF_PART ? reinterpret_cast<const float *>(part_at(f[6], lo)) : nullptr;
+        d.out_partial = f[7] == ES_BUF_PART;
+        d.out = d.out_partial ? (void *)part_at(f[8], lo) : (void *)(outp + (uint64_t)lo * es_);
+        const uint64_t nb = (uint64_t)d.n * ((uint64_t)nsrc * es_ + (d.part_in ? 4 : 0) + (d.out_partial ? 4 : es_));
+        s = h->timed(ES_KERNEL_FOLD, nb, cs, [&] {
+          return es::launch_fold(b.dtype, d, srcs.data(), cs, h->blocks_ov, h->threads_ov);
+        });
+        if (s != ES_OK) return s;
+        break;
+      }
+      case ES_OP_GROUP_BEGIN:
+        if ((s = h->tp->group_begin()) != ES_OK) return h->poison(s, h->tp->err);
+        break;
+      case ES_OP_GROUP_END:
+        if ((s = h->tp->group_end(cs)) != ES_OK) return h->poison(s, h->tp->err);
+        break;
+      case ES_OP_SEND:
+      case ES_OP_RECV: {
+        const int64_t lo = f[1], hi = f[2];
+        const int peer = (int)f[3];
+        unsigned char *ptr = nullptr;
+        uint64_t w = es_;
+        switch (f[4]) {
+          case ES_BUF_SRC: ptr = contrib_at((int32_t)f[5], lo); break;
+          case ES_BUF_STAGE: ptr = contrib_at((int32_t)f[5], lo); break;
+          case ES_BUF_PART: ptr = part_at(f[5], lo); w = 4; break;
+          case ES_BUF_OUT: ptr = outp + (uint64_t)lo * es_; break;
+          default: return h->poison(ES_ESTATE, "corrupt plan: bad buffer kind");
+        }
+        const size_t nbytes = (size_t)(hi - lo) * w;
+        s = f[0] == ES_OP_SEND ? h->tp->send(ptr, nbytes, peer) : h->tp->recv(ptr, nbytes, peer);
+        if (s != ES_OK) return h->poison(s, h->tp->err);
+        break;
+      }
+      default:
+        return h->poison(ES_ESTATE, "corrupt plan: bad opcode");
+    }
+  }
+  if (cudaEventRecord(h->ar_ev[bucket], cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaEventRecord failed");
+  h->ar_recorded[bucket] = 1;
+  h->ar_cap[bucket] = cap;
+  h->last_ar = h->ar_ev[bucket];
+  h->last_ar_cap = cap;
+  for (int32_t li = 0; li < h->n_local; ++li) {
+    h->stashed[(size_t)li * h->B + bucket] = 0;
+    h->borrowed[(size_t)li * h->B + bucket] = nullptr;
+  }
+  return ES_OK;
+}
+
+// ---- instrumentation ---------------------------------------------------------
+
+es_status es_profile_enable(es_handle h, int32_t on) {
+  if (!h) return set_err(ES_EINVAL, "handle is NULL");
+  h->prof = on != 0;
+  return ES_OK;
+}
+
+static void drain(es_handle h) {
+  for (auto &r : h->recs) {
+    float t = 0.f;
+    cudaEventSynchronize(r.b);
+    cudaEventElapsedTime(&t, r.a, r.b);
+    h->ms[r.kind] += t;
+    std::vector<cudaEvent_t> &dst = r.captured ? h->graph_events : h->pool;
+    dst.push_back(r.a);
+    dst.push_back(r.b);
+  }
+  h->recs.clear();
+}
+
+es_status es_profile_reset(es_handle h) {
+  if (!h) return set_err(ES_EINVAL, "handle is NULL");
+  drain(h);
+  for (int k = 0; k < ES_KERNEL_KINDS; ++k) {
+    h->launches[k] = 0;
+    h->bytes[k] = 0;
+    h->ms[k] = 0;
+  }
+  return ES_OK;
+}
+
+es_status es_profile_query(es_handle h, es_kernel_kind kind, uint64_t *launches, double *ms, uint64_t *bytes) {
+  if (!h) return set_err(ES_EINVAL, "handle is NULL");
+  if (kind < 0 || kind >= ES_KERNEL_KINDS) return set_err(ES_EINVAL, "bad kernel kind");
+  drain(h);
+  if (launches) *launches = h->launches[kind];
+  if (ms) *ms = h->ms[kind];
+  if (bytes) *bytes = h->bytes[kind];
+  return ES_OK;
+}
+
+es_status es_set_launch_override(es_handle h, int32_t blocks, int32_t threads) {
+  if (!h) return set_err(ES_EINVAL, "handle is NULL");
+  if (blocks < 0 || threads < 0 || threads > 256 || (threads % 32) != 0)
+    return set_err(ES_EINVAL, "threads must be a multiple of 32 in [0, 256]; blocks >= 0");
+  h->blocks_ov = blocks;
+  h->threads_ov = threads;
+  return ES_OK;
+}
+
+}  // extern "C"

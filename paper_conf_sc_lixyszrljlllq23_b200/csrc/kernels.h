@@ -1,0 +1,57 @@
+// kernels.h -- launchers of the sm_100a kernels of libes (internal).
+#pragma once
+
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "../../include/es.h"
+
+namespace es {
+
+// Canonical fold over the bucket
+// elements [lo, lo+n).  Every pointer below points at element `lo` of its
+// buffer (physical pointers, 16-byte aligned); lo must be a multiple of 8
+// so that no 16-byte vector straddles a chunk (R1 with A % 8 == 0).
+//   rot == true : per-element canonical rotation -- element i = lo+t lies in
+//                 chunk c = i / C and is folded over src[(c+1)%N], ...,
+//                 src[(c+N)%N]  (src holds N entries indexed by EST)
+//   rot == false: sources src[0], ..., src[m-1] in that order (one chain
+//                 segment; src already in canonical order)
+//   part_in     : if non-null, the fold continues from this unrounded fp32
+//                 partial instead of starting from its first source
+//   out_partial : write the unrounded fp32 sum to `out` (fp32); otherwise
+//                 write round_dtype(fl32(s * r)) to `out` (bucket dtype).
+struct FoldDesc {
+  int64_t lo = 0, n = 0;
+  int32_t N = 1;
+  bool rot = true;
+  int32_t m = 0;
+  uint32_t C = 1;
+  const float *part_in = nullptr;
+  void *out = nullptr;
+  bool out_partial = false;
+  float r = 1.0f;
+};
+
+// src: host array of source pointers (N entries if rot, m otherwise).
+cudaError_t launch_fold(es_dtype dtype, const FoldDesc &d, const void *const *src, cudaStream_t s,
+                        int blocks_override, int threads_override);
+
+// Stash: dst[i] = cast(src[i]) for i < n.
+cudaError_t launch_stash(const void *src, es_dtype sdt, void *dst, es_dtype ddt, int64_t n,
+                         cudaStream_t s, int blocks_override, int threads_override);
+
+// Context-switch swap table entry.
+struct SwapEntry {
+  unsigned char *live;   // live buffer (16-byte aligned)
+  unsigned char *slot0;  // saved copy of local EST 0; local EST k at slot0 + k*stride
+  uint64_t stride;
+  uint64_t nbytes;
+};
+
+// One launch: for every entry, slot[cur] <- live, live <- slot[next]
+// (cur < 0: load only).  max_nbytes sizes the grid.
+cudaError_t launch_swap(const SwapEntry *table_dev, int32_t n, uint64_t max_nbytes, int32_t cur,
+                        int32_t next, cudaStream_t s);
+
+}  // namespace es

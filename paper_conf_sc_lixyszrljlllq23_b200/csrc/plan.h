@@ -1,0 +1,82 @@
+// plan.h -- host planner of libes ("canonical plan").
+//
+// Everything the GPU path does for a bucket is decided here, once, at
+// es_init, from (N, G, rank, EST->GPU mapping, bucket layout, A) only:
+// the R1 chunk table, the element shards, the exchange schedule and the
+// exact op list each rank executes.  The plan is never rebuilt while the
+// handle lives -- the D1 rule "reconstruction of the communication channel
+// is disabled".
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/es.h"
+
+namespace es {
+
+struct Op {
+  int64_t f[ES_OP_FIELDS];
+};
+
+// fp32 partial buffer: bucket element range [lo, hi) at byte offset `off`
+// of the partials area.
+struct Part {
+  int64_t lo, hi;
+  uint64_t off;
+};
+
+struct BucketPlan {
+  uint64_t L = 0;
+  es_dtype dtype = ES_F32;
+  uint32_t esize = 4;            // bytes per element of the bucket dtype
+  uint64_t C = 0;                // R1 chunk size
+  int32_t sched = 0;             // 0: G == 1, ES_SCHED_DIRECT, ES_SCHED_CHAIN
+  int64_t shard_lo = 0, shard_hi = 0;   // DIRECT: this rank's shard
+  std::vector<int32_t> stage_index;     // [N]: staging slot of remote EST, -1 if local/unused
+  uint64_t stage_stride = 0;            // bytes per staging slot
+  uint64_t stage_bytes = 0;
+  std::vector<Part> parts;
+  uint64_t part_bytes = 0;
+  std::vector<Op> ops;
+};
+
+struct Plan {
+  int32_t N = 0, G = 0, rank = 0;
+  uint32_t A = 16;
+  std::vector<int32_t> est_to_gpu;
+  std::vector<int32_t> local_ests;      // ascending
+  std::vector<int32_t> local_index;     // [N] -> index into local_ests, -1 if remote
+  std::vector<es_bucket_desc> buckets;
+  std::vector<uint64_t> state_nbytes;
+  es_transport transport = ES_TRANSPORT_NONE;
+  void *comm = nullptr;
+  es_sched sched_req = ES_SCHED_AUTO;
+  std::vector<BucketPlan> bp;
+
+  // Workspace layout (byte offsets from the workspace base, 256-aligned).
+  std::vector<uint64_t> slot_off;       // [n_buckets]: offset inside one EST's gradient block
+  uint64_t slot_block = 0;              // bytes of one EST's gradient block
+  uint64_t grad_off = 0;                // n_local gradient blocks
+  std::vector<uint64_t> state_off;      // [n_state]: offset inside one EST's state block
+  uint64_t state_block = 0;
+  uint64_t state_area_off = 0;          // n_local state blocks
+  uint64_t table_off = 0;               // swap table (n_state entries)
+  uint64_t stage_off = 0;               // exchange staging (max over buckets)
+  uint64_t parts_off = 0;               // chain partials (max over buckets)
+  uint64_t total = 0;
+};
+
+inline uint64_t align256(uint64_t x) { return (x + 255) & ~uint64_t(255); }
+inline uint32_t dtype_size(es_dtype d) { return d == ES_BF16 ? 2u : 4u; }
+
+// R1: C = A * ceil(ceil(L / N) / A).
+uint64_t chunk_elems(uint64_t L, int32_t N, uint32_t A);
+
+// Validates cfg and builds the full plan for cfg->rank.  On failure returns
+// ES_EINVAL and sets *err.
+// need_comm == false (host-only queries) skips the transport/comm checks.
+es_status build_plan(const es_config *cfg, Plan *plan, std::string *err, bool need_comm = true);
+
+}  // namespace es

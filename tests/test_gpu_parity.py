@@ -1,0 +1,264 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle,
+bit for bit (readings R1-R7; north star: "The GPU result must match the
+oracle bit-exactly").  Sizes span several tiles and ragged tails; the
+full-size sampled checks run in the launch configuration bench.py times."""
+import json
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from paper_conf_sc_lixyszrljlllq23_b200 import es, workloads
+
+from gpu_util import assert_bits_equal, reduce_g1, reduce_loopback
+
+pytestmark = pytest.mark.gpu
+
+
+def _bf16(x32):
+    return oracle.f32_to_bf16_bits(np.asarray(x32, np.float32))
+
+
+def _gauss(rng, N, L, dtype="f32", sigma=1e-3):
+    mu = rng.standard_normal(L) * sigma
+    xs = [(mu + rng.standard_normal(L) * sigma).astype(np.float32) for _ in range(N)]
+    return xs if dtype == "f32" else [_bf16(x) for x in xs]
+
+
+# ---- G = 1 -----------------------------------------------------------------------------------
+
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+@pytest.mark.parametrize("N", [1, 2, 3, 4, 8, 12, 16, 32, 33, 129])
+def test_fold_g1_matches_oracle(N, dtype):
+    rng = np.random.default_rng(N * 7 + (dtype == "bf16"))
+    Ls = [100003, 16, 17, 1, 4099]                   # several tiles + ragged tails
+    xs = [_gauss(rng, N, L, dtype) for L in Ls]
+    outs = reduce_g1(xs)
+    for b, L in enumerate(Ls):
+        assert_bits_equal(outs[b], oracle.reduce(xs[b], dtype), f"N={N} L={L} {dtype}")
+
+
+@pytest.mark.parametrize("L", [0, 1, 15, 16, 17, 1000003])
+def test_fold_g1_tails(L):
+    rng = np.random.default_rng(L)
+    for dtype in ["f32", "bf16"]:
+        xs = _gauss(rng, 4, max(L, 1), dtype)
+        if L == 0:
+            xs = [x[:0] for x in xs]
+        out = reduce_g1([xs])[0]
+        assert_bits_equal(out, oracle.reduce(xs, dtype), f"L={L} {dtype}")
+
+
+@pytest.mark.parametrize("A", [8, 16, 64, 4096])
+def test_fold_g1_chunk_align(A):
+    rng = np.random.default_rng(A)
+    xs = _gauss(rng, 7, 50001)
+    assert_bits_equal(reduce_g1([xs], A=A)[0], oracle.reduce(xs, "f32", A=A), f"A={A}")
+
+
+def test_golden_witnesses_on_gpu(golden_dir):
+    g = json.load(open(os.path.join(golden_dir, "witness_n4.json")))
+    for case in g["cases"]:
+        xs = [np.full(g["L"], np.float32(float.fromhex(v) if "0x" in v else float(v)), np.float32) for v in case["x"]]
+        assert_bits_equal(reduce_g1([xs], A=g["A"])[0], oracle.reduce(xs, "f32", A=g["A"]), case["name"])
+    b = json.load(open(os.path.join(golden_dir, "bf16_accumulate.json")))
+    xs = [_bf16(np.full(b["L"], np.float32(float.fromhex(v) if "0x" in v else float(v)))) for v in b["x"]]
+    out = reduce_g1([xs], A=b["A"])[0]
+    assert np.all(oracle.bf16_bits_to_f32(out) == np.float32(float(b["out"])))
+
+
+def test_special_values_on_gpu():
+    t = np.float32(2.0 ** -149)
+    cases = [
+        [np.full(64, -0.0, np.float32)] * 4,                                    # R3 signed zero
+        [np.full(64, 2 * t, np.float32), np.full(64, 4 * t, np.float32)],      # subnormals (no FTZ)
+        [np.full(64, 1.0, np.float32), np.full(64, np.nan, np.float32), np.full(64, 2.0, np.float32)],
+        [np.full(64, np.inf, np.float32), np.full(64, -np.inf, np.float32)],
+        [np.array([0.0, -0.0, 1.5, np.inf, -np.inf, 1e-45, 3.4e38, np.nan] * 8, np.float32)],  # N = 1 identity
+    ]
+    for xs in cases:
+        assert_bits_equal(reduce_g1([xs])[0], oracle.reduce(xs, "f32"))
+        xb = [_bf16(x) for x in xs]
+        assert_bits_equal(reduce_g1([xb])[0], oracle.reduce(xb, "bf16"))
+
+
+def test_wide_dynamic_range():
+    rng = np.random.default_rng(99)
+    N, L = 12, 70001
+    xs = [(rng.choice([-1, 1], L) * 2.0 ** rng.uniform(-20, 20, L)).astype(np.float32) for _ in range(N)]
+    assert_bits_equal(reduce_g1([xs])[0], oracle.reduce(xs, "f32"))
+
+
+def test_launch_config_invariance():
+    """T4 / D2 analogue: grid and block size never change bits."""
+    rng = np.random.default_rng(4)
+    xs_f = _gauss(rng, 12, 123457)
+    xs_b = _gauss(rng, 12, 123457, "bf16")
+    ref_f, ref_b = oracle.reduce(xs_f, "f32"), oracle.reduce(xs_b, "bf16")
+    for ov in [(1, 32), (1, 256), (3, 64), (148, 128), (1184, 256), (7, 96), (0, 0)]:
+        out = reduce_g1([xs_f, xs_b], override=ov)
+        assert_bits_equal(out[0], ref_f, f"override {ov}")
+        assert_bits_equal(out[1], ref_b, f"override {ov}")
+
+
+def test_repeatability_d0():
+    """D0: repeated runs give identical bits."""
+    rng = np.random.default_rng(5)
+    xs = _gauss(rng, 8, 300001)
+    runs = reduce_g1([xs], repeat=10)
+    for r in runs[1:]:
+        assert_bits_equal(r[0], runs[0][0])
+    assert_bits_equal(runs[0][0], oracle.reduce(xs, "f32"))
+
+
+def test_layout_dependence_negative():
+    """D0 failure mode: a different bucket layout (here a
+    different chunk alignment, part of the persisted layout) changes bits --
+    the suite detects layout dependence."""
+    rng = np.random.default_rng(6)
+    xs = _gauss(rng, 8, 200003)
+    a = reduce_g1([xs], A=16)[0]
+    b = reduce_g1([xs], A=1024)[0]
+    assert not np.array_equal(a.view(np.uint32), b.view(np.uint32))
+
+
+# ---- stash -------------------------------------------------------------------------------
+
+@pytest.mark.parametrize("src,dst", [("f32", "f32"), ("f32", "bf16"), ("bf16", "f32"), ("bf16", "bf16")])
+def test_stash_cast_parity(src, dst):
+    """Stash = cast (RNE narrowing, exact widening) then fold: the fold of
+    the cast slots must equal the oracle's fold of the oracle's cast."""
+    rng = np.random.default_rng(8)
+    N, L = 5, 65541
+    base = _gauss(rng, N, L, src, sigma=10.0)
+    oracle_slots = [oracle.stash(x, src, dst) for x in base]
+    # hand the kernel `src`-typed gradients for a `dst` bucket
+    from gpu_util import Aggregator, to_dev, from_dev
+    agg = Aggregator(N, 1, 0, [0] * N, [(L, dst)])
+    devs = [to_dev(x) for x in base]
+    for k in range(N):
+        agg.stash(k, 0, devs[k], es.ES_STASH_COPY)
+    o = agg.new_out(0)
+    agg.allreduce(0, o)
+    torch.cuda.synchronize()
+    agg.sync()
+    assert_bits_equal(from_dev(o), oracle.reduce(oracle_slots, dst), f"{src}->{dst}")
+    agg.close()
+
+
+def test_borrow_equals_copy_and_out_aliasing():
+    rng = np.random.default_rng(9)
+    xs = _gauss(rng, 6, 77777)
+    want = oracle.reduce(xs, "f32")
+    assert_bits_equal(reduce_g1([xs], borrow_last=False)[0], want)
+    assert_bits_equal(reduce_g1([xs], borrow_last=True)[0], want)
+    # out aliases the borrowed buffer of the last EST (in-place)
+    from gpu_util import Aggregator, to_dev, from_dev
+    agg = Aggregator(6, 1, 0, [0] * 6, [(77777, "f32")])
+    devs = [to_dev(x) for x in xs]
+    for k in range(5):
+        agg.stash(k, 0, devs[k])
+    agg.stash(5, 0, devs[5], es.ES_STASH_BORROW)
+    agg.allreduce(0, devs[5])
+    torch.cuda.synchronize()
+    assert_bits_equal(from_dev(devs[5]), want)
+    agg.close()
+
+
+# ---- G > 1 over the loopback transport (one GPU, every mapping) ------------------------------
+
+def _surjections(N, G):
+    import itertools
+    for m in itertools.product(range(G), repeat=N):
+        if len(set(m)) == G:
+            yield list(m)
+
+
+@pytest.mark.parametrize("G", [2, 3, 4])
+def test_all_mappings_n4_loopback(G):
+    rng = np.random.default_rng(40 + G)
+    xs = [_gauss(rng, 4, 1001), _gauss(rng, 4, 64, "bf16"), _gauss(rng, 4, 3)]
+    want = [oracle.reduce(xs[0], "f32"), oracle.reduce(xs[1], "bf16"), oracle.reduce(xs[2], "f32")]
+    for m in _surjections(4, G):
+        for sched in (es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN):
+            res = reduce_loopback(xs, G, m, sched)
+            for g in range(G):
+                for b in range(3):
+                    assert_bits_equal(res[g][b], want[b], f"map={m} sched={sched} rank={g} bucket={b}")
+
+
+@pytest.mark.parametrize("G,kind", [(2, "contiguous"), (4, "contiguous"), (8, "contiguous"), (8, "round_robin"),
+                                    (4, "random"), (8, "random"), (3, "random")])
+@pytest.mark.parametrize("sched", [es.ES_SCHED_AUTO, es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN])
+def test_mappings_n8_loopback(G, kind, sched):
+    rng = np.random.default_rng(G * 10 + len(kind))
+    xs = [_gauss(rng, 8, 200003), _gauss(rng, 8, 4096 + 5, "bf16")]
+    want = [oracle.reduce(xs[0], "f32"), oracle.reduce(xs[1], "bf16")]
+    res = reduce_loopback(xs, G, workloads.mapping(8, G, kind), sched)
+    for g in range(G):
+        for b in range(2):
+            assert_bits_equal(res[g][b], want[b], f"G={G} {kind} sched={sched} rank={g} b={b}")
+
+
+@pytest.mark.parametrize("kind", ["contiguous", "round_robin"])
+def test_bert_uneven_n12_g8_loopback(kind):
+    """BERT config shape: N=12 on G=8, n = [2,2,2,2,1,1,1,1] (contiguous) and
+    k mod 8 (round robin): identical bits, equal to the oracle and to G=1."""
+    rng = np.random.default_rng(12)
+    xs = [_gauss(rng, 12, 120011, "bf16"), _gauss(rng, 12, 30000, "bf16")]
+    want = [oracle.reduce(x, "bf16") for x in xs]
+    g1 = reduce_g1(xs)
+    res = reduce_loopback(xs, 8, workloads.mapping(12, 8, kind))
+    for b in range(2):
+        assert_bits_equal(g1[b], want[b])
+        for g in range(8):
+            assert_bits_equal(res[g][b], want[b], f"{kind} rank={g} b={b}")
+
+
+def test_loopback_multi_step_reuse():
+    """Three global steps on the same handles: slot / staging / partial reuse is ordered."""
+    rng = np.random.default_rng(13)
+    xs = [_gauss(rng, 8, 50001), _gauss(rng, 8, 70001)]
+    want = [oracle.reduce(x, "f32") for x in xs]
+    res = reduce_loopback(xs, 4, workloads.mapping(8, 4, "random"), es.ES_SCHED_CHAIN, steps=3)
+    for g in range(4):
+        for b in range(2):
+            assert_bits_equal(res[g][b], want[b])
+
+
+# ---- full size, in the bench launch configuration: sampled windows -----------------------------
+
+@pytest.mark.parametrize("name", ["tiny", "resnet50"])
+def test_full_size_sampled_parity(name):
+    cfg = workloads.config(name)
+    N = cfg["N"]
+    from gpu_util import Aggregator, from_dev
+    buckets = cfg["buckets"]
+    agg = Aggregator(N, 1, 0, [0] * N, buckets)
+    grads = [[workloads.est_bucket(name, k, b, device="cuda") for b in range(len(buckets))] for k in range(N)]
+    outs = [agg.new_out(b) for b in range(len(buckets))]
+    for k in range(N):
+        for b in range(len(buckets)):
+            agg.stash(k, b, grads[k][b], es.ES_STASH_BORROW if k == N - 1 else es.ES_STASH_COPY)
+    for b in range(len(buckets)):
+        agg.allreduce(b, outs[b])
+    torch.cuda.synchronize()
+    agg.sync()
+    rng = np.random.default_rng(0)
+    for b, (L, d) in enumerate(buckets):
+        C = oracle.chunk_elems(L, N)
+        starts = [0, max(0, L - 4099), max(0, C - 2000)] + list(rng.integers(0, max(1, L - 4099), 3))
+        for s in starts:
+            s = int(s)
+            n = min(4099, L - s)
+            win = [from_dev(grads[k][b][s:s + n]) for k in range(N)]
+            want = oracle.reduce(win, d, L=L, first=s)
+            assert_bits_equal(from_dev(outs[b][s:s + n]), want, f"{name} b={b} s={s}")
+    # property at any size: every element finite and |out| <= max_k |x_k| (up to rounding)
+    for b in range(len(buckets)):
+        o = outs[b].float()
+        mx = torch.stack([g[b].float().abs() for g in grads]).amax(0)
+        assert torch.isfinite(o).all() and bool((o.abs() <= mx * 1.01).all())
+    agg.close()

@@ -1,0 +1,149 @@
+"""GPU: context switch (k_swap) and the C-ABI protocol errors.
+
+PAPER.md:575-598 -- an EST's context is its RNG state and implicit per-worker
+state such as BatchNorm running statistics; only that (plus the
+gradients) is swapped at a mini-batch boundary.  The oracle is
+oracle/switch_model.py: after any interleaving of switches and updates,
+every EST's state equals what a dedicated worker would hold."""
+import numpy as np
+import pytest
+import torch
+
+from oracle.switch_model import SwitchModel
+from paper_conf_sc_lixyszrljlllq23_b200 import es, workloads
+from paper_conf_sc_lixyszrljlllq23_b200.aggregator import Aggregator
+
+pytestmark = pytest.mark.gpu
+
+SIZES = [16, workloads.BN_F32 * 4, workloads.BN_I64 * 8, 37]   # Philox record, BN stats, counters, ragged
+
+
+def _setup(N, seed):
+    rng = np.random.default_rng(seed)
+    agg = Aggregator(N, 1, 0, [0] * N, [(64, "f32")], state_nbytes=SIZES)
+    live = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in SIZES]
+    agg.register_state(live)
+    init = {k: [rng.integers(0, 256, n, dtype=np.uint8).tobytes() for n in SIZES] for k in range(N)}
+    for k in range(N):
+        for i in range(len(SIZES)):
+            agg.init_state(k, i, init[k][i])
+    return agg, live, init, rng
+
+
+def _live_bytes(live):
+    torch.cuda.synchronize()
+    return [t.cpu().numpy().tobytes() for t in live]
+
+
+@pytest.mark.parametrize("N", [1, 4, 32])
+def test_switch_model_random_sequences(N):
+    agg, live, init, rng = _setup(N, N)
+    model = SwitchModel(N, init)
+    agg.switch(0)                       # first switch only loads
+    assert _live_bytes(live) == model.state_of(0)
+    cur = 0
+    for step in range(200):
+        if rng.random() < 0.4:          # the running EST updates its context (BN update, RNG advance)
+            i = int(rng.integers(0, len(SIZES)))
+            nb = rng.integers(0, 256, SIZES[i], dtype=np.uint8)
+            live[i].copy_(torch.from_numpy(nb).cuda())
+            model.mutate(i, nb.tobytes())
+        else:
+            k = int(rng.integers(0, N))
+            agg.switch(k)
+            model.switch(k)
+            cur = k
+        if step % 10 == 0:
+            assert _live_bytes(live) == model.state_of(cur)
+            torch.cuda.synchronize()
+            for k in range(N):
+                if k != cur:
+                    assert [agg.read_state(k, i) for i in range(len(SIZES))] == model.state_of(k)
+    agg.sync()
+    agg.close()
+
+
+def test_switch_to_self_is_identity_and_round_trip():
+    agg, live, init, _ = _setup(3, 1)
+    agg.switch(1)
+    before = _live_bytes(live)
+    agg.switch(1)
+    assert _live_bytes(live) == before
+    agg.switch(2)
+    agg.switch(1)
+    assert _live_bytes(live) == before      # round trip restores the bits
+    agg.close()
+
+
+def test_dropout_masks_follow_the_est():
+    """R12: an EST's dropout masks under time-slicing equal those of a dedicated
+    worker seeded the same way (D0 fixed seeds)."""
+    N, steps = 4, 3
+    seeds = [1234 + 17 * k for k in range(N)]
+    gen = torch.cuda.default_generators[torch.cuda.current_device()]
+    x = torch.ones(4096, device="cuda")
+    dedicated = {}
+    for k in range(N):
+        gen.manual_seed(seeds[k])
+        dedicated[k] = [torch.nn.functional.dropout(x, 0.5).clone() for _ in range(steps)]
+    agg = Aggregator(N, 1, 0, [0] * N, [(64, "f32")])
+    agg.attach_generator(gen, seeds)
+    for s in range(steps):
+        for k in range(N):
+            agg.switch(k)
+            m = torch.nn.functional.dropout(x, 0.5)
+            assert torch.equal(m, dedicated[k][s]), (s, k)
+    agg.close()
+
+
+def test_protocol_errors():
+    N = 4
+    agg = Aggregator(N, 2, 0, [0, 0, 1, 1], [(1000, "f32")], transport=es.ES_TRANSPORT_LOOPBACK,
+                     comm=es.es_loopback_create(2).value)
+    g = torch.zeros(1000, device="cuda")
+    out = torch.zeros(1000, device="cuda")
+    with pytest.raises(es.EsError) as e:
+        agg.stash(2, 0, g)                              # EST 2 lives on rank 1
+    assert e.value.status == es.ES_ESTATE
+    with pytest.raises(es.EsError) as e:
+        agg.stash(9, 0, g)
+    assert e.value.status == es.ES_EINVAL
+    with pytest.raises(es.EsError) as e:
+        agg.stash(0, 3, g)
+    assert e.value.status == es.ES_EINVAL
+    with pytest.raises(es.EsError) as e:
+        es.es_stash_grad(agg.h, 0, 0, g.data_ptr() + 4, es.ES_F32, es.ES_STASH_COPY, 0)   # misaligned
+    assert e.value.status == es.ES_EINVAL
+    with pytest.raises(es.EsError) as e:
+        agg.stash(0, 0, g.to(torch.bfloat16), es.ES_STASH_BORROW)   # borrow needs the bucket dtype
+    assert e.value.status == es.ES_EINVAL
+    agg.stash(0, 0, g)
+    with pytest.raises(es.EsError) as e:
+        agg.allreduce(0, out)                           # EST 1 has not stashed
+    assert e.value.status == es.ES_ESTATE
+    with pytest.raises(es.EsError) as e:
+        agg.switch(3)
+    assert e.value.status == es.ES_ESTATE
+    with pytest.raises(es.EsError) as e:
+        es.es_allreduce(agg.h, 0, agg.workspace.data_ptr() + 256, 0)   # out inside the workspace
+    assert e.value.status == es.ES_EINVAL
+    agg.close()
+
+
+def test_init_errors():
+    cfg = es.Config(4, 1, 0, [0] * 4, [(100, es.ES_F32)])
+    nb = es.es_workspace_bytes(cfg)
+    ws = torch.empty(nb + 512, dtype=torch.uint8, device="cuda")
+    with pytest.raises(es.EsError) as e:
+        es.es_init(cfg, ws.data_ptr(), nb - 256)
+    assert e.value.status == es.ES_ENOMEM
+    with pytest.raises(es.EsError) as e:
+        es.es_init(cfg, ws.data_ptr() + 16, nb)
+    assert e.value.status == es.ES_EINVAL
+    host = torch.empty(nb + 256, dtype=torch.uint8)
+    ptr = (host.data_ptr() + 255) // 256 * 256
+    with pytest.raises(es.EsError) as e:
+        es.es_init(cfg, ptr, nb)
+    assert e.value.status == es.ES_EINVAL
+    h = es.es_init(cfg, ws.data_ptr(), nb)
+    es.es_destroy(h)
