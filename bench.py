@@ -40,6 +40,8 @@ def parse():
     p.add_argument("--mapping", default="contiguous", choices=["contiguous", "round_robin", "random"])
     p.add_argument("--sched", default="auto", choices=["auto", "direct", "chain"])
     p.add_argument("--no-graph", action="store_true", help="eager launches instead of one CUDA graph per step")
+    p.add_argument("--per-bucket", action="store_true",
+                   help="one es_stash_grad / es_allreduce call per bucket (DDP-style) instead of the batched calls")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     p.add_argument("--cpu-seconds", type=float, default=10.0)
@@ -239,34 +241,51 @@ def main():
     def step():
         for i, k in enumerate(local):
             agg.switch(k)
+            mode = es.ES_STASH_BORROW if i == len(local) - 1 else es.ES_STASH_COPY
+            if args.per_bucket:
+                for b in range(B):
+                    agg.stash(k, b, grads[k][b], mode)
+            else:
+                agg.stash_many(k, range(B), grads[k], mode)
+        if args.per_bucket:
             for b in range(B):
-                agg.stash(k, b, grads[k][b], es.ES_STASH_BORROW if i == len(local) - 1 else es.ES_STASH_COPY)
-        for b in range(B):
-            agg.allreduce(b, outs[b])
+                agg.allreduce(b, outs[b])
+        else:
+            agg.allreduce_many(range(B), outs)
 
     use_graph = not args.no_graph
     stream = torch.cuda.Stream(device=dev)
-    for _ in range(max(args.warmup, 3) if not use_graph else 2):
+    for _ in range(2):
         with torch.cuda.stream(stream):
             step()
     torch.cuda.synchronize()
-    graph = None
-    agg.profile(True)
-    agg.profile_reset()
+    graph = graph_prof = None
     if use_graph:
+        # Two captures of the same step: without timing events (the steps we
+        # time) and with per-kernel event nodes (the last timed step, which
+        # provides the kernel durations for the roofline).
         graph = torch.cuda.CUDAGraph()
         with torch.cuda.graph(graph, stream=stream):
             step()
+        agg.profile(True)
+        agg.profile_reset()
+        graph_prof = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph_prof, stream=stream):
+            step()
+        agg.profile(False)
         torch.cuda.synchronize()
         for _ in range(max(args.warmup, 3)):
             with torch.cuda.stream(stream):
                 graph.replay()
+        with torch.cuda.stream(stream):
+            graph_prof.replay()
         torch.cuda.synchronize()
     else:
-        for _ in range(max(args.warmup, 3) - 2):
+        for _ in range(max(args.warmup, 3)):
             with torch.cuda.stream(stream):
                 step()
         torch.cuda.synchronize()
+        agg.profile(True)
         agg.profile_reset()
 
     clocks = Clocks(local_rank)
@@ -284,7 +303,7 @@ def main():
                 flush.zero_()                     # L2 flush between timed steps (untimed)
             starts[i].record(stream)
             if graph is not None:
-                graph.replay()
+                (graph_prof if i == args.steps - 1 else graph).replay()
             else:
                 step()
             ends[i].record(stream)
@@ -323,6 +342,7 @@ def main():
         "vs_baseline": None, "dtype": cfg["dtype"], "data": "synthetic",
         "config": {"workload": name, "N": N, "G": G, "mapping": args.mapping, "sched": args.sched,
                    "buckets": B, "elements": sum(n for n, _ in buckets), "graph": graph is not None,
+                   "api": "per-bucket" if args.per_bucket else "batched",
                    "l2": ("inputs larger than L2 (%.1f MB of EST gradients per GPU per step)" % (in_bytes / 1e6))
                    if flush is None else "L2 flushed between timed steps (512 MB write)",
                    "desc": cfg["desc"]},
@@ -333,6 +353,7 @@ def main():
                      "avg_launch_us": round(fl_ms / max(fl_n, 1) * 1e3, 2), "peak_source": peak_src},
         "breakdown_ms_per_step": {k: round(v[1] / steps_profiled, 4) for k, v in prof.items()},
         "gpu_launches": int(round(launches_per_step * args.steps)),
+        "step_ms_p10_p50_p90": [round(float(np.percentile(step_ms, q)), 4) for q in (10, 50, 90)],
         "clocks": clk,
     }
 
@@ -380,10 +401,9 @@ def main():
                 for b in range(B):
                     live_grad[b].copy_(host[k][b], non_blocking=True)     # "backward" lands in the live buffer
                 agg.switch(k)
-                for b in range(B):
-                    agg.stash(k, b, live_grad[b], es.ES_STASH_BORROW if i == len(local) - 1 else es.ES_STASH_COPY)
+                agg.stash_many(k, range(B), live_grad, es.ES_STASH_BORROW if i == len(local) - 1 else es.ES_STASH_COPY)
+            agg.allreduce_many(range(B), outs)
             for b in range(B):
-                agg.allreduce(b, outs[b])
                 host_out[b].copy_(outs[b], non_blocking=True)
 
         k_e2e = max(3, min(args.steps, 10))

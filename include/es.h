@@ -184,6 +184,15 @@ es_status es_switch_context(es_handle h, int32_t est, es_stream stream);
 es_status es_stash_grad(es_handle h, int32_t est, int32_t bucket, const void *grad,
                         es_dtype grad_dtype, es_stash_mode mode, es_stream stream);
 
+/* Batched form of es_stash_grad: stashes n buckets of local EST `est` (the
+ * paper swaps all of an EST's gradients at its context switch)
+ * with one multi-segment kernel per (grad dtype, bucket dtype) pair.
+ * buckets/grads/grad_dtypes are host arrays of length n; the same rules as
+ * es_stash_grad apply to every entry; validation of all entries happens
+ * before anything is enqueued. */
+es_status es_stash_grads(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
+                         const es_dtype *grad_dtypes, es_stash_mode mode, es_stream stream);
+
 /* ---- aggregation ---------------------------------------------------------- */
 
 /* Collective over the G ranks: every rank calls it for the same bucket
@@ -194,6 +203,13 @@ es_status es_stash_grad(es_handle h, int32_t est, int32_t bucket, const void *gr
  * every rank.  `out` may alias a BORROWed gradient of this bucket; it may
  * not overlap the workspace.  Enqueued on `stream`; no host sync. */
 es_status es_allreduce(es_handle h, int32_t bucket, void *out, es_stream stream);
+
+/* Batched form of es_allreduce over n distinct buckets (host arrays), in the
+ * given order; every rank must pass the same bucket sequence.  Independent
+ * folds are merged into multi-segment launches (G == 1: one launch for all
+ * buckets of a dtype).  Same argument rules and errors as es_allreduce,
+ * checked for every entry before anything is enqueued. */
+es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void *const *outs, es_stream stream);
 
 /* ---- planner introspection (host-only, no CUDA) -------------------------- */
 

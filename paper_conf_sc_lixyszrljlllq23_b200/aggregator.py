@@ -93,6 +93,15 @@ class Aggregator:
     def stash(self, est, bucket, grad, mode=es.ES_STASH_COPY, stream=None):
         es.es_stash_grad(self.h, est, bucket, grad.data_ptr(), DTYPES[grad.dtype], mode, _stream(stream))
 
+    def stash_many(self, est, buckets, grads, mode=es.ES_STASH_COPY, stream=None):
+        """All of EST `est`'s buckets in one call (one multi-segment launch)."""
+        es.es_stash_grads(self.h, est, list(buckets), [g.data_ptr() for g in grads],
+                          [DTYPES[g.dtype] for g in grads], mode, _stream(stream))
+
+    def allreduce_many(self, buckets, outs, stream=None):
+        es.es_allreduce_many(self.h, list(buckets), [o.data_ptr() for o in outs], _stream(stream))
+        return outs
+
     def allreduce(self, bucket, out, stream=None):
         es.es_allreduce(self.h, bucket, out.data_ptr(), _stream(stream))
         return out

@@ -112,7 +112,7 @@ struct es_ctx {
     if (sticky != ES_OK) return set_err(sticky, "handle poisoned by an earlier error: " + sticky_msg);
     return ES_OK;
   }
-  // Runs `launch` bracketed by timing events when profiling is on.
+  // Runs `launch(int* n_launches)` bracketed by timing events when profiling is on.
   template <typename F>
   es_status timed(int kind, uint64_t nbytes, cudaStream_t s, F launch) {
     cudaEvent_t a = nullptr, b = nullptr;
@@ -124,13 +124,14 @@ struct es_ctx {
       b = ev();
       cudaEventRecordWithFlags(a, s, flags);
     }
-    cudaError_t e = launch();
+    int n = 0;
+    cudaError_t e = launch(&n);
     if (e != cudaSuccess) return poison(ES_ECUDA, std::string("kernel launch: ") + cudaGetErrorString(e));
     if (prof) {
       cudaEventRecordWithFlags(b, s, flags);
       recs.push_back({kind, a, b, cap});
     }
-    launches[kind]++;
+    launches[kind] += n;
     bytes[kind] += nbytes;
     return ES_OK;
   }
@@ -331,7 +332,10 @@ es_status es_switch_context(es_handle h, int32_t est, es_stream stream) {
     const int32_t cur = h->cur_local;
     const auto *tab = reinterpret_cast<const es::SwapEntry *>(h->ws + p.table_off);
     s = h->timed(ES_KERNEL_SWAP, (cur >= 0 ? 4 : 2) * tot, cs,
-                 [&] { return es::launch_swap(tab, n, h->max_state, cur, li, cs); });
+                 [&](int *nl) {
+                   *nl = 1;
+                   return es::launch_swap(tab, n, h->max_state, cur, li, cs);
+                 });
     if (s != ES_OK) return s;
   }
   h->cur_local = li;
@@ -340,158 +344,223 @@ es_status es_switch_context(es_handle h, int32_t est, es_stream stream) {
 
 // ---- stash ----------------------------------------------------------------------
 
-es_status es_stash_grad(es_handle h, int32_t est, int32_t bucket, const void *grad, es_dtype gdt, es_stash_mode mode,
-                        es_stream stream) {
+es_status es_stash_grads(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
+                         const es_dtype *gdts, es_stash_mode mode, es_stream stream) {
   es_status s = check_handle(h);
   if (s != ES_OK) return s;
   const es::Plan &p = h->plan;
+  if (n < 0 || (n > 0 && (!buckets || !grads || !gdts))) return set_err(ES_EINVAL, "bad bucket/grad arrays");
   if (est < 0 || est >= p.N) return set_err(ES_EINVAL, "est out of range");
-  if (bucket < 0 || bucket >= h->B) return set_err(ES_EINVAL, "bucket out of range");
-  if (gdt != ES_F32 && gdt != ES_BF16) return set_err(ES_EINVAL, "bad grad dtype");
   if (mode != ES_STASH_COPY && mode != ES_STASH_BORROW) return set_err(ES_EINVAL, "bad stash mode");
-  const es::BucketPlan &b = p.bp[bucket];
-  if (b.L > 0 && (!grad || !aligned16(grad))) return set_err(ES_EINVAL, "grad must be a 16-byte aligned device pointer");
-  if (mode == ES_STASH_BORROW && gdt != b.dtype) return set_err(ES_EINVAL, "BORROW needs grad dtype == bucket dtype");
-  int32_t li = p.local_index[est];
+  for (int32_t i = 0; i < n; ++i) {
+    const int32_t bk = buckets[i];
+    if (bk < 0 || bk >= h->B) return set_err(ES_EINVAL, "bucket out of range");
+    if (gdts[i] != ES_F32 && gdts[i] != ES_BF16) return set_err(ES_EINVAL, "bad grad dtype");
+    const es::BucketPlan &b = p.bp[bk];
+    if (b.L > 0 && (!grads[i] || !aligned16(grads[i])))
+      return set_err(ES_EINVAL, "grad must be a 16-byte aligned device pointer");
+    if (mode == ES_STASH_BORROW && gdts[i] != b.dtype)
+      return set_err(ES_EINVAL, "BORROW needs grad dtype == bucket dtype");
+  }
+  const int32_t li = p.local_index[est];
   if (li < 0) return set_err(ES_ESTATE, "est is not mapped to this rank");
   cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
-  const size_t k = (size_t)li * h->B + bucket;
+  const unsigned long long cap = capture_id(cs);
   if (mode == ES_STASH_COPY) {
-    unsigned char *slot = h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[bucket];
-    if (h->ar_recorded[bucket] && h->ar_cap[bucket] == capture_id(cs) &&
-        cudaStreamWaitEvent(cs, h->ar_ev[bucket], 0) != cudaSuccess)
-      return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
-    const uint64_t nbytes = b.L * (es::dtype_size(gdt) + b.esize);
-    s = h->timed(ES_KERNEL_STASH, nbytes, cs, [&] {
-      return es::launch_stash(grad, gdt, slot, b.dtype, (int64_t)b.L, cs, h->blocks_ov, h->threads_ov);
-    });
-    if (s != ES_OK) return s;
-    h->borrowed[k] = nullptr;
-  } else {
-    h->borrowed[k] = grad;
+    // A slot may be overwritten only after the previous aggregation of its bucket read it.
+    for (int32_t i = 0; i < n; ++i) {
+      const int32_t bk = buckets[i];
+      if (h->ar_recorded[bk] && h->ar_cap[bk] == cap && cudaStreamWaitEvent(cs, h->ar_ev[bk], 0) != cudaSuccess)
+        return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
+    }
+    // One multi-segment launch per (grad dtype, bucket dtype) pair present.
+    for (int sd = 0; sd < 2; ++sd)
+      for (int dd = 0; dd < 2; ++dd) {
+        std::vector<es::StashSegDesc> segs;
+        uint64_t nbytes = 0;
+        for (int32_t i = 0; i < n; ++i) {
+          const int32_t bk = buckets[i];
+          const es::BucketPlan &b = p.bp[bk];
+          if ((int)gdts[i] != sd || (int)b.dtype != dd || b.L == 0) continue;
+          segs.push_back({grads[i], h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[bk], (int64_t)b.L});
+          nbytes += b.L * (es::dtype_size(gdts[i]) + b.esize);
+        }
+        if (segs.empty()) continue;
+        s = h->timed(ES_KERNEL_STASH, nbytes, cs, [&](int *nl) {
+          return es::launch_stash_multi((es_dtype)sd, (es_dtype)dd, segs.data(), (int)segs.size(), cs, h->blocks_ov,
+                                        h->threads_ov, nl);
+        });
+        if (s != ES_OK) return s;
+      }
   }
-  if (cudaEventRecord(h->stash_ev[k], cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaEventRecord failed");
-  h->stash_cap[k] = capture_id(cs);
-  h->stashed[k] = 1;
+  for (int32_t i = 0; i < n; ++i) {
+    const size_t k = (size_t)li * h->B + buckets[i];
+    h->borrowed[k] = mode == ES_STASH_BORROW ? grads[i] : nullptr;
+    if (cudaEventRecord(h->stash_ev[k], cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaEventRecord failed");
+    h->stash_cap[k] = cap;
+    h->stashed[k] = 1;
+  }
   return ES_OK;
+}
+
+es_status es_stash_grad(es_handle h, int32_t est, int32_t bucket, const void *grad, es_dtype gdt, es_stash_mode mode,
+                        es_stream stream) {
+  return es_stash_grads(h, est, 1, &bucket, &grad, &gdt, mode, stream);
 }
 
 // ---- aggregation --------------------------------------------------------------------
 
-es_status es_allreduce(es_handle h, int32_t bucket, void *out, es_stream stream) {
+es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void *const *outs, es_stream stream) {
   es_status s = check_handle(h);
   if (s != ES_OK) return s;
   const es::Plan &p = h->plan;
-  if (bucket < 0 || bucket >= h->B) return set_err(ES_EINVAL, "bucket out of range");
-  const es::BucketPlan &b = p.bp[bucket];
-  const uint64_t out_bytes = b.L * b.esize;
-  if (b.L > 0) {
-    if (!out || !aligned16(out)) return set_err(ES_EINVAL, "out must be a 16-byte aligned device pointer");
-    const unsigned char *o = reinterpret_cast<const unsigned char *>(out);
-    if (o < h->ws + h->ws_bytes && h->ws < o + out_bytes) return set_err(ES_EINVAL, "out overlaps the workspace");
+  if (n < 0 || (n > 0 && (!buckets || !outs))) return set_err(ES_EINVAL, "bad bucket/out arrays");
+  for (int32_t i = 0; i < n; ++i) {
+    const int32_t bk = buckets[i];
+    if (bk < 0 || bk >= h->B) return set_err(ES_EINVAL, "bucket out of range");
+    for (int32_t j = 0; j < i; ++j)
+      if (buckets[j] == bk) return set_err(ES_EINVAL, "bucket listed twice");
+    const es::BucketPlan &b = p.bp[bk];
+    if (b.L == 0) continue;
+    if (!outs[i] || !aligned16(outs[i])) return set_err(ES_EINVAL, "out must be a 16-byte aligned device pointer");
+    const unsigned char *o = reinterpret_cast<const unsigned char *>(outs[i]);
+    if (o < h->ws + h->ws_bytes && h->ws < o + b.L * b.esize) return set_err(ES_EINVAL, "out overlaps the workspace");
+    for (int32_t li = 0; li < h->n_local; ++li)
+      if (!h->stashed[(size_t)li * h->B + bk])
+        return set_err(ES_ESTATE, "es_allreduce before every local EST stashed this bucket");
   }
-  for (int32_t li = 0; li < h->n_local; ++li)
-    if (!h->stashed[(size_t)li * h->B + bucket])
-      return set_err(ES_ESTATE, "es_allreduce before every local EST stashed this bucket");
+  for (int32_t i = 0; i < n; ++i)
+    for (int32_t li = 0; li < h->n_local; ++li)
+      if (!h->stashed[(size_t)li * h->B + buckets[i]])
+        return set_err(ES_ESTATE, "es_allreduce before every local EST stashed this bucket");
   cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
   const unsigned long long cap = capture_id(cs);
-  for (int32_t li = 0; li < h->n_local; ++li) {
-    const size_t k = (size_t)li * h->B + bucket;
-    if (h->stash_cap[k] == cap && cudaStreamWaitEvent(cs, h->stash_ev[k], 0) != cudaSuccess)
-      return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
-  }
+  for (int32_t i = 0; i < n; ++i)
+    for (int32_t li = 0; li < h->n_local; ++li) {
+      const size_t k = (size_t)li * h->B + buckets[i];
+      if (h->stash_cap[k] == cap && cudaStreamWaitEvent(cs, h->stash_ev[k], 0) != cudaSuccess)
+        return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
+    }
   if (h->last_ar && h->last_ar_cap == cap && cudaStreamWaitEvent(cs, h->last_ar, 0) != cudaSuccess)
     return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
 
-  const uint32_t es_ = b.esize;
-  auto src_base = [&](int32_t e) -> unsigned char * {   // element 0 of EST e's contribution
-    int32_t li = p.local_index[e];
-    const void *bw = h->borrowed[(size_t)li * h->B + bucket];
-    if (bw) return reinterpret_cast<unsigned char *>(const_cast<void *>(bw));
-    return h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[bucket];
-  };
-  auto contrib_at = [&](int32_t e, int64_t lo) -> unsigned char * {
-    if (p.local_index[e] >= 0) return src_base(e) + (uint64_t)lo * es_;
-    return h->ws + p.stage_off + (uint64_t)b.stage_index[e] * b.stage_stride + (uint64_t)(lo - b.shard_lo) * es_;
-  };
-  auto part_at = [&](int64_t id, int64_t lo) -> unsigned char * {
-    const es::Part &pt = b.parts[id];
-    return h->ws + p.parts_off + pt.off + (uint64_t)(lo - pt.lo) * 4;
-  };
-  unsigned char *outp = reinterpret_cast<unsigned char *>(out);
   const float r = 1.0f / (float)p.N;   // R5: fl32(1/N), correctly rounded fp32 division
-  std::vector<const void *> srcs(p.N);
 
-  for (const es::Op &op : b.ops) {
-    const int64_t *f = op.f;
-    switch (f[0]) {
-      case ES_OP_FOLD: {
-        const int64_t lo = f[1], hi = f[2];
-        es::FoldDesc d;
-        d.lo = lo;
-        d.n = hi - lo;
-        d.N = p.N;
-        d.C = (uint32_t)b.C;
-        d.r = r;
-        int nsrc;
-        if (f[3] < 0) {
-          d.rot = true;
-          nsrc = p.N;
-          for (int32_t e = 0; e < p.N; ++e) srcs[e] = contrib_at(e, lo);
-        } else {
-          d.rot = false;
-          d.m = (int32_t)f[4];
-          nsrc = d.m;
-          for (int32_t t = 0; t < d.m; ++t) srcs[t] = contrib_at((int32_t)((f[3] + t) % p.N), lo);
+  // Pending FOLD ops: consecutive folds (across buckets for G == 1, within a
+  // chain round for G > 1) are independent and go out as one multi-segment
+  // launch; a transport group flushes them first.
+  std::vector<es::FoldSegDesc> pend;
+  std::vector<std::vector<const void *>> pend_src;
+  es_dtype pend_dt = ES_F32;
+  uint64_t pend_bytes = 0;
+  auto flush = [&]() -> es_status {
+    if (pend.empty()) return ES_OK;
+    for (size_t i = 0; i < pend.size(); ++i) pend[i].src = pend_src[i].data();
+    es_status st = h->timed(ES_KERNEL_FOLD, pend_bytes, cs, [&](int *nl) {
+      return es::launch_fold_multi(pend_dt, p.N, r, pend.data(), (int)pend.size(), cs, h->blocks_ov, h->threads_ov,
+                                   nl);
+    });
+    pend.clear();
+    pend_src.clear();
+    pend_bytes = 0;
+    return st;
+  };
+
+  for (int32_t i = 0; i < n; ++i) {
+    const int32_t bucket = buckets[i];
+    const es::BucketPlan &b = p.bp[bucket];
+    const uint32_t esz = b.esize;
+    auto src_base = [&](int32_t e) -> unsigned char * {   // element 0 of local EST e's contribution
+      const int32_t li = p.local_index[e];
+      const void *bw = h->borrowed[(size_t)li * h->B + bucket];
+      if (bw) return reinterpret_cast<unsigned char *>(const_cast<void *>(bw));
+      return h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[bucket];
+    };
+    auto contrib_at = [&](int32_t e, int64_t lo) -> unsigned char * {
+      if (p.local_index[e] >= 0) return src_base(e) + (uint64_t)lo * esz;
+      return h->ws + p.stage_off + (uint64_t)b.stage_index[e] * b.stage_stride + (uint64_t)(lo - b.shard_lo) * esz;
+    };
+    auto part_at = [&](int64_t id, int64_t lo) -> unsigned char * {
+      const es::Part &pt = b.parts[id];
+      return h->ws + p.parts_off + pt.off + (uint64_t)(lo - pt.lo) * 4;
+    };
+    unsigned char *outp = reinterpret_cast<unsigned char *>(outs[i]);
+    for (const es::Op &op : b.ops) {
+      const int64_t *f = op.f;
+      switch (f[0]) {
+        case ES_OP_FOLD: {
+          if (!pend.empty() && pend_dt != b.dtype && (s = flush()) != ES_OK) return s;
+          pend_dt = b.dtype;
+          const int64_t lo = f[1], hi = f[2];
+          es::FoldSegDesc d;
+          d.lo = lo;
+          d.n = hi - lo;
+          d.C = (uint32_t)b.C;
+          std::vector<const void *> src;
+          if (f[3] < 0) {
+            d.rot = true;
+            for (int32_t e = 0; e < p.N; ++e) src.push_back(contrib_at(e, lo));
+          } else {
+            d.rot = false;
+            d.m = (int32_t)f[4];
+            for (int32_t t = 0; t < d.m; ++t) src.push_back(contrib_at((int32_t)((f[3] + t) % p.N), lo));
+          }
+          d.part_in = f[5] == ES_BUF_PART ? reinterpret_cast<const float *>(part_at(f[6], lo)) : nullptr;
+          d.out_partial = f[7] == ES_BUF_PART;
+          d.out = d.out_partial ? (void *)part_at(f[8], lo) : (void *)(outp + (uint64_t)lo * esz);
+          pend_bytes += (uint64_t)d.n * ((uint64_t)src.size() * esz + (d.part_in ? 4 : 0) + (d.out_partial ? 4 : esz));
+          pend.push_back(d);
+          pend_src.push_back(std::move(src));
+          break;
         }
-        d.part_in = f[5] == ES_BUF_PART ? reinterpret_cast<const float *>(part_at(f[6], lo)) : nullptr;
-        d.out_partial = f[7] == ES_BUF_PART;
-        d.out = d.out_partial ? (void *)part_at(f[8], lo) : (void *)(outp + (uint64_t)lo * es_);
-        const uint64_t nb = (uint64_t)d.n * ((uint64_t)nsrc * es_ + (d.part_in ? 4 : 0) + (d.out_partial ? 4 : es_));
-        s = h->timed(ES_KERNEL_FOLD, nb, cs, [&] {
-          return es::launch_fold(b.dtype, d, srcs.data(), cs, h->blocks_ov, h->threads_ov);
-        });
-        if (s != ES_OK) return s;
-        break;
-      }
-      case ES_OP_GROUP_BEGIN:
-        if ((s = h->tp->group_begin()) != ES_OK) return h->poison(s, h->tp->err);
-        break;
-      case ES_OP_GROUP_END:
-        if ((s = h->tp->group_end(cs)) != ES_OK) return h->poison(s, h->tp->err);
-        break;
-      case ES_OP_SEND:
-      case ES_OP_RECV: {
-        const int64_t lo = f[1], hi = f[2];
-        const int peer = (int)f[3];
-        unsigned char *ptr = nullptr;
-        uint64_t w = es_;
-        switch (f[4]) {
-          case ES_BUF_SRC: ptr = contrib_at((int32_t)f[5], lo); break;
-          case ES_BUF_STAGE: ptr = contrib_at((int32_t)f[5], lo); break;
-          case ES_BUF_PART: ptr = part_at(f[5], lo); w = 4; break;
-          case ES_BUF_OUT: ptr = outp + (uint64_t)lo * es_; break;
-          default: return h->poison(ES_ESTATE, "corrupt plan: bad buffer kind");
+        case ES_OP_GROUP_BEGIN:
+          if ((s = flush()) != ES_OK) return s;
+          if ((s = h->tp->group_begin()) != ES_OK) return h->poison(s, h->tp->err);
+          break;
+        case ES_OP_GROUP_END:
+          if ((s = h->tp->group_end(cs)) != ES_OK) return h->poison(s, h->tp->err);
+          break;
+        case ES_OP_SEND:
+        case ES_OP_RECV: {
+          const int64_t lo = f[1], hi = f[2];
+          const int peer = (int)f[3];
+          unsigned char *ptr = nullptr;
+          uint64_t w = esz;
+          switch (f[4]) {
+            case ES_BUF_SRC:
+            case ES_BUF_STAGE: ptr = contrib_at((int32_t)f[5], lo); break;
+            case ES_BUF_PART: ptr = part_at(f[5], lo); w = 4; break;
+            case ES_BUF_OUT: ptr = outp + (uint64_t)lo * esz; break;
+            default: return h->poison(ES_ESTATE, "corrupt plan: bad buffer kind");
+          }
+          const size_t nbytes = (size_t)(hi - lo) * w;
+          s = f[0] == ES_OP_SEND ? h->tp->send(ptr, nbytes, peer) : h->tp->recv(ptr, nbytes, peer);
+          if (s != ES_OK) return h->poison(s, h->tp->err);
+          break;
         }
-        const size_t nbytes = (size_t)(hi - lo) * w;
-        s = f[0] == ES_OP_SEND ? h->tp->send(ptr, nbytes, peer) : h->tp->recv(ptr, nbytes, peer);
-        if (s != ES_OK) return h->poison(s, h->tp->err);
-        break;
+        default:
+          return h->poison(ES_ESTATE, "corrupt plan: bad opcode");
       }
-      default:
-        return h->poison(ES_ESTATE, "corrupt plan: bad opcode");
     }
   }
-  if (cudaEventRecord(h->ar_ev[bucket], cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaEventRecord failed");
-  h->ar_recorded[bucket] = 1;
-  h->ar_cap[bucket] = cap;
-  h->last_ar = h->ar_ev[bucket];
-  h->last_ar_cap = cap;
-  for (int32_t li = 0; li < h->n_local; ++li) {
-    h->stashed[(size_t)li * h->B + bucket] = 0;
-    h->borrowed[(size_t)li * h->B + bucket] = nullptr;
+  if ((s = flush()) != ES_OK) return s;
+  for (int32_t i = 0; i < n; ++i) {
+    const int32_t bucket = buckets[i];
+    if (cudaEventRecord(h->ar_ev[bucket], cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaEventRecord failed");
+    h->ar_recorded[bucket] = 1;
+    h->ar_cap[bucket] = cap;
+    h->last_ar = h->ar_ev[bucket];
+    h->last_ar_cap = cap;
+    for (int32_t li = 0; li < h->n_local; ++li) {
+      h->stashed[(size_t)li * h->B + bucket] = 0;
+      h->borrowed[(size_t)li * h->B + bucket] = nullptr;
+    }
   }
   return ES_OK;
+}
+
+es_status es_allreduce(es_handle h, int32_t bucket, void *out, es_stream stream) {
+  return es_allreduce_many(h, 1, &bucket, &out, stream);
 }
 
 // ---- instrumentation ---------------------------------------------------------

@@ -6,8 +6,18 @@
 //
 // All three are HBM-streaming kernels (no data reuse, no contraction), so
 // they use 128-bit vector loads on the non-coherent path with L1
-// no-allocate, many independent loads in flight per thread, and grids sized
-// in multiples of the 148 SMs.
+// no-allocate, many independent loads in flight per thread, coalesced lanes,
+// and grids sized in multiples of the 148 SMs.
+//
+// Fold and stash are MULTI-SEGMENT kernels: one launch covers many buckets
+// (or many chain segments), each segment owning a contiguous range of
+// blocks proportional to its size.  Fewer, larger launches remove the
+// per-launch ramp-up/tail that dominated bucket-sized launches on B200.
+// Launches use programmatic dependent launch (PDL): every kernel first
+// waits for its predecessor (griddepcontrol.wait) and then lets its
+// successor's CTAs become resident (griddepcontrol.launch_dependents), so
+// the launch latency of kernel i+1 hides under the tail of kernel i while
+// stream order (and therefore every data dependency) is preserved.
 //
 // Bit-exactness rules (R6): every fp32 add is __fadd_rn and the
 // scale is __fmul_rn (no FMA contraction), no fast-math, no FTZ (nvcc
@@ -20,12 +30,24 @@
 #include <cuda_bf16.h>
 
 #include <algorithm>
+#include <cstdlib>
+#include <vector>
 
 namespace es {
 namespace {
 
 constexpr int kSMs = 148;        // B200
 constexpr int kBatch = 8;        // sources loaded per batch in k_fold
+
+bool g_pdl = [] {
+  const char *e = std::getenv("ES_NO_PDL");
+  return !(e && e[0] == '1');
+}();
+
+__device__ __forceinline__ void pdl_enter() {
+  asm volatile("griddepcontrol.wait;" ::: "memory");             // predecessor complete + visible
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");  // successor may become resident
+}
 
 __device__ __forceinline__ int4 ld_stream(const void *p) {
   int4 r;
@@ -34,11 +56,63 @@ __device__ __forceinline__ int4 ld_stream(const void *p) {
                : "l"(p));
   return r;
 }
+__device__ __forceinline__ uint2 ld_stream(const uint2 *p) {
+  uint2 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v2.u32 {%0, %1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ int4 ld_stream(const int4 *p) { return ld_stream(static_cast<const void *>(p)); }
 
 __device__ __forceinline__ void st_stream(void *p, const int4 &v) {
   asm volatile("st.global.L1::no_allocate.v4.s32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x), "r"(v.y),
                "r"(v.z), "r"(v.w)
                : "memory");
+}
+__device__ __forceinline__ void st_stream(uint2 *p, const uint2 &v) {
+  asm volatile("st.global.L1::no_allocate.v2.u32 [%0], {%1, %2};" ::"l"(p), "r"(v.x), "r"(v.y) : "memory");
+}
+__device__ __forceinline__ void st_stream(int4 *p, const int4 &v) { st_stream(static_cast<void *>(p), v); }
+
+template <typename K, typename P>
+cudaError_t launch(K kernel, dim3 grid, dim3 block, cudaStream_t s, const P &params) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = g_pdl ? 1 : 0;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, kernel, params);
+  return e != cudaSuccess ? e : cudaGetLastError();
+}
+
+// Block -> segment: the last segment whose first block is <= b.
+template <typename Seg>
+__device__ __forceinline__ int find_seg(const Seg *seg, int nseg, int b) {
+  int lo = 0, hi = nseg - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (seg[mid].block0 <= b) lo = mid;
+    else hi = mid - 1;
+  }
+  return lo;
+}
+
+// Split `total` blocks over segments proportionally to their work (>= 1 each).
+void split_blocks(const std::vector<int64_t> &work, int total, std::vector<int32_t> *block0, int *nblocks) {
+  int64_t sum = 0;
+  for (int64_t w : work) sum += std::max<int64_t>(w, 1);
+  block0->resize(work.size());
+  int b = 0;
+  for (size_t i = 0; i < work.size(); ++i) {
+    (*block0)[i] = b;
+    int64_t nb = (int64_t)((double)total * (double)std::max<int64_t>(work[i], 1) / (double)sum + 0.5);
+    b += (int)std::max<int64_t>(nb, 1);
+  }
+  *nblocks = b;
 }
 
 // ---- element-type traits --------------------------------------------------
@@ -75,7 +149,7 @@ struct BF16T {
     widen2((uint32_t)v.x, a + 0); widen2((uint32_t)v.y, a + 2);
     widen2((uint32_t)v.z, a + 4); widen2((uint32_t)v.w, a + 6);
   }
-  __device__ static __forceinline__ uint32_t pack2(float lo, float hi) {
+  __device__ static __forceinline__ uint32_t pack2(float lo, float hi) {   // RNE (R13)
     uint32_t l = __bfloat16_as_ushort(__float2bfloat16_rn(lo));
     uint32_t h = __bfloat16_as_ushort(__float2bfloat16_rn(hi));
     return l | (h << 16);
@@ -94,45 +168,50 @@ struct BF16T {
 
 // ---- k_fold ---------------------------------------------------------------
 
-template <int MAXN>
-struct FoldParams {
-  const void *src[MAXN];
-  const float *part_in;
-  void *out;
-  int64_t lo;
-  int64_t n;
-  int32_t N;
-  int32_t m;
+struct FoldSeg {
+  const float *part_in;   // element lo at part_in[0], or null
+  void *out;              // element lo at out[0]
+  int64_t lo, n;
   uint32_t C;
-  int32_t rot;
+  int32_t rot, m, src0;   // sources: src[src0 ...]
   int32_t out_partial;
-  float r;
+  int32_t block0;         // first block of this segment
 };
 
-template <typename T, int MAXN>
-__device__ __forceinline__ void fold_vector(const FoldParams<MAXN> &p, int64_t t, float *acc) {
+template <int MAXSEG, int MAXSRC>
+struct FoldParams {
+  int32_t nseg, N, nblocks;
+  float r;
+  FoldSeg seg[MAXSEG];
+  const void *src[MAXSRC];
+};
+
+// Fold of one 16-byte vector at segment offset t (elements), into acc[V].
+template <typename T>
+__device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const *src, int32_t N, int64_t t,
+                                            float *acc) {
   constexpr int V = T::kVec;
   int cnt, idx;
-  if (p.rot) {
-    const uint32_t c = (uint32_t)(p.lo + t) / p.C;          // R1: chunk of this vector
-    idx = (int)(c + 1u == (uint32_t)p.N ? 0u : c + 1u);      // R2: start at rank c+1
-    cnt = p.N;
+  if (g.rot) {
+    const uint32_t c = (uint32_t)(g.lo + t) / g.C;           // R1: chunk of this vector
+    idx = (int)(c + 1u == (uint32_t)N ? 0u : c + 1u);         // R2: start at rank c+1
+    cnt = N;
   } else {
     idx = 0;
-    cnt = p.m;
+    cnt = g.m;
   }
-  const int64_t boff = t * T::kSize;                         // byte offset of the vector
+  const int64_t boff = t * T::kSize;
   int done = 0;
-  if (p.part_in) {                                           // continue a chain partial
-    const float *pp = p.part_in + t;
+  if (g.part_in) {                                            // R14: continue a chain partial
+    const float *pp = g.part_in + t;
 #pragma unroll
     for (int q = 0; q < V / 4; ++q) {
       int4 w = ld_stream(pp + 4 * q);
       acc[4 * q + 0] = __int_as_float(w.x); acc[4 * q + 1] = __int_as_float(w.y);
       acc[4 * q + 2] = __int_as_float(w.z); acc[4 * q + 3] = __int_as_float(w.w);
     }
-  } else {                                                   // R3: start from the first contribution
-    int4 w = ld_stream(reinterpret_cast<const char *>(p.src[idx]) + boff);
+  } else {                                                    // R3: start from the first contribution
+    int4 w = ld_stream(reinterpret_cast<const char *>(src[idx]) + boff);
     T::widen(w, acc);
     idx = (idx + 1 == cnt) ? 0 : idx + 1;
     done = 1;
@@ -142,14 +221,14 @@ __device__ __forceinline__ void fold_vector(const FoldParams<MAXN> &p, int64_t t
     int4 buf[kBatch];
     int k = idx;
 #pragma unroll
-    for (int b = 0; b < kBatch; ++b) {                       // all loads of the batch first ...
+    for (int b = 0; b < kBatch; ++b) {                        // all loads of the batch first ...
       if (b < nb) {
-        buf[b] = ld_stream(reinterpret_cast<const char *>(p.src[k]) + boff);
+        buf[b] = ld_stream(reinterpret_cast<const char *>(src[k]) + boff);
         k = (k + 1 == cnt) ? 0 : k + 1;
       }
     }
 #pragma unroll
-    for (int b = 0; b < kBatch; ++b) {                       // ... then the adds, in canonical order
+    for (int b = 0; b < kBatch; ++b) {                        // ... then the adds, in canonical order
       if (b < nb) {
         float x[V];
         T::widen(buf[b], x);
@@ -162,45 +241,50 @@ __device__ __forceinline__ void fold_vector(const FoldParams<MAXN> &p, int64_t t
   }
 }
 
-template <typename T, int MAXN>
-__device__ __forceinline__ float fold_scalar(const FoldParams<MAXN> &p, int64_t t) {
+template <typename T>
+__device__ __forceinline__ float fold_scalar(const FoldSeg &g, const void *const *src, int32_t N, int64_t t) {
   int cnt, idx;
-  if (p.rot) {
-    const uint32_t c = (uint32_t)(p.lo + t) / p.C;
-    idx = (int)(c + 1u == (uint32_t)p.N ? 0u : c + 1u);
-    cnt = p.N;
+  if (g.rot) {
+    const uint32_t c = (uint32_t)(g.lo + t) / g.C;
+    idx = (int)(c + 1u == (uint32_t)N ? 0u : c + 1u);
+    cnt = N;
   } else {
     idx = 0;
-    cnt = p.m;
+    cnt = g.m;
   }
   float s;
   int done = 0;
-  if (p.part_in) {
-    s = p.part_in[t];
+  if (g.part_in) {
+    s = g.part_in[t];
   } else {
-    s = T::load1(p.src[idx], t);
+    s = T::load1(src[idx], t);
     idx = (idx + 1 == cnt) ? 0 : idx + 1;
     done = 1;
   }
   for (; done < cnt; ++done) {
-    s = __fadd_rn(s, T::load1(p.src[idx], t));
+    s = __fadd_rn(s, T::load1(src[idx], t));
     idx = (idx + 1 == cnt) ? 0 : idx + 1;
   }
   return s;
 }
 
-template <typename T, int MAXN>
-__global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams<MAXN> p) {
+template <typename T, int MAXSEG, int MAXSRC>
+__global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams<MAXSEG, MAXSRC> p) {
   constexpr int V = T::kVec;
-  const int64_t nvec = p.n / V;
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  pdl_enter();
+  const int si = find_seg(p.seg, p.nseg, (int)blockIdx.x);
+  const FoldSeg &g = p.seg[si];
+  const int nb = (si + 1 < p.nseg ? p.seg[si + 1].block0 : p.nblocks) - g.block0;
+  const void *const *src = p.src + g.src0;
+  const int64_t nvec = g.n / V;
+  const int64_t stride = (int64_t)nb * blockDim.x;
+  const int64_t gid = (int64_t)(blockIdx.x - g.block0) * blockDim.x + threadIdx.x;
   for (int64_t v = gid; v < nvec; v += stride) {
     const int64_t t = v * V;
     float acc[V];
-    fold_vector<T, MAXN>(p, t, acc);
-    if (p.out_partial) {
-      float *o = reinterpret_cast<float *>(p.out) + t;
+    fold_vector<T>(g, src, p.N, t, acc);
+    if (g.out_partial) {
+      float *o = reinterpret_cast<float *>(g.out) + t;
 #pragma unroll
       for (int q = 0; q < V / 4; ++q)
         st_stream(o + 4 * q, make_int4(__float_as_int(acc[4 * q]), __float_as_int(acc[4 * q + 1]),
@@ -208,124 +292,208 @@ __global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams
     } else {
 #pragma unroll
       for (int e = 0; e < V; ++e) acc[e] = __fmul_rn(acc[e], p.r);   // R5: one rounding
-      st_stream(reinterpret_cast<char *>(p.out) + t * T::kSize, T::narrow(acc));  // R13
+      st_stream(reinterpret_cast<char *>(g.out) + t * T::kSize, T::narrow(acc));  // R13
     }
   }
-  // Ragged tail (< V elements).
-  const int64_t tail0 = nvec * V;
-  if (gid < p.n - tail0) {
+  const int64_t tail0 = nvec * V;                                    // ragged tail (< V elements)
+  if (gid < g.n - tail0) {
     const int64_t t = tail0 + gid;
-    float s = fold_scalar<T, MAXN>(p, t);
-    if (p.out_partial) reinterpret_cast<float *>(p.out)[t] = s;
-    else T::store1(p.out, t, __fmul_rn(s, p.r));
+    const float s = fold_scalar<T>(g, src, p.N, t);
+    if (g.out_partial) reinterpret_cast<float *>(g.out)[t] = s;
+    else T::store1(g.out, t, __fmul_rn(s, p.r));
   }
 }
 
-template <typename T, int MAXN>
-cudaError_t launch_fold_t(const FoldDesc &d, const void *const *src, cudaStream_t s, int bo, int to) {
-  FoldParams<MAXN> p;
-  const int nsrc = d.rot ? d.N : d.m;
-  for (int j = 0; j < nsrc; ++j) p.src[j] = src[j];
-  for (int j = nsrc; j < MAXN; ++j) p.src[j] = nullptr;
-  p.part_in = d.part_in;
-  p.out = d.out;
-  p.lo = d.lo;
-  p.n = d.n;
-  p.N = d.N;
-  p.m = d.m;
-  p.C = d.C;
-  p.rot = d.rot ? 1 : 0;
-  p.out_partial = d.out_partial ? 1 : 0;
-  p.r = d.r;
+template <typename T, int MAXSEG, int MAXSRC>
+cudaError_t launch_fold_group(int32_t N, float r, const FoldSegDesc *d, int nseg, cudaStream_t s, int bo,
+                              int to) {
+  FoldParams<MAXSEG, MAXSRC> p;
+  p.nseg = nseg;
+  p.N = N;
+  p.r = r;
+  int nsrc = 0;
+  std::vector<int64_t> work(nseg);
+  for (int i = 0; i < nseg; ++i) {
+    FoldSeg &g = p.seg[i];
+    const int k = d[i].rot ? N : d[i].m;
+    g.part_in = d[i].part_in;
+    g.out = d[i].out;
+    g.lo = d[i].lo;
+    g.n = d[i].n;
+    g.C = d[i].C;
+    g.rot = d[i].rot ? 1 : 0;
+    g.m = d[i].m;
+    g.src0 = nsrc;
+    g.out_partial = d[i].out_partial ? 1 : 0;
+    for (int j = 0; j < k; ++j) p.src[nsrc + j] = d[i].src[j];
+    nsrc += k;
+    work[i] = (d[i].n + T::kVec - 1) / T::kVec * (int64_t)(k + 1);   // vectors x streams
+  }
   const int threads = to > 0 ? to : 256;
-  const int64_t nvec = d.n / T::kVec;
-  int64_t want = (std::max<int64_t>(nvec, 1) + threads - 1) / threads;
-  int blocks = (int)std::min<int64_t>(want, (int64_t)kSMs * 8);
-  if (bo > 0) blocks = bo;
-  k_fold<T, MAXN><<<blocks, threads, 0, s>>>(p);
-  return cudaGetLastError();
+  int64_t vecs = 0;
+  for (int i = 0; i < nseg; ++i) vecs += (d[i].n + T::kVec - 1) / T::kVec;
+  int total = (int)std::min<int64_t>((vecs + threads - 1) / threads, (int64_t)kSMs * 8);
+  if (bo > 0) total = bo;
+  total = std::max(total, nseg);
+  std::vector<int32_t> block0;
+  split_blocks(work, total, &block0, &p.nblocks);
+  for (int i = 0; i < nseg; ++i) p.seg[i].block0 = block0[i];
+  return launch(k_fold<T, MAXSEG, MAXSRC>, dim3(p.nblocks), dim3(threads), s, p);
 }
 
 template <typename T>
-cudaError_t launch_fold_dt(const FoldDesc &d, const void *const *src, cudaStream_t s, int bo, int to) {
-  const int nsrc = d.rot ? d.N : d.m;
-  if (nsrc <= 8) return launch_fold_t<T, 8>(d, src, s, bo, to);
-  if (nsrc <= 32) return launch_fold_t<T, 32>(d, src, s, bo, to);
-  if (nsrc <= 128) return launch_fold_t<T, 128>(d, src, s, bo, to);
-  return launch_fold_t<T, 1024>(d, src, s, bo, to);
+cudaError_t launch_fold_t(int32_t N, float r, const FoldSegDesc *segs, int nseg, cudaStream_t s, int bo, int to,
+                          int *launches) {
+  constexpr int kSmallSeg = 4, kSmallSrc = 64, kBigSeg = 64, kBigSrc = 1024;
+  int i = 0;
+  while (i < nseg) {
+    int j = i, nsrc = 0;                     // greedy group within the large capacity
+    while (j < nseg) {
+      const int k = segs[j].rot ? N : segs[j].m;
+      if (j - i + 1 > kBigSeg || nsrc + k > kBigSrc) break;
+      nsrc += k;
+      ++j;
+    }
+    if (j == i) return cudaErrorInvalidValue;   // one segment with > 1024 sources (N <= 1024 by contract)
+    cudaError_t e = (j - i <= kSmallSeg && nsrc <= kSmallSrc)
+                        ? launch_fold_group<T, kSmallSeg, kSmallSrc>(N, r, segs + i, j - i, s, bo, to)
+                        : launch_fold_group<T, kBigSeg, kBigSrc>(N, r, segs + i, j - i, s, bo, to);
+    if (e != cudaSuccess) return e;
+    ++*launches;
+    i = j;
+  }
+  return cudaSuccess;
 }
 
 // ---- k_stash ----------------------------------------------------------------
-// Groups of 8 elements: fp32 = 2 vectors, bf16 = 1 vector.  kU groups per
-// thread per iteration, all loads issued before the stores.
+// Each lane moves one "unit" of E elements per access: E = 4 when a cast is
+// involved (fp32 16 B <-> bf16 8 B), else one 16-byte vector.  Consecutive
+// lanes take consecutive units, so every warp-wide load and store covers
+// one contiguous span (fully coalesced).  kU units per thread per
+// iteration, spaced by the segment's grid stride, all loads before stores.
 
-template <typename S, typename D, int kU>
-__global__ void __launch_bounds__(256) k_stash(const void *__restrict__ src, void *__restrict__ dst, int64_t n) {
-  constexpr int kInVec = S::kSize * 8 / 16;    // 16-byte loads per group
-  constexpr int kOutVec = D::kSize * 8 / 16;   // 16-byte stores per group
-  const int64_t ngroups = n / 8;
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  const char *s8 = reinterpret_cast<const char *>(src);
-  char *d8 = reinterpret_cast<char *>(dst);
-  for (int64_t g0 = gid; g0 < ngroups; g0 += stride * kU) {
-    int4 in[kU][kInVec];
+template <int BYTES> struct VecT;
+template <> struct VecT<16> { using T = int4; };
+template <> struct VecT<8> { using T = uint2; };
+
+template <typename S, typename D, int E>
+struct Cast;
+template <> struct Cast<F32T, F32T, 4> {
+  __device__ static __forceinline__ int4 apply(const int4 &v) { return v; }
+};
+template <> struct Cast<BF16T, BF16T, 8> {
+  __device__ static __forceinline__ int4 apply(const int4 &v) { return v; }
+};
+template <> struct Cast<F32T, BF16T, 4> {             // RNE narrowing
+  __device__ static __forceinline__ uint2 apply(const int4 &v) {
+    return make_uint2(BF16T::pack2(__int_as_float(v.x), __int_as_float(v.y)),
+                      BF16T::pack2(__int_as_float(v.z), __int_as_float(v.w)));
+  }
+};
+template <> struct Cast<BF16T, F32T, 4> {             // exact widening
+  __device__ static __forceinline__ int4 apply(const uint2 &v) {
+    float a[4];
+    BF16T::widen2(v.x, a);
+    BF16T::widen2(v.y, a + 2);
+    return make_int4(__float_as_int(a[0]), __float_as_int(a[1]), __float_as_int(a[2]), __float_as_int(a[3]));
+  }
+};
+
+struct StashSeg {
+  const void *src;
+  void *dst;
+  int64_t n;
+  int32_t block0;
+};
+
+template <int MAXSEG>
+struct StashParams {
+  int32_t nseg, nblocks;
+  StashSeg seg[MAXSEG];
+};
+
+template <typename S, typename D, int E, int kU, int MAXSEG>
+__global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashParams<MAXSEG> p) {
+  using In = typename VecT<S::kSize * E>::T;
+  using Out = typename VecT<D::kSize * E>::T;
+  pdl_enter();
+  const int si = find_seg(p.seg, p.nseg, (int)blockIdx.x);
+  const StashSeg &g = p.seg[si];
+  const int nb = (si + 1 < p.nseg ? p.seg[si + 1].block0 : p.nblocks) - g.block0;
+  const In *s = reinterpret_cast<const In *>(g.src);
+  Out *d = reinterpret_cast<Out *>(g.dst);
+  const int64_t nunits = g.n / E;
+  const int64_t stride = (int64_t)nb * blockDim.x;
+  const int64_t gid = (int64_t)(blockIdx.x - g.block0) * blockDim.x + threadIdx.x;
+  for (int64_t u0 = gid; u0 < nunits; u0 += stride * kU) {
+    In in[kU];
 #pragma unroll
     for (int u = 0; u < kU; ++u) {
-      const int64_t g = g0 + u * stride;
-      if (g < ngroups) {
-#pragma unroll
-        for (int q = 0; q < kInVec; ++q) in[u][q] = ld_stream(s8 + g * 8 * S::kSize + q * 16);
-      }
+      const int64_t i = u0 + u * stride;
+      if (i < nunits) in[u] = ld_stream(s + i);
     }
 #pragma unroll
     for (int u = 0; u < kU; ++u) {
-      const int64_t g = g0 + u * stride;
-      if (g < ngroups) {
-        if (S::kSize == D::kSize) {
-#pragma unroll
-          for (int q = 0; q < kInVec; ++q) st_stream(d8 + g * 8 * D::kSize + q * 16, in[u][q]);
-        } else {
-          float a[8];
-#pragma unroll
-          for (int q = 0; q < kInVec; ++q) S::widen(in[u][q], a + q * S::kVec);
-#pragma unroll
-          for (int q = 0; q < kOutVec; ++q) st_stream(d8 + g * 8 * D::kSize + q * 16, D::narrow(a + q * D::kVec));
-        }
-      }
+      const int64_t i = u0 + u * stride;
+      if (i < nunits) st_stream(d + i, Cast<S, D, E>::apply(in[u]));
     }
   }
-  const int64_t tail0 = ngroups * 8;
-  if (gid < n - tail0) {
+  const int64_t tail0 = nunits * E;
+  if (gid < g.n - tail0) {
     const int64_t i = tail0 + gid;
     if (S::kSize == D::kSize) {
-      if (S::kSize == 4) reinterpret_cast<uint32_t *>(dst)[i] = reinterpret_cast<const uint32_t *>(src)[i];
-      else reinterpret_cast<uint16_t *>(dst)[i] = reinterpret_cast<const uint16_t *>(src)[i];
+      if (S::kSize == 4) reinterpret_cast<uint32_t *>(g.dst)[i] = reinterpret_cast<const uint32_t *>(g.src)[i];
+      else reinterpret_cast<uint16_t *>(g.dst)[i] = reinterpret_cast<const uint16_t *>(g.src)[i];
     } else {
-      D::store1(dst, i, S::load1(src, i));
+      D::store1(g.dst, i, S::load1(g.src, i));
     }
   }
 }
 
-template <typename S, typename D>
-cudaError_t launch_stash_t(const void *src, void *dst, int64_t n, cudaStream_t s, int bo, int to) {
-  constexpr int kU = 4;
+template <typename S, typename D, int E>
+cudaError_t launch_stash_t(const StashSegDesc *segs, int nseg, cudaStream_t s, int bo, int to, int *launches) {
+  constexpr int kU = 4, kMaxSeg = 32;
   const int threads = to > 0 ? to : 256;
-  const int64_t groups = std::max<int64_t>(n / 8, 1);
-  int64_t want = (groups + (int64_t)threads * kU - 1) / ((int64_t)threads * kU);
-  int blocks = (int)std::min<int64_t>(std::max<int64_t>(want, 1), (int64_t)kSMs * 8);
-  if (bo > 0) blocks = bo;
-  k_stash<S, D, kU><<<blocks, threads, 0, s>>>(src, dst, n);
-  return cudaGetLastError();
+  for (int i = 0; i < nseg; i += kMaxSeg) {
+    const int k = std::min(kMaxSeg, nseg - i);
+    StashParams<kMaxSeg> p;
+    p.nseg = k;
+    std::vector<int64_t> work(k);
+    int64_t units = 0;
+    for (int j = 0; j < k; ++j) {
+      p.seg[j].src = segs[i + j].src;
+      p.seg[j].dst = segs[i + j].dst;
+      p.seg[j].n = segs[i + j].n;
+      work[j] = (segs[i + j].n + E - 1) / E;
+      units += work[j];
+    }
+    int total = (int)std::min<int64_t>((units + (int64_t)threads * kU - 1) / ((int64_t)threads * kU),
+                                       (int64_t)kSMs * 8);
+    if (bo > 0) total = bo;
+    total = std::max(total, k);
+    std::vector<int32_t> block0;
+    split_blocks(work, total, &block0, &p.nblocks);
+    for (int j = 0; j < k; ++j) p.seg[j].block0 = block0[j];
+    cudaError_t e = launch(k_stash<S, D, E, kU, kMaxSeg>, dim3(p.nblocks), dim3(threads), s, p);
+    if (e != cudaSuccess) return e;
+    ++*launches;
+  }
+  return cudaSuccess;
 }
 
 // ---- k_swap -----------------------------------------------------------------
 
-__global__ void __launch_bounds__(256) k_swap(const SwapEntry *__restrict__ tab, int32_t cur, int32_t next) {
-  const SwapEntry e = tab[blockIdx.y];
+struct SwapParams {
+  const SwapEntry *tab;
+  int32_t cur, next;
+};
+
+__global__ void __launch_bounds__(256) k_swap(const __grid_constant__ SwapParams p) {
+  pdl_enter();
+  const SwapEntry e = p.tab[blockIdx.y];
   unsigned char *live = e.live;
-  unsigned char *sn = e.slot0 + (uint64_t)next * e.stride;
-  unsigned char *sc = cur >= 0 ? e.slot0 + (uint64_t)cur * e.stride : nullptr;
+  unsigned char *sn = e.slot0 + (uint64_t)p.next * e.stride;
+  unsigned char *sc = p.cur >= 0 ? e.slot0 + (uint64_t)p.cur * e.stride : nullptr;
   const uint64_t nw = e.nbytes / 16;
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < nw; w += stride) {
@@ -345,20 +513,36 @@ __global__ void __launch_bounds__(256) k_swap(const SwapEntry *__restrict__ tab,
 
 }  // namespace
 
-cudaError_t launch_fold(es_dtype dtype, const FoldDesc &d, const void *const *src, cudaStream_t s,
-                        int blocks_override, int threads_override) {
-  if (d.n <= 0) return cudaSuccess;
-  if (dtype == ES_BF16) return launch_fold_dt<BF16T>(d, src, s, blocks_override, threads_override);
-  return launch_fold_dt<F32T>(d, src, s, blocks_override, threads_override);
+void set_pdl(bool on) { g_pdl = on; }
+
+cudaError_t launch_fold_multi(es_dtype dtype, int32_t N, float r, const FoldSegDesc *segs, int nseg,
+                              cudaStream_t s, int blocks_override, int threads_override, int *launches) {
+  int dummy = 0;
+  if (!launches) launches = &dummy;
+  std::vector<FoldSegDesc> live;
+  live.reserve(nseg);
+  for (int i = 0; i < nseg; ++i)
+    if (segs[i].n > 0) live.push_back(segs[i]);
+  if (live.empty()) return cudaSuccess;
+  if (dtype == ES_BF16)
+    return launch_fold_t<BF16T>(N, r, live.data(), (int)live.size(), s, blocks_override, threads_override,
+                                launches);
+  return launch_fold_t<F32T>(N, r, live.data(), (int)live.size(), s, blocks_override, threads_override, launches);
 }
 
-cudaError_t launch_stash(const void *src, es_dtype sdt, void *dst, es_dtype ddt, int64_t n, cudaStream_t s,
-                         int bo, int to) {
-  if (n <= 0) return cudaSuccess;
-  if (sdt == ES_F32 && ddt == ES_F32) return launch_stash_t<F32T, F32T>(src, dst, n, s, bo, to);
-  if (sdt == ES_BF16 && ddt == ES_BF16) return launch_stash_t<BF16T, BF16T>(src, dst, n, s, bo, to);
-  if (sdt == ES_F32 && ddt == ES_BF16) return launch_stash_t<F32T, BF16T>(src, dst, n, s, bo, to);
-  return launch_stash_t<BF16T, F32T>(src, dst, n, s, bo, to);
+cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *segs, int nseg, cudaStream_t s,
+                               int bo, int to, int *launches) {
+  int dummy = 0;
+  if (!launches) launches = &dummy;
+  std::vector<StashSegDesc> live;
+  for (int i = 0; i < nseg; ++i)
+    if (segs[i].n > 0) live.push_back(segs[i]);
+  if (live.empty()) return cudaSuccess;
+  const int n = (int)live.size();
+  if (sdt == ES_F32 && ddt == ES_F32) return launch_stash_t<F32T, F32T, 4>(live.data(), n, s, bo, to, launches);
+  if (sdt == ES_BF16 && ddt == ES_BF16) return launch_stash_t<BF16T, BF16T, 8>(live.data(), n, s, bo, to, launches);
+  if (sdt == ES_F32 && ddt == ES_BF16) return launch_stash_t<F32T, BF16T, 4>(live.data(), n, s, bo, to, launches);
+  return launch_stash_t<BF16T, F32T, 4>(live.data(), n, s, bo, to, launches);
 }
 
 cudaError_t launch_swap(const SwapEntry *table_dev, int32_t n, uint64_t max_nbytes, int32_t cur, int32_t next,
@@ -366,9 +550,8 @@ cudaError_t launch_swap(const SwapEntry *table_dev, int32_t n, uint64_t max_nbyt
   if (n <= 0) return cudaSuccess;
   uint64_t words = max_nbytes / 16 + 1;
   int bx = (int)std::min<uint64_t>((words + 255) / 256, 64);
-  dim3 grid(std::max(bx, 1), (unsigned)n);
-  k_swap<<<grid, 256, 0, s>>>(table_dev, cur, next);
-  return cudaGetLastError();
+  SwapParams p{table_dev, cur, next};
+  return launch(k_swap, dim3(std::max(bx, 1), (unsigned)n), dim3(256), s, p);
 }
 
 }  // namespace es

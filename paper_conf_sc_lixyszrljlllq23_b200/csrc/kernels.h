@@ -8,38 +8,46 @@
 
 namespace es {
 
-// Canonical fold over the bucket
-// elements [lo, lo+n).  Every pointer below points at element `lo` of its
-// buffer (physical pointers, 16-byte aligned); lo must be a multiple of 8
-// so that no 16-byte vector straddles a chunk (R1 with A % 8 == 0).
+// One independent fold range over the
+// bucket elements [lo, lo+n).  Every pointer points at element `lo` of its
+// buffer (physical pointers, 16-byte aligned); lo must be a multiple of 8 so
+// that no 16-byte vector straddles a chunk (R1 with A % 8 == 0).
 //   rot == true : per-element canonical rotation -- element i = lo+t lies in
 //                 chunk c = i / C and is folded over src[(c+1)%N], ...,
-//                 src[(c+N)%N]  (src holds N entries indexed by EST)
+//                 src[(c+N)%N]  (src holds N pointers indexed by EST)
 //   rot == false: sources src[0], ..., src[m-1] in that order (one chain
-//                 segment; src already in canonical order)
+//                 segment, already in canonical order)
 //   part_in     : if non-null, the fold continues from this unrounded fp32
-//                 partial instead of starting from its first source
+//                 partial (R14) instead of starting from its first source
 //   out_partial : write the unrounded fp32 sum to `out` (fp32); otherwise
 //                 write round_dtype(fl32(s * r)) to `out` (bucket dtype).
-struct FoldDesc {
+struct FoldSegDesc {
   int64_t lo = 0, n = 0;
-  int32_t N = 1;
+  uint32_t C = 1;
   bool rot = true;
   int32_t m = 0;
-  uint32_t C = 1;
+  const void *const *src = nullptr;   // host array: N (rot) or m pointers
   const float *part_in = nullptr;
   void *out = nullptr;
   bool out_partial = false;
-  float r = 1.0f;
 };
 
-// src: host array of source pointers (N entries if rot, m otherwise).
-cudaError_t launch_fold(es_dtype dtype, const FoldDesc &d, const void *const *src, cudaStream_t s,
-                        int blocks_override, int threads_override);
+// Folds all segments (same dtype, same N) with as few launches as the
+// parameter capacity allows (one for every configuration this build plans
+// for up to 64 segments and 1024 source pointers).  *launches receives the
+// number of kernels enqueued.
+cudaError_t launch_fold_multi(es_dtype dtype, int32_t N, float r, const FoldSegDesc *segs, int nseg,
+                              cudaStream_t s, int blocks_override, int threads_override, int *launches);
 
-// Stash: dst[i] = cast(src[i]) for i < n.
-cudaError_t launch_stash(const void *src, es_dtype sdt, void *dst, es_dtype ddt, int64_t n,
-                         cudaStream_t s, int blocks_override, int threads_override);
+// Stash segments: dst[i] = cast(src[i]) for i < n, all with
+// the same (source dtype, destination dtype).
+struct StashSegDesc {
+  const void *src;
+  void *dst;
+  int64_t n;
+};
+cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *segs, int nseg, cudaStream_t s,
+                               int blocks_override, int threads_override, int *launches);
 
 // Context-switch swap table entry.
 struct SwapEntry {
@@ -51,7 +59,10 @@ struct SwapEntry {
 
 // One launch: for every entry, slot[cur] <- live, live <- slot[next]
 // (cur < 0: load only).  max_nbytes sizes the grid.
-cudaError_t launch_swap(const SwapEntry *table_dev, int32_t n, uint64_t max_nbytes, int32_t cur,
-                        int32_t next, cudaStream_t s);
+cudaError_t launch_swap(const SwapEntry *table_dev, int32_t n, uint64_t max_nbytes, int32_t cur, int32_t next,
+                        cudaStream_t s);
+
+// Programmatic dependent launch (on by default; ES_NO_PDL=1 disables).
+void set_pdl(bool on);
 
 }  // namespace es

@@ -25,7 +25,8 @@ ES_BUF_NONE, ES_BUF_SRC, ES_BUF_STAGE, ES_BUF_PART, ES_BUF_OUT = 0, 1, 2, 3, 4
 
 EXPORTED = [
     "es_workspace_bytes", "es_init", "es_destroy", "es_sync", "es_register_state", "es_init_state",
-    "es_read_state", "es_switch_context", "es_stash_grad", "es_allreduce", "es_chunk_elems",
+    "es_read_state", "es_switch_context", "es_stash_grad", "es_stash_grads", "es_allreduce",
+    "es_allreduce_many", "es_chunk_elems",
     "es_plan_ops", "es_loopback_create", "es_loopback_destroy", "es_profile_enable",
     "es_profile_reset", "es_profile_query", "es_set_launch_override", "es_status_string",
     "es_last_error", "es_abi_version",
@@ -83,6 +84,9 @@ def lib():
         "es_switch_context": (st, [P, i32, P]),
         "es_stash_grad": (st, [P, i32, i32, P, ctypes.c_int, ctypes.c_int, P]),
         "es_allreduce": (st, [P, i32, P, P]),
+        "es_stash_grads": (st, [P, i32, i32, ctypes.POINTER(i32), ctypes.POINTER(P), ctypes.POINTER(ctypes.c_int),
+                                ctypes.c_int, P]),
+        "es_allreduce_many": (st, [P, i32, ctypes.POINTER(i32), ctypes.POINTER(P), P]),
         "es_chunk_elems": (u64, [u64, i32, u32]),
         "es_plan_ops": (st, [cfgp, i32, ctypes.POINTER(i64), sz, ctypes.POINTER(sz), ctypes.POINTER(i32)]),
         "es_loopback_create": (st, [i32, ctypes.POINTER(P)]),
@@ -177,6 +181,21 @@ def es_stash_grad(h, est, bucket, grad_ptr, grad_dtype, mode, stream):
 
 def es_allreduce(h, bucket, out_ptr, stream):
     _check(lib().es_allreduce(h, bucket, ctypes.c_void_p(out_ptr), ctypes.c_void_p(stream)), "es_allreduce")
+
+
+def es_stash_grads(h, est, buckets, grad_ptrs, grad_dtypes, mode, stream):
+    n = len(buckets)
+    b = (ctypes.c_int32 * max(n, 1))(*buckets)
+    g = (ctypes.c_void_p * max(n, 1))(*grad_ptrs)
+    d = (ctypes.c_int * max(n, 1))(*grad_dtypes)
+    _check(lib().es_stash_grads(h, est, n, b, g, d, mode, ctypes.c_void_p(stream)), "es_stash_grads")
+
+
+def es_allreduce_many(h, buckets, out_ptrs, stream):
+    n = len(buckets)
+    b = (ctypes.c_int32 * max(n, 1))(*buckets)
+    o = (ctypes.c_void_p * max(n, 1))(*out_ptrs)
+    _check(lib().es_allreduce_many(h, n, b, o, ctypes.c_void_p(stream)), "es_allreduce_many")
 
 
 def es_chunk_elems(L, N, A=16):

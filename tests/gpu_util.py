@@ -52,7 +52,7 @@ def assert_bits_equal(got, want, what=""):
                              f"got {got[bad[:5]]} want {want[bad[:5]]}")
 
 
-def reduce_g1(xs_per_bucket, A=16, borrow_last=True, override=None, stash_dtypes=None, repeat=1):
+def reduce_g1(xs_per_bucket, A=16, borrow_last=True, override=None, stash_dtypes=None, repeat=1, batched=False):
     """G = 1.  xs_per_bucket: list over buckets of lists over ESTs of arrays.
     stash_dtypes: optional per-bucket dtype of the *gradient* handed to the
     stash (a cast happens when it differs from the bucket dtype)."""
@@ -75,12 +75,19 @@ def reduce_g1(xs_per_bucket, A=16, borrow_last=True, override=None, stash_dtypes
     results = []
     for _ in range(repeat):
         for k in range(N):
+            if batched:
+                mode = es.ES_STASH_BORROW if borrow_last and k == N - 1 else es.ES_STASH_COPY
+                agg.stash_many(k, range(len(buckets)), [devs[b][k] for b in range(len(buckets))], mode)
+                continue
             for b in range(len(buckets)):
                 mode = es.ES_STASH_BORROW if (borrow_last and k == N - 1 and devs[b][k].dtype == outs[b].dtype) \
                     else es.ES_STASH_COPY
                 agg.stash(k, b, devs[b][k], mode)
-        for b in range(len(buckets)):
-            agg.allreduce(b, outs[b])
+        if batched:
+            agg.allreduce_many(range(len(buckets)), outs)
+        else:
+            for b in range(len(buckets)):
+                agg.allreduce(b, outs[b])
         torch.cuda.synchronize()
         agg.sync()
         results.append([from_dev(o) for o in outs])
@@ -88,7 +95,8 @@ def reduce_g1(xs_per_bucket, A=16, borrow_last=True, override=None, stash_dtypes
     return results if repeat > 1 else results[0]
 
 
-def reduce_loopback(xs_per_bucket, G, mapping, sched=es.ES_SCHED_AUTO, A=16, borrow_last=True, steps=1):
+def reduce_loopback(xs_per_bucket, G, mapping, sched=es.ES_SCHED_AUTO, A=16, borrow_last=True, steps=1,
+                    batched=False):
     """G ranks in one process over the LOOPBACK transport, one host thread and
     one CUDA stream per rank, all on the current GPU.  Returns per-rank lists
     of outputs (each rank must hold the full averaged buckets)."""
@@ -112,11 +120,17 @@ def reduce_loopback(xs_per_bucket, G, mapping, sched=es.ES_SCHED_AUTO, A=16, bor
                 for _ in range(steps):
                     loc = a.local_ests
                     for i, k in enumerate(loc):
+                        mode = es.ES_STASH_BORROW if (borrow_last and i == len(loc) - 1) else es.ES_STASH_COPY
+                        if batched:
+                            a.stash_many(k, range(len(buckets)), [devs[b][k] for b in range(len(buckets))], mode)
+                        else:
+                            for b in range(len(buckets)):
+                                a.stash(k, b, devs[b][k], mode)
+                    if batched:
+                        a.allreduce_many(range(len(buckets)), outs[g])
+                    else:
                         for b in range(len(buckets)):
-                            mode = es.ES_STASH_BORROW if (borrow_last and i == len(loc) - 1) else es.ES_STASH_COPY
-                            a.stash(k, b, devs[b][k], mode)
-                    for b in range(len(buckets)):
-                        a.allreduce(b, outs[g][b])
+                            a.allreduce(b, outs[g][b])
         except Exception as e:  # surfaced below
             errors.append((g, e))
 

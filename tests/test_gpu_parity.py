@@ -40,6 +40,30 @@ def test_fold_g1_matches_oracle(N, dtype):
         assert_bits_equal(outs[b], oracle.reduce(xs[b], dtype), f"N={N} L={L} {dtype}")
 
 
+@pytest.mark.parametrize("N", [3, 8, 32])
+def test_batched_api_mixed_dtypes(N):
+    """es_stash_grads / es_allreduce_many: many buckets (mixed fp32 / bf16,
+    ragged, empty) per multi-segment launch give the oracle's bits."""
+    rng = np.random.default_rng(300 + N)
+    Ls = [100003, 16, 0, 17, 65536, 4099, 1, 2049000 // 8]
+    dts = ["f32", "bf16", "f32", "bf16", "bf16", "f32", "f32", "f32"]
+    xs = [_gauss(rng, N, L, d) for L, d in zip(Ls, dts)]
+    for batched in (True, False):
+        outs = reduce_g1(xs, batched=batched)
+        for b, (L, d) in enumerate(zip(Ls, dts)):
+            assert_bits_equal(outs[b], oracle.reduce(xs[b], d), f"batched={batched} N={N} b={b}")
+
+
+def test_batched_launch_shapes():
+    rng = np.random.default_rng(301)
+    xs = [_gauss(rng, 12, L) for L in (50001, 7, 300000, 129)]
+    want = [oracle.reduce(x, "f32") for x in xs]
+    for ov in [(4, 32), (5, 256), (64, 64), (2000, 128), (0, 0)]:
+        outs = reduce_g1(xs, batched=True, override=ov)
+        for b in range(4):
+            assert_bits_equal(outs[b], want[b], f"override {ov} b={b}")
+
+
 @pytest.mark.parametrize("L", [0, 1, 15, 16, 17, 1000003])
 def test_fold_g1_tails(L):
     rng = np.random.default_rng(L)
@@ -217,14 +241,16 @@ def test_bert_uneven_n12_g8_loopback(kind):
             assert_bits_equal(res[g][b], want[b], f"{kind} rank={g} b={b}")
 
 
-def test_loopback_multi_step_reuse():
+@pytest.mark.parametrize("sched", [es.ES_SCHED_CHAIN, es.ES_SCHED_DIRECT])
+@pytest.mark.parametrize("batched", [False, True])
+def test_loopback_multi_step_reuse(sched, batched):
     """Three global steps on the same handles: slot / staging / partial reuse is ordered."""
     rng = np.random.default_rng(13)
-    xs = [_gauss(rng, 8, 50001), _gauss(rng, 8, 70001)]
-    want = [oracle.reduce(x, "f32") for x in xs]
-    res = reduce_loopback(xs, 4, workloads.mapping(8, 4, "random"), es.ES_SCHED_CHAIN, steps=3)
+    xs = [_gauss(rng, 8, 50001), _gauss(rng, 8, 70001), _gauss(rng, 8, 3001, "bf16")]
+    want = [oracle.reduce(x, d) for x, d in zip(xs, ["f32", "f32", "bf16"])]
+    res = reduce_loopback(xs, 4, workloads.mapping(8, 4, "random"), sched, steps=3, batched=batched)
     for g in range(4):
-        for b in range(2):
+        for b in range(3):
             assert_bits_equal(res[g][b], want[b])
 
 
