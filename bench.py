@@ -42,6 +42,8 @@ def parse():
     p.add_argument("--no-graph", action="store_true", help="eager launches instead of one CUDA graph per step")
     p.add_argument("--per-bucket", action="store_true",
                    help="one es_stash_grad / es_allreduce call per bucket (DDP-style) instead of the batched calls")
+    p.add_argument("--no-fuse", action="store_true",
+                   help="separate es_switch_context and es_stash_grads launches instead of es_stash_and_switch")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     p.add_argument("--cpu-seconds", type=float, default=10.0)
@@ -238,8 +240,19 @@ def main():
     flush = None if in_bytes > 2 * L2_BYTES else torch.empty(4 * L2_BYTES, dtype=torch.uint8, device=dev)
     torch.cuda.synchronize()
 
+    fuse = not (args.per_bucket or args.no_fuse)
+
     def step():
-        for i, k in enumerate(local):
+        if fuse:
+            # switch-in of the first local EST, then per EST: stash its
+            # buckets + switch to the next EST in one launch
+            agg.switch(local[0])
+            for i, k in enumerate(local):
+                if i == len(local) - 1:
+                    agg.stash_many(k, range(B), grads[k], es.ES_STASH_BORROW)
+                else:
+                    agg.stash_and_switch(k, range(B), grads[k], local[i + 1], es.ES_STASH_COPY)
+        for i, k in enumerate(local if not fuse else []):
             agg.switch(k)
             mode = es.ES_STASH_BORROW if i == len(local) - 1 else es.ES_STASH_COPY
             if args.per_bucket:
@@ -342,7 +355,7 @@ def main():
         "vs_baseline": None, "dtype": cfg["dtype"], "data": "synthetic",
         "config": {"workload": name, "N": N, "G": G, "mapping": args.mapping, "sched": args.sched,
                    "buckets": B, "elements": sum(n for n, _ in buckets), "graph": graph is not None,
-                   "api": "per-bucket" if args.per_bucket else "batched",
+                   "api": "per-bucket" if args.per_bucket else ("batched" if args.no_fuse else "batched+fused-switch"),
                    "l2": ("inputs larger than L2 (%.1f MB of EST gradients per GPU per step)" % (in_bytes / 1e6))
                    if flush is None else "L2 flushed between timed steps (512 MB write)",
                    "desc": cfg["desc"]},

@@ -193,6 +193,16 @@ es_status es_stash_grad(es_handle h, int32_t est, int32_t bucket, const void *gr
 es_status es_stash_grads(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
                          const es_dtype *grad_dtypes, es_stash_mode mode, es_stream stream);
 
+/* The paper's context switch at a mini-batch boundary: stash
+ * the outgoing local EST `est`'s gradients (n buckets, as es_stash_grads)
+ * AND switch the RNG / BN context to local EST `next_est` (as
+ * es_switch_context) with ONE kernel launch -- the two are independent, so
+ * the swap blocks ride along in the stash grid.  Equivalent to
+ * es_stash_grads(...) followed by es_switch_context(next_est).  next_est must
+ * be a valid local EST (ES_EINVAL / ES_ESTATE otherwise). */
+es_status es_stash_and_switch(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
+                              const es_dtype *grad_dtypes, es_stash_mode mode, int32_t next_est, es_stream stream);
+
 /* ---- aggregation ---------------------------------------------------------- */
 
 /* Collective over the G ranks: every rank calls it for the same bucket

@@ -81,6 +81,9 @@ class Aggregator:
 
     def switch(self, est, stream=None):
         es.es_switch_context(self.h, est, _stream(stream))
+        self._mirror_generator(est)
+
+    def _mirror_generator(self, est):
         if self._gen is not None and est != self._cur:
             if self._cur is not None:
                 self._philox[self._cur] = (self._gen.initial_seed(), self._gen.get_offset())
@@ -97,6 +100,13 @@ class Aggregator:
         """All of EST `est`'s buckets in one call (one multi-segment launch)."""
         es.es_stash_grads(self.h, est, list(buckets), [g.data_ptr() for g in grads],
                           [DTYPES[g.dtype] for g in grads], mode, _stream(stream))
+
+    def stash_and_switch(self, est, buckets, grads, next_est, mode=es.ES_STASH_COPY, stream=None):
+        """EST `est` finished its local step: stash its buckets and switch to
+        `next_est` in one launch."""
+        es.es_stash_and_switch(self.h, est, list(buckets), [g.data_ptr() for g in grads],
+                               [DTYPES[g.dtype] for g in grads], mode, next_est, _stream(stream))
+        self._mirror_generator(next_est)
 
     def allreduce_many(self, buckets, outs, stream=None):
         es.es_allreduce_many(self.h, list(buckets), [o.data_ptr() for o in outs], _stream(stream))

@@ -344,8 +344,12 @@ es_status es_switch_context(es_handle h, int32_t est, es_stream stream) {
 
 // ---- stash ----------------------------------------------------------------------
 
-es_status es_stash_grads(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
-                         const es_dtype *gdts, es_stash_mode mode, es_stream stream) {
+namespace {
+
+// Stash of `n` buckets of local EST `est`, optionally fused with a context
+// switch to local EST `next_est` (-1: no switch) in the same launch.
+es_status stash_impl(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
+                     const es_dtype *gdts, es_stash_mode mode, int32_t next_est, es_stream stream) {
   es_status s = check_handle(h);
   if (s != ES_OK) return s;
   const es::Plan &p = h->plan;
@@ -364,8 +368,29 @@ es_status es_stash_grads(es_handle h, int32_t est, int32_t n, const int32_t *buc
   }
   const int32_t li = p.local_index[est];
   if (li < 0) return set_err(ES_ESTATE, "est is not mapped to this rank");
+  // optional fused context switch
+  es::SwapArgs swap;
+  int32_t next_li = h->cur_local;
+  if (next_est >= 0) {
+    if (next_est >= p.N) return set_err(ES_EINVAL, "next est out of range");
+    next_li = p.local_index[next_est];
+    if (next_li < 0) return set_err(ES_ESTATE, "next est is not mapped to this rank");
+    const int32_t nst = (int32_t)p.state_nbytes.size();
+    if (nst > 0 && !h->state_registered) return set_err(ES_ESTATE, "es_register_state has not been called");
+    if (nst > 0 && next_li != h->cur_local) {
+      swap.tab = reinterpret_cast<const es::SwapEntry *>(h->ws + p.table_off);
+      swap.n = nst;
+      swap.max_nbytes = h->max_state;
+      swap.cur = h->cur_local;
+      swap.next = next_li;
+    }
+  }
+  uint64_t swap_bytes = 0;
+  for (uint64_t b : p.state_nbytes) swap_bytes += b;
+  swap_bytes *= swap.cur >= 0 ? 4 : 2;
   cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
   const unsigned long long cap = capture_id(cs);
+  bool swapped = swap.n == 0;
   if (mode == ES_STASH_COPY) {
     // A slot may be overwritten only after the previous aggregation of its bucket read it.
     for (int32_t i = 0; i < n; ++i) {
@@ -386,13 +411,23 @@ es_status es_stash_grads(es_handle h, int32_t est, int32_t n, const int32_t *buc
           nbytes += b.L * (es::dtype_size(gdts[i]) + b.esize);
         }
         if (segs.empty()) continue;
-        s = h->timed(ES_KERNEL_STASH, nbytes, cs, [&](int *nl) {
+        const es::SwapArgs *sw = swapped ? nullptr : &swap;
+        s = h->timed(ES_KERNEL_STASH, nbytes + (sw ? swap_bytes : 0), cs, [&](int *nl) {
           return es::launch_stash_multi((es_dtype)sd, (es_dtype)dd, segs.data(), (int)segs.size(), cs, h->blocks_ov,
-                                        h->threads_ov, nl);
+                                        h->threads_ov, nl, sw);
         });
         if (s != ES_OK) return s;
+        swapped = true;
       }
   }
+  if (!swapped) {   // BORROW (or nothing to copy): the switch runs alone
+    s = h->timed(ES_KERNEL_SWAP, swap_bytes, cs, [&](int *nl) {
+      *nl = 1;
+      return es::launch_swap(swap.tab, swap.n, swap.max_nbytes, swap.cur, swap.next, cs);
+    });
+    if (s != ES_OK) return s;
+  }
+  h->cur_local = next_li;
   for (int32_t i = 0; i < n; ++i) {
     const size_t k = (size_t)li * h->B + buckets[i];
     h->borrowed[k] = mode == ES_STASH_BORROW ? grads[i] : nullptr;
@@ -403,9 +438,22 @@ es_status es_stash_grads(es_handle h, int32_t est, int32_t n, const int32_t *buc
   return ES_OK;
 }
 
+}  // namespace
+
+es_status es_stash_grads(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
+                         const es_dtype *gdts, es_stash_mode mode, es_stream stream) {
+  return stash_impl(h, est, n, buckets, grads, gdts, mode, -1, stream);
+}
+
+es_status es_stash_and_switch(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
+                              const es_dtype *gdts, es_stash_mode mode, int32_t next_est, es_stream stream) {
+  if (next_est < 0) return set_err(ES_EINVAL, "next_est must be a valid EST (use es_stash_grads to only stash)");
+  return stash_impl(h, est, n, buckets, grads, gdts, mode, next_est, stream);
+}
+
 es_status es_stash_grad(es_handle h, int32_t est, int32_t bucket, const void *grad, es_dtype gdt, es_stash_mode mode,
                         es_stream stream) {
-  return es_stash_grads(h, est, 1, &bucket, &grad, &gdt, mode, stream);
+  return stash_impl(h, est, 1, &bucket, &grad, &gdt, mode, -1, stream);
 }
 
 // ---- aggregation --------------------------------------------------------------------

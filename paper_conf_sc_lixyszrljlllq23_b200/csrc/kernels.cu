@@ -38,6 +38,11 @@ namespace {
 
 constexpr int kSMs = 148;        // B200
 constexpr int kBatch = 8;        // sources loaded per batch in k_fold
+// Grid cap: measured on B200 (scripts/sweep_launch.py, profiles/), near
+// one-shot grids (each thread ~1 vector per segment) stream better than
+// persistent grid-stride ones; 148 x 64 blocks covers every bucket this build
+// plans for, larger ones loop.
+constexpr int kMaxBlocks = kSMs * 64;
 
 bool g_pdl = [] {
   const char *e = std::getenv("ES_NO_PDL");
@@ -332,7 +337,7 @@ cudaError_t launch_fold_group(int32_t N, float r, const FoldSegDesc *d, int nseg
   const int threads = to > 0 ? to : 256;
   int64_t vecs = 0;
   for (int i = 0; i < nseg; ++i) vecs += (d[i].n + T::kVec - 1) / T::kVec;
-  int total = (int)std::min<int64_t>((vecs + threads - 1) / threads, (int64_t)kSMs * 8);
+  int total = (int)std::min<int64_t>((vecs + threads - 1) / threads, (int64_t)kMaxBlocks);
   if (bo > 0) total = bo;
   total = std::max(total, nseg);
   std::vector<int32_t> block0;
@@ -409,22 +414,61 @@ struct StashSeg {
 template <int MAXSEG>
 struct StashParams {
   int32_t nseg, nblocks;
+  // fused context swap: blocks [0, swap_bx * swap_n) swap, the rest stash
+  const SwapEntry *swap_tab;
+  int32_t swap_n, swap_bx, swap_cur, swap_next;
   StashSeg seg[MAXSEG];
 };
+
+// Context swap of table entry `entry` by block `bx` of `nbx` (see k_swap).
+__device__ __forceinline__ void swap_entry(const SwapEntry *tab, int entry, int bx, int nbx, int32_t cur,
+                                           int32_t next) {
+  const SwapEntry e = tab[entry];
+  unsigned char *live = e.live;
+  unsigned char *sn = e.slot0 + (uint64_t)next * e.stride;
+  unsigned char *sc = cur >= 0 ? e.slot0 + (uint64_t)cur * e.stride : nullptr;
+  const uint64_t nw = e.nbytes / 16;
+  const uint64_t stride = (uint64_t)nbx * blockDim.x;
+  for (uint64_t w = (uint64_t)bx * blockDim.x + threadIdx.x; w < nw; w += stride) {
+    // Same thread reads both copies before writing either: no save/load race.
+    int4 a = reinterpret_cast<const int4 *>(live)[w];
+    int4 b = reinterpret_cast<const int4 *>(sn)[w];
+    if (sc) reinterpret_cast<int4 *>(sc)[w] = a;
+    reinterpret_cast<int4 *>(live)[w] = b;
+  }
+  if (bx == 0 && threadIdx.x < e.nbytes - nw * 16) {
+    const uint64_t i = nw * 16 + threadIdx.x;
+    unsigned char a = live[i], b = sn[i];
+    if (sc) sc[i] = a;
+    live[i] = b;
+  }
+}
+
+int swap_blocks_per_entry(uint64_t max_nbytes) {
+  const uint64_t words = max_nbytes / 16 + 1;
+  return (int)std::max<uint64_t>(1, std::min<uint64_t>((words + 255) / 256, 64));
+}
 
 template <typename S, typename D, int E, int kU, int MAXSEG>
 __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashParams<MAXSEG> p) {
   using In = typename VecT<S::kSize * E>::T;
   using Out = typename VecT<D::kSize * E>::T;
   pdl_enter();
-  const int si = find_seg(p.seg, p.nseg, (int)blockIdx.x);
+  const int nswap = p.swap_bx * p.swap_n;
+  if ((int)blockIdx.x < nswap) {
+    swap_entry(p.swap_tab, (int)blockIdx.x / p.swap_bx, (int)blockIdx.x % p.swap_bx, p.swap_bx, p.swap_cur,
+               p.swap_next);
+    return;
+  }
+  const int bid = (int)blockIdx.x - nswap;
+  const int si = find_seg(p.seg, p.nseg, bid);
   const StashSeg &g = p.seg[si];
   const int nb = (si + 1 < p.nseg ? p.seg[si + 1].block0 : p.nblocks) - g.block0;
   const In *s = reinterpret_cast<const In *>(g.src);
   Out *d = reinterpret_cast<Out *>(g.dst);
   const int64_t nunits = g.n / E;
   const int64_t stride = (int64_t)nb * blockDim.x;
-  const int64_t gid = (int64_t)(blockIdx.x - g.block0) * blockDim.x + threadIdx.x;
+  const int64_t gid = (int64_t)(bid - g.block0) * blockDim.x + threadIdx.x;
   for (int64_t u0 = gid; u0 < nunits; u0 += stride * kU) {
     In in[kU];
 #pragma unroll
@@ -451,13 +495,20 @@ __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashPara
 }
 
 template <typename S, typename D, int E>
-cudaError_t launch_stash_t(const StashSegDesc *segs, int nseg, cudaStream_t s, int bo, int to, int *launches) {
+cudaError_t launch_stash_t(const StashSegDesc *segs, int nseg, cudaStream_t s, int bo, int to, int *launches,
+                           const SwapArgs *swap) {
   constexpr int kU = 4, kMaxSeg = 32;
   const int threads = to > 0 ? to : 256;
   for (int i = 0; i < nseg; i += kMaxSeg) {
     const int k = std::min(kMaxSeg, nseg - i);
     StashParams<kMaxSeg> p;
     p.nseg = k;
+    const bool fuse = i == 0 && swap && swap->n > 0;
+    p.swap_tab = fuse ? swap->tab : nullptr;
+    p.swap_n = fuse ? swap->n : 0;
+    p.swap_bx = fuse ? swap_blocks_per_entry(swap->max_nbytes) : 0;
+    p.swap_cur = fuse ? swap->cur : -1;
+    p.swap_next = fuse ? swap->next : 0;
     std::vector<int64_t> work(k);
     int64_t units = 0;
     for (int j = 0; j < k; ++j) {
@@ -468,13 +519,14 @@ cudaError_t launch_stash_t(const StashSegDesc *segs, int nseg, cudaStream_t s, i
       units += work[j];
     }
     int total = (int)std::min<int64_t>((units + (int64_t)threads * kU - 1) / ((int64_t)threads * kU),
-                                       (int64_t)kSMs * 8);
+                                       (int64_t)kMaxBlocks);
     if (bo > 0) total = bo;
     total = std::max(total, k);
     std::vector<int32_t> block0;
     split_blocks(work, total, &block0, &p.nblocks);
     for (int j = 0; j < k; ++j) p.seg[j].block0 = block0[j];
-    cudaError_t e = launch(k_stash<S, D, E, kU, kMaxSeg>, dim3(p.nblocks), dim3(threads), s, p);
+    const int grid = p.nblocks + p.swap_bx * p.swap_n;
+    cudaError_t e = launch(k_stash<S, D, E, kU, kMaxSeg>, dim3(grid), dim3(threads), s, p);
     if (e != cudaSuccess) return e;
     ++*launches;
   }
@@ -490,25 +542,7 @@ struct SwapParams {
 
 __global__ void __launch_bounds__(256) k_swap(const __grid_constant__ SwapParams p) {
   pdl_enter();
-  const SwapEntry e = p.tab[blockIdx.y];
-  unsigned char *live = e.live;
-  unsigned char *sn = e.slot0 + (uint64_t)p.next * e.stride;
-  unsigned char *sc = p.cur >= 0 ? e.slot0 + (uint64_t)p.cur * e.stride : nullptr;
-  const uint64_t nw = e.nbytes / 16;
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < nw; w += stride) {
-    // Same thread reads both copies before writing either: no save/load race.
-    int4 a = reinterpret_cast<const int4 *>(live)[w];
-    int4 b = reinterpret_cast<const int4 *>(sn)[w];
-    if (sc) reinterpret_cast<int4 *>(sc)[w] = a;
-    reinterpret_cast<int4 *>(live)[w] = b;
-  }
-  if (blockIdx.x == 0 && threadIdx.x < e.nbytes - nw * 16) {
-    const uint64_t i = nw * 16 + threadIdx.x;
-    unsigned char a = live[i], b = sn[i];
-    if (sc) sc[i] = a;
-    live[i] = b;
-  }
+  swap_entry(p.tab, (int)blockIdx.y, (int)blockIdx.x, (int)gridDim.x, p.cur, p.next);
 }
 
 }  // namespace
@@ -531,27 +565,33 @@ cudaError_t launch_fold_multi(es_dtype dtype, int32_t N, float r, const FoldSegD
 }
 
 cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *segs, int nseg, cudaStream_t s,
-                               int bo, int to, int *launches) {
+                               int bo, int to, int *launches, const SwapArgs *swap) {
   int dummy = 0;
   if (!launches) launches = &dummy;
   std::vector<StashSegDesc> live;
   for (int i = 0; i < nseg; ++i)
     if (segs[i].n > 0) live.push_back(segs[i]);
-  if (live.empty()) return cudaSuccess;
+  if (live.empty()) {
+    if (swap && swap->n > 0) {
+      ++*launches;
+      return launch_swap(swap->tab, swap->n, swap->max_nbytes, swap->cur, swap->next, s);
+    }
+    return cudaSuccess;
+  }
   const int n = (int)live.size();
-  if (sdt == ES_F32 && ddt == ES_F32) return launch_stash_t<F32T, F32T, 4>(live.data(), n, s, bo, to, launches);
-  if (sdt == ES_BF16 && ddt == ES_BF16) return launch_stash_t<BF16T, BF16T, 8>(live.data(), n, s, bo, to, launches);
-  if (sdt == ES_F32 && ddt == ES_BF16) return launch_stash_t<F32T, BF16T, 4>(live.data(), n, s, bo, to, launches);
-  return launch_stash_t<BF16T, F32T, 4>(live.data(), n, s, bo, to, launches);
+  if (sdt == ES_F32 && ddt == ES_F32) return launch_stash_t<F32T, F32T, 4>(live.data(), n, s, bo, to, launches, swap);
+  if (sdt == ES_BF16 && ddt == ES_BF16)
+    return launch_stash_t<BF16T, BF16T, 8>(live.data(), n, s, bo, to, launches, swap);
+  if (sdt == ES_F32 && ddt == ES_BF16)
+    return launch_stash_t<F32T, BF16T, 4>(live.data(), n, s, bo, to, launches, swap);
+  return launch_stash_t<BF16T, F32T, 4>(live.data(), n, s, bo, to, launches, swap);
 }
 
 cudaError_t launch_swap(const SwapEntry *table_dev, int32_t n, uint64_t max_nbytes, int32_t cur, int32_t next,
                         cudaStream_t s) {
   if (n <= 0) return cudaSuccess;
-  uint64_t words = max_nbytes / 16 + 1;
-  int bx = (int)std::min<uint64_t>((words + 255) / 256, 64);
   SwapParams p{table_dev, cur, next};
-  return launch(k_swap, dim3(std::max(bx, 1), (unsigned)n), dim3(256), s, p);
+  return launch(k_swap, dim3(swap_blocks_per_entry(max_nbytes), (unsigned)n), dim3(256), s, p);
 }
 
 }  // namespace es

@@ -46,9 +46,6 @@ struct StashSegDesc {
   void *dst;
   int64_t n;
 };
-cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *segs, int nseg, cudaStream_t s,
-                               int blocks_override, int threads_override, int *launches);
-
 // Context-switch swap table entry.
 struct SwapEntry {
   unsigned char *live;   // live buffer (16-byte aligned)
@@ -56,6 +53,21 @@ struct SwapEntry {
   uint64_t stride;
   uint64_t nbytes;
 };
+
+// A context swap to fuse into a stash launch (n == 0: none).
+struct SwapArgs {
+  const SwapEntry *tab = nullptr;
+  int32_t n = 0;
+  uint64_t max_nbytes = 0;
+  int32_t cur = -1, next = 0;
+};
+
+// If `swap` has entries, its blocks ride in the first stash launch (the
+// outgoing EST's stash and the context switch are independent), saving one
+// launch per context switch.
+cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *segs, int nseg, cudaStream_t s,
+                               int blocks_override, int threads_override, int *launches,
+                               const SwapArgs *swap = nullptr);
 
 // One launch: for every entry, slot[cur] <- live, live <- slot[next]
 // (cur < 0: load only).  max_nbytes sizes the grid.

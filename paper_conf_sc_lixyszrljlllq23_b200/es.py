@@ -25,7 +25,7 @@ ES_BUF_NONE, ES_BUF_SRC, ES_BUF_STAGE, ES_BUF_PART, ES_BUF_OUT = 0, 1, 2, 3, 4
 
 EXPORTED = [
     "es_workspace_bytes", "es_init", "es_destroy", "es_sync", "es_register_state", "es_init_state",
-    "es_read_state", "es_switch_context", "es_stash_grad", "es_stash_grads", "es_allreduce",
+    "es_read_state", "es_switch_context", "es_stash_grad", "es_stash_grads", "es_stash_and_switch", "es_allreduce",
     "es_allreduce_many", "es_chunk_elems",
     "es_plan_ops", "es_loopback_create", "es_loopback_destroy", "es_profile_enable",
     "es_profile_reset", "es_profile_query", "es_set_launch_override", "es_status_string",
@@ -87,6 +87,8 @@ def lib():
         "es_stash_grads": (st, [P, i32, i32, ctypes.POINTER(i32), ctypes.POINTER(P), ctypes.POINTER(ctypes.c_int),
                                 ctypes.c_int, P]),
         "es_allreduce_many": (st, [P, i32, ctypes.POINTER(i32), ctypes.POINTER(P), P]),
+        "es_stash_and_switch": (st, [P, i32, i32, ctypes.POINTER(i32), ctypes.POINTER(P),
+                                     ctypes.POINTER(ctypes.c_int), ctypes.c_int, i32, P]),
         "es_chunk_elems": (u64, [u64, i32, u32]),
         "es_plan_ops": (st, [cfgp, i32, ctypes.POINTER(i64), sz, ctypes.POINTER(sz), ctypes.POINTER(i32)]),
         "es_loopback_create": (st, [i32, ctypes.POINTER(P)]),
@@ -189,6 +191,15 @@ def es_stash_grads(h, est, buckets, grad_ptrs, grad_dtypes, mode, stream):
     g = (ctypes.c_void_p * max(n, 1))(*grad_ptrs)
     d = (ctypes.c_int * max(n, 1))(*grad_dtypes)
     _check(lib().es_stash_grads(h, est, n, b, g, d, mode, ctypes.c_void_p(stream)), "es_stash_grads")
+
+
+def es_stash_and_switch(h, est, buckets, grad_ptrs, grad_dtypes, mode, next_est, stream):
+    n = len(buckets)
+    b = (ctypes.c_int32 * max(n, 1))(*buckets)
+    g = (ctypes.c_void_p * max(n, 1))(*grad_ptrs)
+    d = (ctypes.c_int * max(n, 1))(*grad_dtypes)
+    _check(lib().es_stash_and_switch(h, est, n, b, g, d, mode, next_est, ctypes.c_void_p(stream)),
+           "es_stash_and_switch")
 
 
 def es_allreduce_many(h, buckets, out_ptrs, stream):

@@ -1,0 +1,79 @@
+"""Summarise ncu outputs into profiles/ (run here, on the CPU box).
+
+  python scripts/ncu_summary.py launches gpurun_out/launches.csv  > profiles/rNN_launches.md
+  python scripts/ncu_summary.py full gpurun_out/prof_fold.ncu-rep  > profiles/rNN_fold_full.md
+
+`launches`: per-kernel count, total and mean device time from an
+`ncu --metrics gpu__time_duration.sum` launch list, and each kernel's share of
+the profiled time (cold-cache, serialised -- compare shares, not absolutes).
+`full`: the key `--set full` metrics per profiled launch (duration, DRAM
+bytes read/written, DRAM throughput, occupancy, registers, stall summary).
+"""
+import collections
+import csv
+import io
+import json
+import subprocess
+import sys
+
+KEYS = [
+    ("gpu__time_duration.sum", "duration"),
+    ("dram__bytes_read.sum", "dram_read"),
+    ("dram__bytes_write.sum", "dram_write"),
+    ("dram__bytes.sum.per_second", "dram_rate"),
+    ("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "dram_pct_peak"),
+    ("lts__t_bytes.sum", "l2_bytes"),
+    ("sm__warps_active.avg.pct_of_peak_sustained_active", "achieved_occupancy_pct"),
+    ("launch__registers_per_thread", "regs"),
+    ("launch__grid_size", "grid"),
+    ("launch__block_size", "block"),
+    ("sm__throughput.avg.pct_of_peak_sustained_elapsed", "sm_pct"),
+    ("smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio", "stall_long_sb"),
+]
+
+
+def _csv_after_header(text):
+    lines = text.splitlines()
+    start = next(i for i, l in enumerate(lines) if l.startswith('"ID"'))
+    return list(csv.DictReader(lines[start:]))
+
+
+def launches(path):
+    rows = _csv_after_header(open(path).read())
+    agg = collections.OrderedDict()
+    for r in rows:
+        if r.get("Metric Name") != "gpu__time_duration.sum":
+            continue
+        name = r["Kernel Name"]
+        short = name.split("(")[0].replace("void ", "")
+        for k in ("k_fold", "k_stash", "k_swap"):
+            if k in short:
+                short = k + ("<bf16>" if "BF16T" in name and k != "k_swap" else "")
+        ns = float(r["Metric Value"]) * (1000.0 if r.get("Metric Unit") == "us" else 1.0)
+        a = agg.setdefault(short, [0, 0.0])
+        a[0] += 1
+        a[1] += ns
+    total = sum(v[1] for v in agg.values()) or 1.0
+    print(f"# ncu launch list: {path}\n")
+    print("| kernel | launches | total us | mean us | share of profiled time |")
+    print("|---|---|---|---|---|")
+    for k, (n, ns) in sorted(agg.items(), key=lambda kv: -kv[1][1]):
+        print(f"| {k} | {n} | {ns / 1e3:.1f} | {ns / n / 1e3:.2f} | {100 * ns / total:.1f} % |")
+
+
+def full(path):
+    out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(io.StringIO(out)))
+    hdr, units = rows[0], rows[1]
+    print(f"# ncu --set full summary: {path}\n")
+    for r in rows[2:]:
+        d = {"kernel": r[hdr.index("Kernel Name")][:90]}
+        for key, nice in KEYS:
+            if key in hdr:
+                i = hdr.index(key)
+                d[nice] = f"{r[i]} {units[i]}".strip()
+        print("```json\n" + json.dumps(d, indent=1) + "\n```")
+
+
+if __name__ == "__main__":
+    {"launches": launches, "full": full}[sys.argv[1]](sys.argv[2])

@@ -47,25 +47,21 @@ def main():
     ms = e0.elapsed_time(e1) / a.reps
     print(json.dumps({"what": "torch_copy", "ms_per_est": round(ms, 4), "GBps": round(2 * tot * esz / ms / 1e6, 1)}))
 
-    shapes = [(0, 0), (148, 256), (296, 256), (592, 256), (1184, 256), (2368, 256), (4736, 256), (148 * 16, 128),
-              (148 * 32, 128), (148 * 4, 512 // 2), (148 * 6, 256), (148 * 12, 256)]
+    shapes = [(0, 0), (592, 256), (1184, 256), (2368, 256), (4736, 256), (9472, 256), (18944, 256), (37888, 256),
+              (9472, 128), (18944, 128), (37888, 128), (37888, 64)]
     for blocks, threads in shapes:
         agg.set_launch_override(blocks, threads)
         for _ in range(2):
             for k in range(N):
-                for b in range(B):
-                    agg.stash(k, b, grads[k][b])
-            for b in range(B):
-                agg.allreduce(b, outs[b])
+                agg.stash_many(k, range(B), grads[k])
+            agg.allreduce_many(range(B), outs)
         torch.cuda.synchronize()
         agg.profile(True)
         agg.profile_reset()
         for _ in range(a.reps):
             for k in range(N):
-                for b in range(B):
-                    agg.stash(k, b, grads[k][b])
-            for b in range(B):
-                agg.allreduce(b, outs[b])
+                agg.stash_many(k, range(B), grads[k])
+            agg.allreduce_many(range(B), outs)
         torch.cuda.synchronize()
         st = agg.profile_query(es.ES_KERNEL_STASH)
         fo = agg.profile_query(es.ES_KERNEL_FOLD)

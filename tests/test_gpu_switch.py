@@ -147,3 +147,51 @@ def test_init_errors():
     assert e.value.status == es.ES_EINVAL
     h = es.es_init(cfg, ws.data_ptr(), nb)
     es.es_destroy(h)
+
+
+def test_stash_and_switch_fused():
+    """es_stash_and_switch == es_stash_grads + es_switch_context: same fold
+    bits (oracle) and same per-EST context (switch model), one launch each."""
+    import oracle
+    from gpu_util import assert_bits_equal, from_dev, to_dev
+    N = 6
+    rng = np.random.default_rng(21)
+    Ls = [70001, 33, 4096]
+    xs = [[(rng.standard_normal(L) * 1e-3).astype(np.float32) for _ in range(N)] for L in Ls]
+    agg = Aggregator(N, 1, 0, [0] * N, [(L, "f32") for L in Ls], state_nbytes=SIZES)
+    live = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in SIZES]
+    agg.register_state(live)
+    init = {k: [rng.integers(0, 256, n, dtype=np.uint8).tobytes() for n in SIZES] for k in range(N)}
+    for k in range(N):
+        for i in range(len(SIZES)):
+            agg.init_state(k, i, init[k][i])
+    model = SwitchModel(N, init)
+    devs = [[to_dev(xs[b][k]) for b in range(len(Ls))] for k in range(N)]
+    outs = [agg.new_out(b) for b in range(len(Ls))]
+    for step in range(3):
+        agg.switch(0)
+        model.switch(0)
+        for k in range(N):
+            nb = rng.integers(0, 256, SIZES[1], dtype=np.uint8)   # EST k's local step updates its BN stats
+            live[1].copy_(torch.from_numpy(nb).cuda())
+            model.mutate(1, nb.tobytes())
+            agg.profile(True)
+            agg.profile_reset()
+            if k < N - 1:
+                agg.stash_and_switch(k, range(len(Ls)), devs[k], k + 1)
+                model.switch(k + 1)
+                n_st, _, _ = agg.profile_query(es.ES_KERNEL_STASH)
+                n_sw, _, _ = agg.profile_query(es.ES_KERNEL_SWAP)
+                assert (n_st, n_sw) == (1, 0)          # one fused launch
+            else:
+                agg.stash_many(k, range(len(Ls)), devs[k], es.ES_STASH_BORROW)
+            agg.profile(False)
+            torch.cuda.synchronize()
+            assert _live_bytes(live) == model.state_of(k + 1 if k < N - 1 else k)
+        agg.allreduce_many(range(len(Ls)), outs)
+        torch.cuda.synchronize()
+        for b in range(len(Ls)):
+            assert_bits_equal(from_dev(outs[b]), oracle.reduce(xs[b], "f32"), f"step {step} b={b}")
+        for k in range(N - 1):
+            assert [agg.read_state(k, i) for i in range(len(SIZES))] == model.state_of(k)
+    agg.close()
