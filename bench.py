@@ -365,6 +365,9 @@ def main():
                      "launches_per_step": int(fl_n / steps_profiled),
                      "avg_launch_us": round(fl_ms / max(fl_n, 1) * 1e3, 2), "peak_source": peak_src},
         "breakdown_ms_per_step": {k: round(v[1] / steps_profiled, 4) for k, v in prof.items()},
+        # SURVEY 8(d)'s narrower metric: es_allreduce time only (stashes already done)
+        "allreduce_only": {"ms": round(fl_ms / steps_profiled, 4),
+                           "GBps": round(payload / (fl_ms / steps_profiled / 1e3) / 1e9, 1) if fl_ms > 0 else None},
         "gpu_launches": int(round(launches_per_step * args.steps)),
         "step_ms_p10_p50_p90": [round(float(np.percentile(step_ms, q)), 4) for q in (10, 50, 90)],
         "clocks": clk,

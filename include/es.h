@@ -73,7 +73,10 @@ typedef enum { ES_F32 = 0, ES_BF16 = 1 } es_dtype;
  * EST, whose gradients are synchronised in place; the buffer
  * must stay unchanged until es_allreduce of that bucket has completed on
  * its stream, and must already hold the bucket dtype. */
-typedef enum { ES_STASH_COPY = 0, ES_STASH_BORROW = 1 } es_stash_mode;
+/* ES_STASH_INPLACE: the gradient was produced directly in the EST's slot
+ * (es_slot_ptr -- DDP bucket views bound to the slot);
+ * `grad` must be that slot pointer; no kernel runs. */
+typedef enum { ES_STASH_COPY = 0, ES_STASH_BORROW = 1, ES_STASH_INPLACE = 2 } es_stash_mode;
 
 /* Exchange schedule for G > 1.  Both produce the
  * same bits; they differ only in NVLink bytes.
@@ -220,6 +223,33 @@ es_status es_allreduce(es_handle h, int32_t bucket, void *out, es_stream stream)
  * buckets of a dtype).  Same argument rules and errors as es_allreduce,
  * checked for every entry before anything is enqueued. */
 es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void *const *outs, es_stream stream);
+
+/* ---- zero-copy slots and elastic resume -------------- */
+
+/* Device pointer of local EST `est`'s slot for `bucket` (bucket dtype,
+ * numel elements, 256-byte aligned, inside the workspace).  A training loop
+ * may bind EST est's gradient bucket there and stash with
+ * ES_STASH_INPLACE: the stash then moves no bytes. */
+es_status es_slot_ptr(es_handle h, int32_t est, int32_t bucket, void **ptr);
+
+/* On-demand checkpoint of one EST's context ("EST
+ * contexts" = RNG / BN state + the gradients already produced in this global
+ * step), so that a job can be resumed on a different G / mapping mid-step
+ * with bit-identical results (D1; synthetic Fig. 9).
+ *   es_context_bytes: size of one exported context for this layout.
+ *   es_export_context: writes local EST `est`'s context to host memory:
+ *     header (layout hash of N, A, bucket numels/dtypes and state sizes --
+ *     the persisted bucket indices of D1), which buckets are stashed, their
+ *     contributions (from slot or borrowed buffer), and the saved (or, for the
+ *     running EST, live) context buffers.  Synchronises `stream`.
+ *   es_import_context: loads such a blob into local EST `est` of this handle
+ *     (any G / mapping with the same N, A and layout; ES_ESTATE if the layout
+ *     hash differs, ES_EINVAL if the blob is malformed).  Stashed buckets
+ *     become stashed here (ordered on `stream`); state goes to the EST's
+ *     slots (and to the live buffers if `est` is the running EST). */
+es_status es_context_bytes(es_handle h, size_t *bytes);
+es_status es_export_context(es_handle h, int32_t est, void *host_dst, size_t bytes, es_stream stream);
+es_status es_import_context(es_handle h, int32_t est, const void *host_src, size_t bytes, es_stream stream);
 
 /* ---- planner introspection (host-only, no CUDA) -------------------------- */
 

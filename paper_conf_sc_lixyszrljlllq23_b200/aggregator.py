@@ -120,6 +120,22 @@ class Aggregator:
         n, d = self.buckets[bucket]
         return torch.empty(n, dtype=TORCH_DTYPES[d], device=self.device)
 
+    # ---- zero-copy slots / elastic resume (NEXT-2) ------------------------------------
+    def slot(self, est, bucket):
+        """Tensor view of local EST `est`'s slot for `bucket` (bind gradients here,
+        then stash with ES_STASH_INPLACE: no bytes move)."""
+        ptr = es.es_slot_ptr(self.h, est, bucket)
+        n, d = self.buckets[bucket]
+        off = ptr - self.workspace.data_ptr()
+        esz = 2 if d == es.ES_BF16 else 4
+        return self.workspace[off:off + n * esz].view(TORCH_DTYPES[d])
+
+    def export_context(self, est, stream=None):
+        return es.es_export_context(self.h, est, _stream(stream))
+
+    def import_context(self, est, blob, stream=None):
+        es.es_import_context(self.h, est, blob, _stream(stream))
+
     def sync(self):
         es.es_sync(self.h)
 

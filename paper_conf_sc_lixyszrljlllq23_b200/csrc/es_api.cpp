@@ -63,6 +63,7 @@ struct es_ctx {
 
   // context state
   bool state_registered = false;
+  std::vector<void *> live_ptr;
   uint64_t max_state = 0;
   int32_t cur_local = -1;
 
@@ -276,6 +277,7 @@ es_status es_register_state(es_handle h, int32_t n, void *const *live) {
   if (n > 0 && cudaMemcpy(h->ws + p.table_off, tab.data(), sizeof(es::SwapEntry) * n, cudaMemcpyHostToDevice) !=
                    cudaSuccess)
     return h->poison(ES_ECUDA, "cudaMemcpy of the swap table failed");
+  h->live_ptr.assign(live, live + n);
   h->state_registered = true;
   return ES_OK;
 }
@@ -355,7 +357,8 @@ es_status stash_impl(es_handle h, int32_t est, int32_t n, const int32_t *buckets
   const es::Plan &p = h->plan;
   if (n < 0 || (n > 0 && (!buckets || !grads || !gdts))) return set_err(ES_EINVAL, "bad bucket/grad arrays");
   if (est < 0 || est >= p.N) return set_err(ES_EINVAL, "est out of range");
-  if (mode != ES_STASH_COPY && mode != ES_STASH_BORROW) return set_err(ES_EINVAL, "bad stash mode");
+  if (mode != ES_STASH_COPY && mode != ES_STASH_BORROW && mode != ES_STASH_INPLACE)
+    return set_err(ES_EINVAL, "bad stash mode");
   for (int32_t i = 0; i < n; ++i) {
     const int32_t bk = buckets[i];
     if (bk < 0 || bk >= h->B) return set_err(ES_EINVAL, "bucket out of range");
@@ -363,11 +366,16 @@ es_status stash_impl(es_handle h, int32_t est, int32_t n, const int32_t *buckets
     const es::BucketPlan &b = p.bp[bk];
     if (b.L > 0 && (!grads[i] || !aligned16(grads[i])))
       return set_err(ES_EINVAL, "grad must be a 16-byte aligned device pointer");
-    if (mode == ES_STASH_BORROW && gdts[i] != b.dtype)
-      return set_err(ES_EINVAL, "BORROW needs grad dtype == bucket dtype");
+    if (mode != ES_STASH_COPY && gdts[i] != b.dtype)
+      return set_err(ES_EINVAL, "BORROW / INPLACE need grad dtype == bucket dtype");
   }
   const int32_t li = p.local_index[est];
   if (li < 0) return set_err(ES_ESTATE, "est is not mapped to this rank");
+  if (mode == ES_STASH_INPLACE)
+    for (int32_t i = 0; i < n; ++i)
+      if (p.bp[buckets[i]].L > 0 &&
+          grads[i] != h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[buckets[i]])
+        return set_err(ES_EINVAL, "INPLACE needs grad == es_slot_ptr(est, bucket)");
   // optional fused context switch
   es::SwapArgs swap;
   int32_t next_li = h->cur_local;
@@ -430,7 +438,7 @@ es_status stash_impl(es_handle h, int32_t est, int32_t n, const int32_t *buckets
   h->cur_local = next_li;
   for (int32_t i = 0; i < n; ++i) {
     const size_t k = (size_t)li * h->B + buckets[i];
-    h->borrowed[k] = mode == ES_STASH_BORROW ? grads[i] : nullptr;
+    h->borrowed[k] = mode == ES_STASH_BORROW ? grads[i] : nullptr;   // INPLACE: the slot itself
     if (cudaEventRecord(h->stash_ev[k], cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaEventRecord failed");
     h->stash_cap[k] = cap;
     h->stashed[k] = 1;
@@ -609,6 +617,184 @@ es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void
 
 es_status es_allreduce(es_handle h, int32_t bucket, void *out, es_stream stream) {
   return es_allreduce_many(h, 1, &bucket, &out, stream);
+}
+
+// ---- zero-copy slots and elastic resume ------------------------------------------
+
+namespace {
+
+struct CtxHeader {
+  char magic[8];           // "ESCTX001"
+  uint32_t version;
+  int32_t N;
+  uint32_t A;
+  int32_t n_buckets;
+  int32_t n_state;
+  int32_t est;
+  uint64_t layout_hash;
+  uint64_t payload_bytes;
+};
+
+uint64_t fnv(uint64_t h, const void *p, size_t n) {
+  const unsigned char *c = reinterpret_cast<const unsigned char *>(p);
+  for (size_t i = 0; i < n; ++i) h = (h ^ c[i]) * 1099511628211ull;
+  return h;
+}
+
+// Hash of the persisted layout (D1): N, A, every bucket's numel and dtype,
+// every context buffer's size.  G and the mapping are deliberately absent.
+uint64_t layout_hash(const es::Plan &p) {
+  uint64_t h = 1469598103934665603ull;
+  h = fnv(h, &p.N, sizeof p.N);
+  h = fnv(h, &p.A, sizeof p.A);
+  for (const es_bucket_desc &b : p.buckets) {
+    h = fnv(h, &b.numel, sizeof b.numel);
+    int32_t d = (int32_t)b.dtype;
+    h = fnv(h, &d, sizeof d);
+  }
+  for (uint64_t n : p.state_nbytes) h = fnv(h, &n, sizeof n);
+  return h;
+}
+
+size_t context_bytes(const es::Plan &p) {
+  size_t n = sizeof(CtxHeader) + ((p.buckets.size() + 7) & ~size_t(7));
+  for (const es::BucketPlan &b : p.bp) n += b.L * b.esize;
+  for (uint64_t s : p.state_nbytes) n += s;
+  return n;
+}
+
+}  // namespace
+
+es_status es_slot_ptr(es_handle h, int32_t est, int32_t bucket, void **ptr) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  const es::Plan &p = h->plan;
+  if (!ptr) return set_err(ES_EINVAL, "ptr is NULL");
+  if (est < 0 || est >= p.N) return set_err(ES_EINVAL, "est out of range");
+  if (bucket < 0 || bucket >= h->B) return set_err(ES_EINVAL, "bucket out of range");
+  const int32_t li = p.local_index[est];
+  if (li < 0) return set_err(ES_ESTATE, "est is not mapped to this rank");
+  *ptr = h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[bucket];
+  return ES_OK;
+}
+
+es_status es_context_bytes(es_handle h, size_t *bytes) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  if (!bytes) return set_err(ES_EINVAL, "bytes is NULL");
+  *bytes = context_bytes(h->plan);
+  return ES_OK;
+}
+
+es_status es_export_context(es_handle h, int32_t est, void *host_dst, size_t bytes, es_stream stream) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  const es::Plan &p = h->plan;
+  if (!host_dst) return set_err(ES_EINVAL, "host_dst is NULL");
+  if (bytes < context_bytes(p)) return set_err(ES_EINVAL, "buffer smaller than es_context_bytes()");
+  if (est < 0 || est >= p.N) return set_err(ES_EINVAL, "est out of range");
+  const int32_t li = p.local_index[est];
+  if (li < 0) return set_err(ES_ESTATE, "est is not mapped to this rank");
+  const int32_t nst = (int32_t)p.state_nbytes.size();
+  if (nst > 0 && !h->state_registered) return set_err(ES_ESTATE, "es_register_state has not been called");
+  cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
+  unsigned char *o = reinterpret_cast<unsigned char *>(host_dst);
+  CtxHeader hd;
+  std::memset(&hd, 0, sizeof hd);
+  std::memcpy(hd.magic, "ESCTX001", 8);
+  hd.version = 1;
+  hd.N = p.N;
+  hd.A = p.A;
+  hd.n_buckets = h->B;
+  hd.n_state = nst;
+  hd.est = est;
+  hd.layout_hash = layout_hash(p);
+  hd.payload_bytes = context_bytes(p);
+  std::memcpy(o, &hd, sizeof hd);
+  unsigned char *mask = o + sizeof hd;
+  size_t off = sizeof hd + ((p.buckets.size() + 7) & ~size_t(7));
+  std::memset(mask, 0, off - sizeof hd);
+  for (int32_t b = 0; b < h->B; ++b) {
+    const es::BucketPlan &bp = p.bp[b];
+    const size_t k = (size_t)li * h->B + b;
+    const size_t nb = bp.L * bp.esize;
+    if (h->stashed[k] && nb > 0) {
+      mask[b] = 1;
+      const void *src = h->borrowed[k] ? h->borrowed[k]
+                                       : (const void *)(h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[b]);
+      if (h->stash_cap[k] == 0 && cudaStreamWaitEvent(cs, h->stash_ev[k], 0) != cudaSuccess)
+        return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
+      if (cudaMemcpyAsync(o + off, src, nb, cudaMemcpyDeviceToHost, cs) != cudaSuccess)
+        return h->poison(ES_ECUDA, "cudaMemcpyAsync D2H of a stashed bucket failed");
+    } else {
+      mask[b] = h->stashed[k] ? 1 : 0;
+      std::memset(o + off, 0, nb);
+    }
+    off += nb;
+  }
+  for (int32_t i = 0; i < nst; ++i) {
+    const void *src = li == h->cur_local ? h->live_ptr[i]
+                                         : (const void *)(h->ws + p.state_area_off + (uint64_t)li * p.state_block +
+                                                          p.state_off[i]);
+    if (cudaMemcpyAsync(o + off, src, p.state_nbytes[i], cudaMemcpyDeviceToHost, cs) != cudaSuccess)
+      return h->poison(ES_ECUDA, "cudaMemcpyAsync D2H of EST state failed");
+    off += p.state_nbytes[i];
+  }
+  if (cudaStreamSynchronize(cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaStreamSynchronize failed");
+  return ES_OK;
+}
+
+es_status es_import_context(es_handle h, int32_t est, const void *host_src, size_t bytes, es_stream stream) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  const es::Plan &p = h->plan;
+  if (!host_src) return set_err(ES_EINVAL, "host_src is NULL");
+  if (bytes < sizeof(CtxHeader)) return set_err(ES_EINVAL, "blob too small");
+  CtxHeader hd;
+  std::memcpy(&hd, host_src, sizeof hd);
+  if (std::memcmp(hd.magic, "ESCTX001", 8) != 0 || hd.version != 1) return set_err(ES_EINVAL, "not an es context blob");
+  if (hd.layout_hash != layout_hash(p) || hd.N != p.N || hd.A != p.A || hd.n_buckets != h->B)
+    return set_err(ES_ESTATE, "context was exported under a different N / A / bucket layout (D1 mismatch)");
+  if (bytes < context_bytes(p) || hd.payload_bytes != context_bytes(p)) return set_err(ES_EINVAL, "blob truncated");
+  if (est < 0 || est >= p.N) return set_err(ES_EINVAL, "est out of range");
+  if (hd.est != est) return set_err(ES_EINVAL, "blob belongs to another EST");
+  const int32_t li = p.local_index[est];
+  if (li < 0) return set_err(ES_ESTATE, "est is not mapped to this rank");
+  const int32_t nst = (int32_t)p.state_nbytes.size();
+  if (nst > 0 && li == h->cur_local && !h->state_registered)
+    return set_err(ES_ESTATE, "es_register_state has not been called");
+  cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
+  const unsigned long long cap = capture_id(cs);
+  const unsigned char *in = reinterpret_cast<const unsigned char *>(host_src);
+  const unsigned char *mask = in + sizeof hd;
+  size_t off = sizeof hd + ((p.buckets.size() + 7) & ~size_t(7));
+  for (int32_t b = 0; b < h->B; ++b) {
+    const es::BucketPlan &bp = p.bp[b];
+    const size_t k = (size_t)li * h->B + b;
+    const size_t nb = bp.L * bp.esize;
+    if (mask[b]) {
+      unsigned char *dst = h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[b];
+      if (h->ar_recorded[b] && h->ar_cap[b] == cap && cudaStreamWaitEvent(cs, h->ar_ev[b], 0) != cudaSuccess)
+        return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
+      if (nb > 0 && cudaMemcpyAsync(dst, in + off, nb, cudaMemcpyHostToDevice, cs) != cudaSuccess)
+        return h->poison(ES_ECUDA, "cudaMemcpyAsync H2D of a stashed bucket failed");
+      h->borrowed[k] = nullptr;
+      if (cudaEventRecord(h->stash_ev[k], cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaEventRecord failed");
+      h->stash_cap[k] = cap;
+      h->stashed[k] = 1;
+    }
+    off += nb;
+  }
+  for (int32_t i = 0; i < nst; ++i) {
+    void *dst = li == h->cur_local ? h->live_ptr[i]
+                                   : (void *)(h->ws + p.state_area_off + (uint64_t)li * p.state_block + p.state_off[i]);
+    if (cudaMemcpyAsync(dst, in + off, p.state_nbytes[i], cudaMemcpyHostToDevice, cs) != cudaSuccess)
+      return h->poison(ES_ECUDA, "cudaMemcpyAsync H2D of EST state failed");
+    off += p.state_nbytes[i];
+  }
+  // host_src may be released by the caller on return
+  if (cudaStreamSynchronize(cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaStreamSynchronize failed");
+  return ES_OK;
 }
 
 // ---- instrumentation ---------------------------------------------------------

@@ -15,7 +15,7 @@ from . import _build
 
 ES_OK, ES_EINVAL, ES_ESTATE, ES_ENOMEM, ES_ECUDA, ES_ENCCL, ES_EUNSUPPORTED = range(7)
 ES_F32, ES_BF16 = 0, 1
-ES_STASH_COPY, ES_STASH_BORROW = 0, 1
+ES_STASH_COPY, ES_STASH_BORROW, ES_STASH_INPLACE = 0, 1, 2
 ES_SCHED_AUTO, ES_SCHED_DIRECT, ES_SCHED_CHAIN = 0, 1, 2
 ES_TRANSPORT_NONE, ES_TRANSPORT_NCCL, ES_TRANSPORT_LOOPBACK = 0, 1, 2
 ES_KERNEL_STASH, ES_KERNEL_FOLD, ES_KERNEL_SWAP = 0, 1, 2
@@ -26,7 +26,8 @@ ES_BUF_NONE, ES_BUF_SRC, ES_BUF_STAGE, ES_BUF_PART, ES_BUF_OUT = 0, 1, 2, 3, 4
 EXPORTED = [
     "es_workspace_bytes", "es_init", "es_destroy", "es_sync", "es_register_state", "es_init_state",
     "es_read_state", "es_switch_context", "es_stash_grad", "es_stash_grads", "es_stash_and_switch", "es_allreduce",
-    "es_allreduce_many", "es_chunk_elems",
+    "es_allreduce_many", "es_chunk_elems", "es_slot_ptr", "es_context_bytes", "es_export_context",
+    "es_import_context",
     "es_plan_ops", "es_loopback_create", "es_loopback_destroy", "es_profile_enable",
     "es_profile_reset", "es_profile_query", "es_set_launch_override", "es_status_string",
     "es_last_error", "es_abi_version",
@@ -90,6 +91,10 @@ def lib():
         "es_stash_and_switch": (st, [P, i32, i32, ctypes.POINTER(i32), ctypes.POINTER(P),
                                      ctypes.POINTER(ctypes.c_int), ctypes.c_int, i32, P]),
         "es_chunk_elems": (u64, [u64, i32, u32]),
+        "es_slot_ptr": (st, [P, i32, i32, ctypes.POINTER(P)]),
+        "es_context_bytes": (st, [P, ctypes.POINTER(sz)]),
+        "es_export_context": (st, [P, i32, P, sz, P]),
+        "es_import_context": (st, [P, i32, P, sz, P]),
         "es_plan_ops": (st, [cfgp, i32, ctypes.POINTER(i64), sz, ctypes.POINTER(sz), ctypes.POINTER(i32)]),
         "es_loopback_create": (st, [i32, ctypes.POINTER(P)]),
         "es_loopback_destroy": (st, [P]),
@@ -207,6 +212,30 @@ def es_allreduce_many(h, buckets, out_ptrs, stream):
     b = (ctypes.c_int32 * max(n, 1))(*buckets)
     o = (ctypes.c_void_p * max(n, 1))(*out_ptrs)
     _check(lib().es_allreduce_many(h, n, b, o, ctypes.c_void_p(stream)), "es_allreduce_many")
+
+
+def es_slot_ptr(h, est, bucket):
+    p = ctypes.c_void_p()
+    _check(lib().es_slot_ptr(h, est, bucket, ctypes.byref(p)), "es_slot_ptr")
+    return p.value
+
+
+def es_context_bytes(h):
+    n = ctypes.c_size_t()
+    _check(lib().es_context_bytes(h, ctypes.byref(n)), "es_context_bytes")
+    return n.value
+
+
+def es_export_context(h, est, stream):
+    n = es_context_bytes(h)
+    buf = ctypes.create_string_buffer(n)
+    _check(lib().es_export_context(h, est, buf, n, ctypes.c_void_p(stream)), "es_export_context")
+    return buf.raw
+
+
+def es_import_context(h, est, blob, stream):
+    buf = ctypes.create_string_buffer(bytes(blob), len(blob))
+    _check(lib().es_import_context(h, est, buf, len(blob), ctypes.c_void_p(stream)), "es_import_context")
 
 
 def es_chunk_elems(L, N, A=16):

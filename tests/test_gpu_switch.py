@@ -195,3 +195,159 @@ def test_stash_and_switch_fused():
         for k in range(N - 1):
             assert [agg.read_state(k, i) for i in range(len(SIZES))] == model.state_of(k)
     agg.close()
+
+
+# ---- NEXT-2: zero-copy stash and elastic resume --------------------------------------------
+
+def test_inplace_stash_moves_no_bytes():
+    import oracle
+    from gpu_util import assert_bits_equal, from_dev
+    N, Ls = 5, [40001, 1000, 7]
+    rng = np.random.default_rng(31)
+    xs = [[(rng.standard_normal(L) * 1e-2).astype(np.float32) for _ in range(N)] for L in Ls]
+    agg = Aggregator(N, 1, 0, [0] * N, [(L, "f32") for L in Ls])
+    for k in range(N):
+        for b in range(len(Ls)):
+            agg.slot(k, b).copy_(torch.from_numpy(xs[b][k]).cuda())   # "backward" writes into the slot
+    agg.profile(True)
+    agg.profile_reset()
+    for k in range(N):
+        agg.stash_many(k, range(len(Ls)), [agg.slot(k, b) for b in range(len(Ls))], es.ES_STASH_INPLACE)
+    assert agg.profile_query(es.ES_KERNEL_STASH)[0] == 0
+    outs = [agg.new_out(b) for b in range(len(Ls))]
+    agg.allreduce_many(range(len(Ls)), outs)
+    torch.cuda.synchronize()
+    for b in range(len(Ls)):
+        assert_bits_equal(from_dev(outs[b]), oracle.reduce(xs[b], "f32"))
+    with pytest.raises(es.EsError) as e:       # INPLACE must name the slot itself
+        agg.stash(0, 0, torch.zeros(Ls[0], device="cuda"), es.ES_STASH_INPLACE)
+    assert e.value.status == es.ES_EINVAL
+    agg.close()
+
+
+def _threads(G, fn):
+    import threading
+    errs = []
+    dev = torch.cuda.current_device()
+
+    def run(g):
+        try:
+            torch.cuda.set_device(dev)
+            fn(g)
+        except Exception as ex:
+            errs.append(ex)
+    ts = [threading.Thread(target=run, args=(g,)) for g in range(G)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join(timeout=300)
+    torch.cuda.synchronize()
+    if errs:
+        raise errs[0]
+
+
+def test_elastic_resume_mid_step_fig9():
+    """Synthetic Fig. 9: a global step starts on G=4, is
+    revoked after 5 of 8 ESTs ran (on-demand checkpoint of every EST context,
+    P:608-624), resumes on G=2 with another mapping, and the next step runs on
+    G=3 unevenly.  Every aggregate equals the oracle (and hence G=1) bit for
+    bit, and every EST's context continues unchanged (D1)."""
+    import oracle
+    from gpu_util import assert_bits_equal, from_dev, to_dev
+    from paper_conf_sc_lixyszrljlllq23_b200 import workloads as wl
+    N, Ls, dts = 8, [30011, 4096, 9], ["f32", "bf16", "f32"]
+    rng = np.random.default_rng(41)
+
+    def data():
+        out = []
+        for L, d in zip(Ls, dts):
+            row = [(rng.standard_normal(L) * 1e-3).astype(np.float32) for _ in range(N)]
+            out.append(row if d == "f32" else [oracle.f32_to_bf16_bits(x) for x in row])
+        return out
+
+    init = {k: [rng.integers(0, 256, n, dtype=np.uint8).tobytes() for n in SIZES] for k in range(N)}
+
+    def stage(G, mapping):
+        world = es.es_loopback_create(G)
+        aggs = [Aggregator(N, G, g, mapping, list(zip(Ls, dts)), state_nbytes=SIZES,
+                           transport=es.ES_TRANSPORT_LOOPBACK, comm=world.value) for g in range(G)]
+        lives = []
+        for a in aggs:
+            live = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in SIZES]
+            a.register_state(live)
+            lives.append(live)
+        return world, aggs, lives
+
+    def allreduce(G, aggs):
+        outs = [[a.new_out(b) for b in range(len(Ls))] for a in aggs]
+        streams = [torch.cuda.Stream() for _ in range(G)]
+        torch.cuda.synchronize()
+
+        def fn(g):
+            with torch.cuda.stream(streams[g]):
+                aggs[g].allreduce_many(range(len(Ls)), outs[g])
+        _threads(G, fn)
+        return outs
+
+    def check(outs, xs, what):
+        for g, row in enumerate(outs):
+            for b in range(len(Ls)):
+                assert_bits_equal(from_dev(row[b]), oracle.reduce(xs[b], dts[b]), f"{what} rank {g} bucket {b}")
+
+    # stage 0: G=4 contiguous; one full step
+    m0 = wl.mapping(N, 4, "contiguous")
+    w0, aggs0, _ = stage(4, m0)
+    for k in range(N):
+        for i in range(len(SIZES)):
+            aggs0[m0[k]].init_state(k, i, init[k][i])
+    x1 = data()
+    d1 = [[to_dev(x1[b][k]) for b in range(len(Ls))] for k in range(N)]
+    for k in range(N):
+        aggs0[m0[k]].stash_many(k, range(len(Ls)), d1[k])
+    check(allreduce(4, aggs0), x1, "stage0 step1")
+    # step 2 starts: ESTs 0..4 run (stash), then the job is revoked
+    x2 = data()
+    d2 = [[to_dev(x2[b][k]) for b in range(len(Ls))] for k in range(N)]
+    for k in range(5):
+        aggs0[m0[k]].stash_many(k, range(len(Ls)), d2[k],
+                                es.ES_STASH_BORROW if k == 4 else es.ES_STASH_COPY)
+    torch.cuda.synchronize()
+    blobs = {k: aggs0[m0[k]].export_context(k) for k in range(N)}
+    for a in aggs0:
+        a.close()
+    es.es_loopback_destroy(w0)
+
+    # stage 1: G=2 round robin; resume mid-step
+    m1 = wl.mapping(N, 2, "round_robin")
+    w1, aggs1, _ = stage(2, m1)
+    for k in range(N):
+        aggs1[m1[k]].import_context(k, blobs[k])
+    for k in range(5, N):
+        aggs1[m1[k]].stash_many(k, range(len(Ls)), d2[k])
+    check(allreduce(2, aggs1), x2, "stage1 resumed step2")
+    for k in range(N):                               # contexts survived the move
+        assert [aggs1[m1[k]].read_state(k, i) for i in range(len(SIZES))] == init[k]
+    blobs = {k: aggs1[m1[k]].export_context(k) for k in range(N)}
+    for a in aggs1:
+        a.close()
+    es.es_loopback_destroy(w1)
+
+    # stage 2: G=3 uneven random mapping; a fresh step
+    m2 = wl.mapping(N, 3, "random", seed=3)
+    w2, aggs2, _ = stage(3, m2)
+    for k in range(N):
+        aggs2[m2[k]].import_context(k, blobs[k])
+    x3 = data()
+    d3 = [[to_dev(x3[b][k]) for b in range(len(Ls))] for k in range(N)]
+    for k in range(N):
+        aggs2[m2[k]].stash_many(k, range(len(Ls)), d3[k])
+    check(allreduce(3, aggs2), x3, "stage2 step3")
+    # a layout change is refused (D0 failure mode, P:1058-1065)
+    other = Aggregator(N, 1, 0, [0] * N, [(L + 16, d) for L, d in zip(Ls, dts)], state_nbytes=SIZES)
+    with pytest.raises(es.EsError) as e:
+        other.import_context(0, blobs[0])
+    assert e.value.status == es.ES_ESTATE
+    other.close()
+    for a in aggs2:
+        a.close()
+    es.es_loopback_destroy(w2)
