@@ -43,6 +43,10 @@ def lib():
         L.es_oracle_reduce.argtypes = [ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
                                        ctypes.POINTER(ctypes.c_void_p), ctypes.c_int64, ctypes.c_int64,
                                        ctypes.c_void_p]
+        L.es_oracle_reduce_ex.restype = ctypes.c_int
+        L.es_oracle_reduce_ex.argtypes = [ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
+                                          ctypes.c_uint32, ctypes.POINTER(ctypes.c_void_p), ctypes.c_int64,
+                                          ctypes.c_int64, ctypes.c_void_p]
         L.es_oracle_stash.restype = ctypes.c_int
         L.es_oracle_stash.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p, ctypes.c_int32,
                                       ctypes.c_int64]
@@ -89,6 +93,27 @@ def reduce(xs, dtype, L=None, A=16, first=0):
                                 out.ctypes.data)
     if rc != 0:
         raise ValueError("es_oracle_reduce: bad arguments")
+    return out
+
+
+COMPAT_PREDIV, COMPAT_PREMUL, COMPAT_BF16HOP = 1, 2, 4
+
+
+def reduce_ex(xs, dtype, compat, L=None, A=16, first=0):
+    """NEXT-3 compatibility variants (pre-divide, pre-multiply, per-hop bf16
+    rounding) in the same canonical order; compat=0 equals reduce()."""
+    code = _code(dtype)
+    N = len(xs)
+    xs = [np.ascontiguousarray(x) for x in xs]
+    count = xs[0].size
+    if L is None:
+        L = first + count
+    out = np.empty(count, dtype=xs[0].dtype)
+    ptrs = (ctypes.c_void_p * N)(*[x.ctypes.data for x in xs])
+    rc = lib().es_oracle_reduce_ex(N, int(L), int(A), code, int(compat), ptrs, int(first), int(count),
+                                   out.ctypes.data)
+    if rc != 0:
+        raise ValueError("es_oracle_reduce_ex: bad arguments")
     return out
 
 

@@ -144,3 +144,53 @@ int es_oracle_stash(const void *src, int32_t src_dtype, void *dst, int32_t dst_d
     }
     return 0;
 }
+
+/* ------------------------------------------------------------------ */
+/* NEXT-3 compatibility variants   */
+/* ------------------------------------------------------------------ */
+
+#define ORACLE_COMPAT_PREDIV 1u   /* each contribution divided by N first (DDP 1.8 div_ before all-reduce) */
+#define ORACLE_COMPAT_PREMUL 2u   /* each contribution multiplied by fl32(1/N) first (NCCL ncclAvg PreMulSum) */
+#define ORACLE_COMPAT_BF16HOP 4u  /* bf16 buckets: every stored intermediate rounded to bf16 (NCCL bf16 ring) */
+
+static float round_bf16(float v) { return es_oracle_bf16_to_f32(es_oracle_f32_to_bf16(v)); }
+
+/*
+ * Same canonical order (R1-R3) as es_oracle_reduce; only the arithmetic of
+ * each step changes with `compat`:
+ *   v_k = widen(x[k][i]); if PREDIV: v_k = fl32(v_k / N); if PREMUL:
+ *   v_k = fl32(v_k * r); if BF16HOP (bf16 only): v_k = bf16(v_k);
+ *   s = v_first; s = fl32(s + v_k) [then bf16(s) if BF16HOP]; finally, if no
+ *   pre-scale, s = fl32(s * r); out = round_to_dtype(s).
+ * compat == 0 gives exactly es_oracle_reduce.
+ */
+int es_oracle_reduce_ex(int32_t N, int64_t L, int32_t A, int32_t dtype, uint32_t compat,
+                        const void *const *x, int64_t first, int64_t count, void *out)
+{
+    if (N <= 0 || A <= 0 || L < 0 || first < 0 || count < 0 || first + count > L) return -1;
+    if (dtype != ORACLE_F32 && dtype != ORACLE_BF16) return -1;
+    if (compat & ~7u) return -1;
+    if ((compat & ORACLE_COMPAT_PREDIV) && (compat & ORACLE_COMPAT_PREMUL)) return -1;
+    if (count == 0) return 0;
+    const int hop = (compat & ORACLE_COMPAT_BF16HOP) && dtype == ORACLE_BF16;
+    const int pre = (compat & (ORACLE_COMPAT_PREDIV | ORACLE_COMPAT_PREMUL)) != 0;
+    const int64_t C = es_oracle_chunk_elems(L, N, A);
+    const float r = 1.0f / (float)N;
+    for (int64_t i = first; i < first + count; ++i) {
+        const int64_t c = i / C;
+        float s = 0.0f;
+        for (int32_t j = 1; j <= N; ++j) {
+            const int32_t k = (int32_t)((c + j) % N);
+            float v = load_widened(x[k], dtype, i - first);
+            if (compat & ORACLE_COMPAT_PREDIV) v = v / (float)N;
+            if (compat & ORACLE_COMPAT_PREMUL) v = v * r;
+            if (hop) v = round_bf16(v);
+            if (j == 1) s = v;
+            else s = s + v;
+            if (hop) s = round_bf16(s);
+        }
+        if (!pre) s = s * r;
+        store_rounded(out, dtype, i - first, s);
+    }
+    return 0;
+}

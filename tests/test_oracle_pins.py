@@ -307,3 +307,66 @@ def test_stash_bf16_to_f32_is_exact_and_identity():
     x = np.random.default_rng(0).standard_normal(1000).astype(np.float32)
     assert np.all(_bits(oracle.stash(x, "f32", "f32")) == _bits(x))
     assert np.all(oracle.stash(allb, "bf16", "bf16") == allb)
+
+
+# ---- NEXT-3 compatibility variants (oracle.reduce_ex) ------------------------------------------
+
+def test_compat_zero_is_canonical():
+    rng = np.random.default_rng(50)
+    for N in (3, 8, 12):
+        xs = [rng.standard_normal(777).astype(np.float32) for _ in range(N)]
+        assert np.all(_bits(oracle.reduce_ex(xs, "f32", 0)) == _bits(oracle.reduce(xs, "f32")))
+        xb = [oracle.f32_to_bf16_bits(x) for x in xs]
+        assert np.all(oracle.reduce_ex(xb, "bf16", 0) == oracle.reduce(xb, "bf16"))
+
+
+def test_compat_prescale_power_of_two_identity():
+    """For N = 2^k, dividing or multiplying by 1/N is exact (normal range), so
+    pre-divide == pre-multiply == post-scale bit for bit."""
+    rng = np.random.default_rng(51)
+    for N in (2, 4, 8, 16, 32):
+        xs = [(rng.standard_normal(1000) * 1e-3).astype(np.float32) for _ in range(N)]
+        want = _bits(oracle.reduce(xs, "f32"))
+        assert np.all(_bits(oracle.reduce_ex(xs, "f32", oracle.COMPAT_PREDIV)) == want)
+        assert np.all(_bits(oracle.reduce_ex(xs, "f32", oracle.COMPAT_PREMUL)) == want)
+
+
+def test_compat_prescale_closed_forms_n12():
+    N, L = 12, 512
+    rng = np.random.default_rng(52)
+    r = np.float32(1) / np.float32(N)
+    # multiples of 12: x/12 is an exact integer, every sum exact -> S/12
+    ints = [rng.integers(-1000, 1001, L) * 12 for _ in range(N)]
+    xs = [i.astype(np.float32) for i in ints]
+    S = np.sum(np.stack(ints), 0) // 12
+    assert np.all(_bits(oracle.reduce_ex(xs, "f32", oracle.COMPAT_PREDIV)) == _bits(S.astype(np.float32)))
+    # one non-zero contribution per element: the fold adds +0s only
+    v = (rng.standard_normal(L) * 3).astype(np.float32)
+    xs = [np.zeros(L, np.float32) for _ in range(N)]
+    xs[5] = v
+    assert np.all(_bits(oracle.reduce_ex(xs, "f32", oracle.COMPAT_PREDIV)) == _bits(v / np.float32(N)))
+    assert np.all(_bits(oracle.reduce_ex(xs, "f32", oracle.COMPAT_PREMUL)) == _bits(v * r))
+    assert np.any(_bits(v / np.float32(N)) != _bits(v * r))          # the two conventions do differ
+
+
+def test_compat_bf16_hop_witness(golden_dir):
+    g = json.load(open(os.path.join(golden_dir, "bf16_hop.json")))
+    C = g["L"] // g["N"]
+    xs = [_bf16_bits_torch(np.full(g["L"], _f(v), dtype=np.float32)) for v in g["x"]]
+    hop = oracle.bf16_bits_to_f32(oracle.reduce_ex(xs, "bf16", oracle.COMPAT_BF16HOP, A=g["A"]))
+    acc = oracle.bf16_bits_to_f32(oracle.reduce(xs, "bf16", A=g["A"]))
+    for c in range(g["N"]):
+        assert np.all(hop[c * C:(c + 1) * C] == np.float32(float(g["out_per_chunk"][c]))), c
+        assert np.all(acc[c * C:(c + 1) * C] == np.float32(float(g["canonical_fp32_accumulate_per_chunk"][c]))), c
+
+
+def test_compat_bf16_hop_exact_when_partials_representable():
+    """Small integers whose every partial sum fits bf16's 8-bit significand:
+    per-hop rounding changes nothing."""
+    rng = np.random.default_rng(53)
+    N = 8
+    ints = [rng.integers(-15, 16, 333) for _ in range(N)]       # |partial| <= 120 < 256
+    xs = [_bf16_bits_torch(i.astype(np.float32)) for i in ints]
+    assert np.all(oracle.reduce_ex(xs, "bf16", oracle.COMPAT_BF16HOP) == oracle.reduce(xs, "bf16"))
+    assert np.all(oracle.reduce_ex(xs, "bf16", oracle.COMPAT_BF16HOP | oracle.COMPAT_PREMUL)
+                  == oracle.reduce(xs, "bf16"))                   # N = 8: 1/8 scaling exact too
