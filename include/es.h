@@ -127,7 +127,22 @@ typedef struct {
   es_transport transport;
   void *comm;                     /* ncclComm_t (NCCL), es_loopback world (LOOPBACK), NULL (NONE) */
   es_sched sched;
+  uint32_t compat;                /* 0 = the canonical definition (R1-R6, R13); else ES_COMPAT_*
+                                     bits.  Part of the persisted definition. */
 } es_config;
+
+/* NEXT-3 compatibility variants -- same canonical order, different step
+ * arithmetic:
+ *   PREDIV:   each contribution is divided by N first (PyTorch 1.8 DDP's
+ *             div_ before the all-reduce); no post-scale.
+ *   PREMUL:   each contribution is multiplied by fl32(1/N) first (NCCL
+ *             ncclAvg / PreMulSum); no post-scale.  Exclusive with PREDIV.
+ *   BF16_HOP: bf16 buckets only: every stored intermediate (scaled
+ *             contribution, partial sum) is rounded to bf16, as an NCCL bf16
+ *             ring stores it between hops.  Ignored for fp32 buckets. */
+#define ES_COMPAT_PREDIV 1u
+#define ES_COMPAT_PREMUL 2u
+#define ES_COMPAT_BF16_HOP 4u
 
 /* ---- sizing / lifetime --------------------------------------------------- */
 

@@ -37,12 +37,12 @@ class Aggregator:
     """
 
     def __init__(self, N, G, rank, est_to_gpu, buckets, chunk_align=16, state_nbytes=(),
-                 transport=None, comm=None, sched=es.ES_SCHED_AUTO, device=None):
+                 transport=None, comm=None, sched=es.ES_SCHED_AUTO, device=None, compat=0):
         if transport is None:
             transport = es.ES_TRANSPORT_NONE if G == 1 else es.ES_TRANSPORT_NCCL
         self.buckets = [(int(n), DTYPES[d]) for n, d in buckets]
         self.cfg = es.Config(N, G, rank, est_to_gpu, self.buckets, chunk_align, tuple(state_nbytes),
-                             transport, comm, sched)
+                             transport, comm, sched, compat)
         self.N, self.G, self.rank = N, G, rank
         self.local_ests = [e for e in range(N) if est_to_gpu[e] == rank]
         self.device = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())

@@ -513,8 +513,8 @@ es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void
     if (pend.empty()) return ES_OK;
     for (size_t i = 0; i < pend.size(); ++i) pend[i].src = pend_src[i].data();
     es_status st = h->timed(ES_KERNEL_FOLD, pend_bytes, cs, [&](int *nl) {
-      return es::launch_fold_multi(pend_dt, p.N, r, pend.data(), (int)pend.size(), cs, h->blocks_ov, h->threads_ov,
-                                   nl);
+      return es::launch_fold_multi(pend_dt, p.N, r, p.compat, pend.data(), (int)pend.size(), cs, h->blocks_ov,
+                                   h->threads_ov, nl);
     });
     pend.clear();
     pend_src.clear();
@@ -653,6 +653,7 @@ uint64_t layout_hash(const es::Plan &p) {
     h = fnv(h, &d, sizeof d);
   }
   for (uint64_t n : p.state_nbytes) h = fnv(h, &n, sizeof n);
+  h = fnv(h, &p.compat, sizeof p.compat);
   return h;
 }
 

@@ -187,14 +187,40 @@ template <int MAXSEG, int MAXSRC>
 struct FoldParams {
   int32_t nseg, N, nblocks;
   float r;
+  uint32_t compat;        // NEXT-3 variant bits (COMPAT kernels only)
   FoldSeg seg[MAXSEG];
   const void *src[MAXSRC];
 };
 
+// NEXT-3 compatibility variants: the
+// canonical order is unchanged; only each step's arithmetic differs.
+constexpr uint32_t kPreDiv = 1, kPreMul = 2, kBf16Hop = 4;
+
+__device__ __forceinline__ float round_bf16(float v) { return __bfloat162float(__float2bfloat16_rn(v)); }
+
+// A widened contribution as the variant sees it (pre-scale, bf16 storage).
+template <bool COMPAT>
+__device__ __forceinline__ float prep(float v, uint32_t compat, float r, float fN) {
+  if (COMPAT) {
+    if (compat & kPreDiv) v = __fdiv_rn(v, fN);
+    if (compat & kPreMul) v = __fmul_rn(v, r);
+    if (compat & kBf16Hop) v = round_bf16(v);
+  }
+  return v;
+}
+
+template <bool COMPAT>
+__device__ __forceinline__ float add_step(float s, float v, uint32_t compat) {
+  s = __fadd_rn(s, v);
+  if (COMPAT && (compat & kBf16Hop)) s = round_bf16(s);
+  return s;
+}
+
 // Fold of one 16-byte vector at segment offset t (elements), into acc[V].
-template <typename T>
+template <typename T, bool COMPAT>
 __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const *src, int32_t N, int64_t t,
-                                            float *acc) {
+                                            float *acc, uint32_t compat, float r) {
+  const float fN = (float)N;
   constexpr int V = T::kVec;
   int cnt, idx;
   if (g.rot) {
@@ -218,6 +244,8 @@ __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const 
   } else {                                                    // R3: start from the first contribution
     int4 w = ld_stream(reinterpret_cast<const char *>(src[idx]) + boff);
     T::widen(w, acc);
+#pragma unroll
+    for (int e = 0; e < V; ++e) acc[e] = prep<COMPAT>(acc[e], compat, r, fN);
     idx = (idx + 1 == cnt) ? 0 : idx + 1;
     done = 1;
   }
@@ -238,7 +266,7 @@ __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const 
         float x[V];
         T::widen(buf[b], x);
 #pragma unroll
-        for (int e = 0; e < V; ++e) acc[e] = __fadd_rn(acc[e], x[e]);
+        for (int e = 0; e < V; ++e) acc[e] = add_step<COMPAT>(acc[e], prep<COMPAT>(x[e], compat, r, fN), compat);
       }
     }
     idx = k;
@@ -246,8 +274,10 @@ __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const 
   }
 }
 
-template <typename T>
-__device__ __forceinline__ float fold_scalar(const FoldSeg &g, const void *const *src, int32_t N, int64_t t) {
+template <typename T, bool COMPAT>
+__device__ __forceinline__ float fold_scalar(const FoldSeg &g, const void *const *src, int32_t N, int64_t t,
+                                             uint32_t compat, float r) {
+  const float fN = (float)N;
   int cnt, idx;
   if (g.rot) {
     const uint32_t c = (uint32_t)(g.lo + t) / g.C;
@@ -262,20 +292,22 @@ __device__ __forceinline__ float fold_scalar(const FoldSeg &g, const void *const
   if (g.part_in) {
     s = g.part_in[t];
   } else {
-    s = T::load1(src[idx], t);
+    s = prep<COMPAT>(T::load1(src[idx], t), compat, r, fN);
     idx = (idx + 1 == cnt) ? 0 : idx + 1;
     done = 1;
   }
   for (; done < cnt; ++done) {
-    s = __fadd_rn(s, T::load1(src[idx], t));
+    s = add_step<COMPAT>(s, prep<COMPAT>(T::load1(src[idx], t), compat, r, fN), compat);
     idx = (idx + 1 == cnt) ? 0 : idx + 1;
   }
   return s;
 }
 
-template <typename T, int MAXSEG, int MAXSRC>
+template <typename T, int MAXSEG, int MAXSRC, bool COMPAT>
 __global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams<MAXSEG, MAXSRC> p) {
   constexpr int V = T::kVec;
+  // post-scale unless a pre-scale variant already applied 1/N (R5 vs NEXT-3)
+  const bool post = !COMPAT || !(p.compat & (kPreDiv | kPreMul));
   pdl_enter();
   const int si = find_seg(p.seg, p.nseg, (int)blockIdx.x);
   const FoldSeg &g = p.seg[si];
@@ -287,7 +319,7 @@ __global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams
   for (int64_t v = gid; v < nvec; v += stride) {
     const int64_t t = v * V;
     float acc[V];
-    fold_vector<T>(g, src, p.N, t, acc);
+    fold_vector<T, COMPAT>(g, src, p.N, t, acc, p.compat, p.r);
     if (g.out_partial) {
       float *o = reinterpret_cast<float *>(g.out) + t;
 #pragma unroll
@@ -295,27 +327,30 @@ __global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams
         st_stream(o + 4 * q, make_int4(__float_as_int(acc[4 * q]), __float_as_int(acc[4 * q + 1]),
                                        __float_as_int(acc[4 * q + 2]), __float_as_int(acc[4 * q + 3])));
     } else {
+      if (post) {
 #pragma unroll
-      for (int e = 0; e < V; ++e) acc[e] = __fmul_rn(acc[e], p.r);   // R5: one rounding
+        for (int e = 0; e < V; ++e) acc[e] = __fmul_rn(acc[e], p.r);   // R5: one rounding
+      }
       st_stream(reinterpret_cast<char *>(g.out) + t * T::kSize, T::narrow(acc));  // R13
     }
   }
   const int64_t tail0 = nvec * V;                                    // ragged tail (< V elements)
   if (gid < g.n - tail0) {
     const int64_t t = tail0 + gid;
-    const float s = fold_scalar<T>(g, src, p.N, t);
+    const float s = fold_scalar<T, COMPAT>(g, src, p.N, t, p.compat, p.r);
     if (g.out_partial) reinterpret_cast<float *>(g.out)[t] = s;
-    else T::store1(g.out, t, __fmul_rn(s, p.r));
+    else T::store1(g.out, t, post ? __fmul_rn(s, p.r) : s);
   }
 }
 
 template <typename T, int MAXSEG, int MAXSRC>
-cudaError_t launch_fold_group(int32_t N, float r, const FoldSegDesc *d, int nseg, cudaStream_t s, int bo,
-                              int to) {
+cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSegDesc *d, int nseg, cudaStream_t s,
+                              int bo, int to) {
   FoldParams<MAXSEG, MAXSRC> p;
   p.nseg = nseg;
   p.N = N;
   p.r = r;
+  p.compat = compat;
   int nsrc = 0;
   std::vector<int64_t> work(nseg);
   for (int i = 0; i < nseg; ++i) {
@@ -343,12 +378,13 @@ cudaError_t launch_fold_group(int32_t N, float r, const FoldSegDesc *d, int nseg
   std::vector<int32_t> block0;
   split_blocks(work, total, &block0, &p.nblocks);
   for (int i = 0; i < nseg; ++i) p.seg[i].block0 = block0[i];
-  return launch(k_fold<T, MAXSEG, MAXSRC>, dim3(p.nblocks), dim3(threads), s, p);
+  if (compat) return launch(k_fold<T, MAXSEG, MAXSRC, true>, dim3(p.nblocks), dim3(threads), s, p);
+  return launch(k_fold<T, MAXSEG, MAXSRC, false>, dim3(p.nblocks), dim3(threads), s, p);
 }
 
 template <typename T>
-cudaError_t launch_fold_t(int32_t N, float r, const FoldSegDesc *segs, int nseg, cudaStream_t s, int bo, int to,
-                          int *launches) {
+cudaError_t launch_fold_t(int32_t N, float r, uint32_t compat, const FoldSegDesc *segs, int nseg, cudaStream_t s,
+                          int bo, int to, int *launches) {
   constexpr int kSmallSeg = 4, kSmallSrc = 64, kBigSeg = 64, kBigSrc = 1024;
   int i = 0;
   while (i < nseg) {
@@ -361,8 +397,8 @@ cudaError_t launch_fold_t(int32_t N, float r, const FoldSegDesc *segs, int nseg,
     }
     if (j == i) return cudaErrorInvalidValue;   // one segment with > 1024 sources (N <= 1024 by contract)
     cudaError_t e = (j - i <= kSmallSeg && nsrc <= kSmallSrc)
-                        ? launch_fold_group<T, kSmallSeg, kSmallSrc>(N, r, segs + i, j - i, s, bo, to)
-                        : launch_fold_group<T, kBigSeg, kBigSrc>(N, r, segs + i, j - i, s, bo, to);
+                        ? launch_fold_group<T, kSmallSeg, kSmallSrc>(N, r, compat, segs + i, j - i, s, bo, to)
+                        : launch_fold_group<T, kBigSeg, kBigSrc>(N, r, compat, segs + i, j - i, s, bo, to);
     if (e != cudaSuccess) return e;
     ++*launches;
     i = j;
@@ -549,8 +585,9 @@ __global__ void __launch_bounds__(256) k_swap(const __grid_constant__ SwapParams
 
 void set_pdl(bool on) { g_pdl = on; }
 
-cudaError_t launch_fold_multi(es_dtype dtype, int32_t N, float r, const FoldSegDesc *segs, int nseg,
+cudaError_t launch_fold_multi(es_dtype dtype, int32_t N, float r, uint32_t compat, const FoldSegDesc *segs, int nseg,
                               cudaStream_t s, int blocks_override, int threads_override, int *launches) {
+  if (dtype != ES_BF16) compat &= ~kBf16Hop;   // bf16 storage rounding only exists for bf16 buckets
   int dummy = 0;
   if (!launches) launches = &dummy;
   std::vector<FoldSegDesc> live;
@@ -559,9 +596,10 @@ cudaError_t launch_fold_multi(es_dtype dtype, int32_t N, float r, const FoldSegD
     if (segs[i].n > 0) live.push_back(segs[i]);
   if (live.empty()) return cudaSuccess;
   if (dtype == ES_BF16)
-    return launch_fold_t<BF16T>(N, r, live.data(), (int)live.size(), s, blocks_override, threads_override,
+    return launch_fold_t<BF16T>(N, r, compat, live.data(), (int)live.size(), s, blocks_override, threads_override,
                                 launches);
-  return launch_fold_t<F32T>(N, r, live.data(), (int)live.size(), s, blocks_override, threads_override, launches);
+  return launch_fold_t<F32T>(N, r, compat, live.data(), (int)live.size(), s, blocks_override, threads_override,
+                             launches);
 }
 
 cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *segs, int nseg, cudaStream_t s,

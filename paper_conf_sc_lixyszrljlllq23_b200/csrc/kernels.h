@@ -36,7 +36,8 @@ struct FoldSegDesc {
 // parameter capacity allows (one for every configuration this build plans
 // for up to 64 segments and 1024 source pointers).  *launches receives the
 // number of kernels enqueued.
-cudaError_t launch_fold_multi(es_dtype dtype, int32_t N, float r, const FoldSegDesc *segs, int nseg,
+// compat: NEXT-3 variant bits (ES_COMPAT_*); 0 = the canonical definition.
+cudaError_t launch_fold_multi(es_dtype dtype, int32_t N, float r, uint32_t compat, const FoldSegDesc *segs, int nseg,
                               cudaStream_t s, int blocks_override, int threads_override, int *launches);
 
 // Stash segments: dst[i] = cast(src[i]) for i < n, all with

@@ -255,6 +255,10 @@ bool validate(const es_config *cfg, std::string *err, bool need_comm) {
       return fail(err, "state_nbytes must be in [1, 2^31]");
   if (cfg->sched != ES_SCHED_AUTO && cfg->sched != ES_SCHED_DIRECT && cfg->sched != ES_SCHED_CHAIN)
     return fail(err, "bad sched");
+  if (cfg->compat & ~(uint32_t)(ES_COMPAT_PREDIV | ES_COMPAT_PREMUL | ES_COMPAT_BF16_HOP))
+    return fail(err, "unknown compat bits");
+  if ((cfg->compat & ES_COMPAT_PREDIV) && (cfg->compat & ES_COMPAT_PREMUL))
+    return fail(err, "compat PREDIV and PREMUL are exclusive");
   if (cfg->G > 1 && need_comm) {
     if (cfg->transport != ES_TRANSPORT_NCCL && cfg->transport != ES_TRANSPORT_LOOPBACK)
       return fail(err, "G > 1 needs transport NCCL or LOOPBACK");
@@ -287,6 +291,7 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
   p->transport = cfg->G > 1 ? cfg->transport : ES_TRANSPORT_NONE;
   p->comm = cfg->G > 1 ? cfg->comm : nullptr;
   p->sched_req = cfg->sched;
+  p->compat = cfg->compat;
 
   p->bp.resize(cfg->n_buckets);
   uint64_t max_stage = 0, max_parts = 0;

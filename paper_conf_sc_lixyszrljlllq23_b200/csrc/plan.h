@@ -53,6 +53,7 @@ struct Plan {
   es_transport transport = ES_TRANSPORT_NONE;
   void *comm = nullptr;
   es_sched sched_req = ES_SCHED_AUTO;
+  uint32_t compat = 0;                  // NEXT-3 variant bits
   std::vector<BucketPlan> bp;
 
   // Workspace layout (byte offsets from the workspace base, 256-aligned).

@@ -22,6 +22,7 @@ ES_KERNEL_STASH, ES_KERNEL_FOLD, ES_KERNEL_SWAP = 0, 1, 2
 ES_OP_FIELDS = 10
 ES_OP_FOLD, ES_OP_SEND, ES_OP_RECV, ES_OP_GROUP_BEGIN, ES_OP_GROUP_END = 1, 2, 3, 4, 5
 ES_BUF_NONE, ES_BUF_SRC, ES_BUF_STAGE, ES_BUF_PART, ES_BUF_OUT = 0, 1, 2, 3, 4
+ES_COMPAT_PREDIV, ES_COMPAT_PREMUL, ES_COMPAT_BF16_HOP = 1, 2, 4
 
 EXPORTED = [
     "es_workspace_bytes", "es_init", "es_destroy", "es_sync", "es_register_state", "es_init_state",
@@ -52,6 +53,7 @@ class es_config(ctypes.Structure):
         ("chunk_align", ctypes.c_uint32),
         ("n_state", ctypes.c_int32), ("state_nbytes", ctypes.POINTER(ctypes.c_uint64)),
         ("transport", ctypes.c_int), ("comm", ctypes.c_void_p), ("sched", ctypes.c_int),
+        ("compat", ctypes.c_uint32),
     ]
 
 
@@ -124,7 +126,7 @@ class Config:
     """Owns an es_config and the host arrays it points to."""
 
     def __init__(self, N, G, rank, est_to_gpu, buckets, chunk_align=16, state_nbytes=(),
-                 transport=ES_TRANSPORT_NONE, comm=None, sched=ES_SCHED_AUTO):
+                 transport=ES_TRANSPORT_NONE, comm=None, sched=ES_SCHED_AUTO, compat=0):
         self.N, self.G, self.rank = int(N), int(G), int(rank)
         self.est_to_gpu = list(int(g) for g in est_to_gpu)
         self.buckets = [(int(n), int(d)) for n, d in buckets]
@@ -133,7 +135,7 @@ class Config:
         self._sn = (ctypes.c_uint64 * max(len(state_nbytes), 1))(*state_nbytes)
         self.state_nbytes = list(state_nbytes)
         self.c = es_config(self.N, self.G, self.rank, self._map, self._bk, len(self.buckets), int(chunk_align),
-                           len(state_nbytes), self._sn, int(transport), comm, int(sched))
+                           len(state_nbytes), self._sn, int(transport), comm, int(sched), int(compat))
 
     def ptr(self):
         return ctypes.byref(self.c)

@@ -58,14 +58,14 @@ def test_chunk_elems_matches_hand_table():
 @pytest.mark.parametrize("bad", [
     dict(N=0), dict(N=1025), dict(G=0), dict(G=5), dict(rank=2), dict(map=[0, 0, 0, 0]),
     dict(map=[0, 1, 2, 0]), dict(buckets=[(1 << 31, es.ES_F32)]), dict(buckets=[(10, 7)]), dict(A=12),
-    dict(sched=9), dict(states=[0]),
+    dict(sched=9), dict(states=[0]), dict(compat=8), dict(compat=3),
 ])
 def test_config_validation(bad):
     N = bad.get("N", 4)
     G = bad.get("G", 2)
     m = bad.get("map", [0, 0, 1, 1][:max(N, 0)] if N == 4 else [0] * max(N, 0))
     cfg = es.Config(N, G, bad.get("rank", 0), m, bad.get("buckets", [(100, es.ES_F32)]), bad.get("A", 16),
-                    bad.get("states", ()), sched=bad.get("sched", 0))
+                    bad.get("states", ()), sched=bad.get("sched", 0), compat=bad.get("compat", 0))
     with pytest.raises(es.EsError) as e:
         es.es_workspace_bytes(cfg)
     assert e.value.status == es.ES_EINVAL

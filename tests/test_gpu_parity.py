@@ -288,3 +288,77 @@ def test_full_size_sampled_parity(name):
         mx = torch.stack([g[b].float().abs() for g in grads]).amax(0)
         assert torch.isfinite(o).all() and bool((o.abs() <= mx * 1.01).all())
     agg.close()
+
+
+# ---- NEXT-3 compatibility variants -------------------------------------------------------------
+
+COMPATS = [es.ES_COMPAT_PREDIV, es.ES_COMPAT_PREMUL, es.ES_COMPAT_BF16_HOP,
+           es.ES_COMPAT_PREDIV | es.ES_COMPAT_BF16_HOP, es.ES_COMPAT_PREMUL | es.ES_COMPAT_BF16_HOP]
+
+
+@pytest.mark.parametrize("compat", COMPATS)
+@pytest.mark.parametrize("N", [3, 12, 16])
+def test_compat_variants_g1(compat, N):
+    from gpu_util import Aggregator, from_dev, to_dev
+    rng = np.random.default_rng(600 + N + compat)
+    Ls, dts = [50003, 17, 4096], ["f32", "bf16", "bf16"]
+    xs = [_gauss(rng, N, L, d, sigma=1.0) for L, d in zip(Ls, dts)]
+    agg = Aggregator(N, 1, 0, [0] * N, list(zip(Ls, dts)), compat=compat)
+    devs = [[to_dev(xs[b][k]) for b in range(3)] for k in range(N)]
+    for k in range(N):
+        agg.stash_many(k, range(3), devs[k], es.ES_STASH_BORROW if k == N - 1 else es.ES_STASH_COPY)
+    outs = [agg.new_out(b) for b in range(3)]
+    agg.allreduce_many(range(3), outs)
+    torch.cuda.synchronize()
+    for b in range(3):
+        assert_bits_equal(from_dev(outs[b]), oracle.reduce_ex(xs[b], dts[b], compat), f"compat={compat} b={b}")
+    agg.close()
+
+
+@pytest.mark.parametrize("sched", [es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN])
+def test_compat_variants_loopback(sched):
+    """Chain partials carry the variant's (bf16-rounded) value between GPUs."""
+    rng = np.random.default_rng(700)
+    for compat in COMPATS:
+        xs = [_gauss(rng, 12, 30001, "bf16", sigma=1.0), _gauss(rng, 12, 999, "f32", sigma=1.0)]
+        want = [oracle.reduce_ex(xs[0], "bf16", compat), oracle.reduce_ex(xs[1], "f32", compat)]
+        from gpu_util import Aggregator, from_dev, to_dev  # noqa: F401
+        res = _loopback_compat(xs, 4, workloads.mapping(12, 4, "random", seed=compat), sched, compat)
+        for g in range(4):
+            for b in range(2):
+                assert_bits_equal(res[g][b], want[b], f"compat={compat} sched={sched} rank={g} b={b}")
+
+
+def _loopback_compat(xs_per_bucket, G, mapping, sched, compat):
+    import threading
+    from gpu_util import Aggregator, code, from_dev, to_dev
+    N = len(xs_per_bucket[0])
+    buckets = [(x[0].size, code(x[0])) for x in xs_per_bucket]
+    world = es.es_loopback_create(G)
+    aggs = [Aggregator(N, G, g, mapping, buckets, transport=es.ES_TRANSPORT_LOOPBACK, comm=world.value,
+                       sched=sched, compat=compat) for g in range(G)]
+    devs = [[to_dev(x) for x in xs] for xs in xs_per_bucket]
+    outs = [[a.new_out(b) for b in range(len(buckets))] for a in aggs]
+    streams = [torch.cuda.Stream() for _ in range(G)]
+    torch.cuda.synchronize()
+    errs = []
+
+    def run(g):
+        try:
+            with torch.cuda.stream(streams[g]):
+                for k in aggs[g].local_ests:
+                    aggs[g].stash_many(k, range(len(buckets)), [devs[b][k] for b in range(len(buckets))])
+                aggs[g].allreduce_many(range(len(buckets)), outs[g])
+        except Exception as e:
+            errs.append(e)
+    ts = [threading.Thread(target=run, args=(g,)) for g in range(G)]
+    [t.start() for t in ts]
+    [t.join(timeout=300) for t in ts]
+    torch.cuda.synchronize()
+    if errs:
+        raise errs[0]
+    res = [[from_dev(o) for o in row] for row in outs]
+    for a in aggs:
+        a.close()
+    es.es_loopback_destroy(world)
+    return res
