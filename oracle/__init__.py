@@ -47,6 +47,12 @@ def lib():
         L.es_oracle_reduce_ex.argtypes = [ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
                                           ctypes.c_uint32, ctypes.POINTER(ctypes.c_void_p), ctypes.c_int64,
                                           ctypes.c_int64, ctypes.c_void_p]
+        L.es_oracle_philox4x32_10.restype = None
+        L.es_oracle_philox4x32_10.argtypes = [ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32),
+                                              ctypes.POINTER(ctypes.c_uint32)]
+        L.es_oracle_dropout.restype = ctypes.c_int
+        L.es_oracle_dropout.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64,
+                                        ctypes.c_int32, ctypes.c_float, ctypes.c_uint64, ctypes.c_uint64]
         L.es_oracle_stash.restype = ctypes.c_int
         L.es_oracle_stash.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p, ctypes.c_int32,
                                       ctypes.c_int64]
@@ -115,6 +121,27 @@ def reduce_ex(xs, dtype, compat, L=None, A=16, first=0):
     if rc != 0:
         raise ValueError("es_oracle_reduce_ex: bad arguments")
     return out
+
+
+def philox4x32_10(ctr, key):
+    c = (ctypes.c_uint32 * 4)(*ctr)
+    k = (ctypes.c_uint32 * 2)(*key)
+    o = (ctypes.c_uint32 * 4)()
+    lib().es_oracle_philox4x32_10(c, k, o)
+    return list(o)
+
+
+def dropout(x, dtype, p, seed, offset):
+    """NEXT-4 per-EST dropout (see es_oracle.c).  Returns (y, mask)."""
+    code = _code(dtype)
+    x = np.ascontiguousarray(x)
+    y = np.empty_like(x)
+    mask = np.empty(x.size, np.uint8)
+    rc = lib().es_oracle_dropout(x.ctypes.data, y.ctypes.data, mask.ctypes.data, x.size, code, float(p),
+                                 int(seed), int(offset))
+    if rc != 0:
+        raise ValueError("es_oracle_dropout: bad arguments")
+    return y, mask
 
 
 def stash(src, src_dtype, dst_dtype):

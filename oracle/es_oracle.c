@@ -194,3 +194,58 @@ int es_oracle_reduce_ex(int32_t N, int64_t L, int32_t A, int32_t dtype, uint32_t
     }
     return 0;
 }
+
+/* ------------------------------------------------------------------ */
+/* NEXT-4: per-EST Philox dropout         */
+/* ------------------------------------------------------------------ */
+
+/* Philox4x32-10 (Salmon et al., SC'11 "Parallel random numbers: as easy as
+ * 1, 2, 3"), written from its published definition: 10 rounds of
+ *   (c0,c1,c2,c3) -> (hi(M1*c2) ^ c1 ^ k0, lo(M1*c2), hi(M0*c0) ^ c3 ^ k1, lo(M0*c0))
+ * with the key bumped by the Weyl constants between rounds. */
+void es_oracle_philox4x32_10(const uint32_t ctr[4], const uint32_t key[2], uint32_t out[4])
+{
+    const uint32_t M0 = 0xD2511F53u, M1 = 0xCD9E8D57u, W0 = 0x9E3779B9u, W1 = 0xBB67AE85u;
+    uint32_t c0 = ctr[0], c1 = ctr[1], c2 = ctr[2], c3 = ctr[3];
+    uint32_t k0 = key[0], k1 = key[1];
+    for (int round = 0; round < 10; ++round) {
+        if (round > 0) { k0 += W0; k1 += W1; }
+        const uint64_t p0 = (uint64_t)M0 * c0;
+        const uint64_t p1 = (uint64_t)M1 * c2;
+        const uint32_t n0 = (uint32_t)(p1 >> 32) ^ c1 ^ k0;
+        const uint32_t n1 = (uint32_t)p1;
+        const uint32_t n2 = (uint32_t)(p0 >> 32) ^ c3 ^ k1;
+        const uint32_t n3 = (uint32_t)p0;
+        c0 = n0; c1 = n1; c2 = n2; c3 = n3;
+    }
+    out[0] = c0; out[1] = c1; out[2] = c2; out[3] = c3;
+}
+
+/*
+ * The dropout an EST's RNG context drives ("the Dropout operator
+ * depends on the random number generator (RNG) states"):
+ *   element i uses Philox4x32-10 with key = (seed lo, seed hi) and counter
+ *   = (i/4 lo, i/4 hi, offset lo, offset hi); word w = out[i % 4];
+ *   u = (w >> 8) * 2^-24;  keep = (u >= p);  scale = fl32(1 / fl32(1 - p));
+ *   y = keep ? round_dtype(fl32(x * scale)) : +0;  mask[i] = keep.
+ * One call consumes one offset unit (the caller advances offset by 1).
+ */
+int es_oracle_dropout(const void *x, void *y, uint8_t *mask, int64_t n, int32_t dtype, float p,
+                      uint64_t seed, uint64_t offset)
+{
+    if (n < 0 || (dtype != ORACLE_F32 && dtype != ORACLE_BF16) || !(p >= 0.0f && p < 1.0f)) return -1;
+    const float scale = 1.0f / (1.0f - p);
+    const uint32_t key[2] = {(uint32_t)seed, (uint32_t)(seed >> 32)};
+    for (int64_t i = 0; i < n; ++i) {
+        const uint64_t q = (uint64_t)i >> 2;
+        const uint32_t ctr[4] = {(uint32_t)q, (uint32_t)(q >> 32), (uint32_t)offset, (uint32_t)(offset >> 32)};
+        uint32_t w[4];
+        es_oracle_philox4x32_10(ctr, key, w);
+        const float u = (float)(w[i & 3] >> 8) * (1.0f / 16777216.0f);
+        const int keep = u >= p;
+        if (mask) mask[i] = (uint8_t)keep;
+        if (keep) store_rounded(y, dtype, i, load_widened(x, dtype, i) * scale);
+        else store_rounded(y, dtype, i, 0.0f);
+    }
+    return 0;
+}

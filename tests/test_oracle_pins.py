@@ -370,3 +370,37 @@ def test_compat_bf16_hop_exact_when_partials_representable():
     assert np.all(oracle.reduce_ex(xs, "bf16", oracle.COMPAT_BF16HOP) == oracle.reduce(xs, "bf16"))
     assert np.all(oracle.reduce_ex(xs, "bf16", oracle.COMPAT_BF16HOP | oracle.COMPAT_PREMUL)
                   == oracle.reduce(xs, "bf16"))                   # N = 8: 1/8 scaling exact too
+
+
+# ---- NEXT-4 per-EST Philox dropout ---------------------------------------------------------------
+
+def test_philox_known_answer_vectors(golden_dir):
+    g = json.load(open(os.path.join(golden_dir, "philox_kat.json")))
+    for c in g["cases"]:
+        out = oracle.philox4x32_10([int(v, 16) for v in c["ctr"]], [int(v, 16) for v in c["key"]])
+        assert out == [int(v, 16) for v in c["out"]]
+
+
+def test_dropout_definition_and_statistics():
+    x = np.linspace(-3, 3, 40001).astype(np.float32)
+    for p in (0.1, 0.5, 0.9):
+        y, m = oracle.dropout(x, "f32", p, seed=123, offset=7)
+        n = x.size
+        keep = m.mean()
+        assert abs(keep - (1 - p)) < 5 * np.sqrt(p * (1 - p) / n)          # binomial 5-sigma
+        scale = np.float32(1) / (np.float32(1) - np.float32(p))
+        assert np.all(_bits(y[m == 1]) == _bits(x[m == 1] * scale))
+        assert np.all(_bits(y[m == 0]) == 0)                              # dropped -> +0
+    # element i's decision depends only on (seed, offset, i): prefixes agree
+    _, m1 = oracle.dropout(x[:1001], "f32", 0.5, 5, 9)
+    _, m2 = oracle.dropout(x, "f32", 0.5, 5, 9)
+    assert np.array_equal(m1, m2[:1001])
+    # word i % 4 of counter i // 4: element 0..3 take the 4 output words of counter (0,0,off lo,off hi)
+    w = oracle.philox4x32_10([0, 0, 9, 0], [5, 0])
+    u = np.array([(v >> 8) / 16777216.0 for v in w], np.float32)
+    assert np.array_equal(m2[:4], (u >= np.float32(0.5)).astype(np.uint8))
+    # a new offset gives a different mask; p = 0 keeps everything
+    _, m3 = oracle.dropout(x, "f32", 0.5, 5, 10)
+    assert not np.array_equal(m2, m3)
+    y0, m0 = oracle.dropout(x, "f32", 0.0, 5, 9)
+    assert m0.all() and np.all(_bits(y0) == _bits(x))
