@@ -266,6 +266,24 @@ es_status es_context_bytes(es_handle h, size_t *bytes);
 es_status es_export_context(es_handle h, int32_t est, void *host_dst, size_t bytes, es_stream stream);
 es_status es_import_context(es_handle h, int32_t est, const void *host_src, size_t bytes, es_stream stream);
 
+/* ---- NEXT-4: a per-EST RNG consumer ---------------------------------------- */
+
+/* Dropout of the running EST (Dropout "depends on the
+ * random number generator (RNG) states"), driven on the device by the
+ * 16-byte Philox record {seed u64, offset u64} registered as context buffer
+ * `state_idx` -- the record es_switch_context swaps -- so the masks an EST
+ * draws are the same whether it runs time-sliced or on a dedicated GPU, and
+ * the call is CUDA-graph capturable.  Element i: Philox4x32-10 with key =
+ * seed, counter = (i/4 lo, i/4 hi, offset lo, offset hi), word i % 4;
+ * u = (w >> 8)*2^-24; kept iff u >= p; y = kept ? round(fl32(x*fl32(1/fl32(1-p)))) : +0.
+ * One call consumes offset += 1 (advanced on the device).  x, y: device,
+ * n elements of dtype, 16-byte aligned; mask: NULL or n bytes (1 = kept).
+ * Calls on one handle must be stream-ordered.  ES_ESTATE if no EST is
+ * running or no state is registered; ES_EINVAL for p outside [0, 1) or a
+ * state_idx that is not a 16-byte buffer. */
+es_status es_dropout(es_handle h, const void *x, void *y, uint8_t *mask, uint64_t n, es_dtype dtype, float p,
+                     int32_t state_idx, es_stream stream);
+
 /* ---- planner introspection (host-only, no CUDA) -------------------------- */
 
 /* R1 chunk size C = A*ceil(ceil(L/N)/A) (A = 0 means 16). */
@@ -305,7 +323,9 @@ es_status es_loopback_destroy(void *world);
 
 /* ---- instrumentation ------------------------------------------------------ */
 
-typedef enum { ES_KERNEL_STASH = 0, ES_KERNEL_FOLD = 1, ES_KERNEL_SWAP = 2, ES_KERNEL_KINDS = 3 } es_kernel_kind;
+typedef enum {
+  ES_KERNEL_STASH = 0, ES_KERNEL_FOLD = 1, ES_KERNEL_SWAP = 2, ES_KERNEL_DROPOUT = 3, ES_KERNEL_KINDS = 4
+} es_kernel_kind;
 
 /* When enabled, every kernel launch of this handle is bracketed by CUDA
  * events on its own stream.  es_profile_query synchronises on those events

@@ -120,6 +120,15 @@ class Aggregator:
         n, d = self.buckets[bucket]
         return torch.empty(n, dtype=TORCH_DTYPES[d], device=self.device)
 
+    # ---- per-EST dropout (NEXT-4) ---------------------------------------------------------
+    def dropout(self, x, p, state_idx=0, with_mask=False, stream=None):
+        """Dropout of the running EST from its device Philox record."""
+        y = torch.empty_like(x)
+        mask = torch.empty(x.numel(), dtype=torch.uint8, device=x.device) if with_mask else None
+        es.es_dropout(self.h, x.data_ptr(), y.data_ptr(), mask.data_ptr() if mask is not None else 0, x.numel(),
+                      DTYPES[x.dtype], p, state_idx, _stream(stream))
+        return (y, mask) if with_mask else y
+
     # ---- zero-copy slots / elastic resume (NEXT-2) ------------------------------------
     def slot(self, est, bucket):
         """Tensor view of local EST `est`'s slot for `bucket` (bind gradients here,

@@ -80,9 +80,9 @@ struct es_ctx {
   std::vector<Rec> recs;
   std::vector<cudaEvent_t> pool;
   std::vector<cudaEvent_t> graph_events;
-  uint64_t launches[ES_KERNEL_KINDS] = {0, 0, 0};
-  uint64_t bytes[ES_KERNEL_KINDS] = {0, 0, 0};
-  double ms[ES_KERNEL_KINDS] = {0, 0, 0};
+  uint64_t launches[ES_KERNEL_KINDS] = {};
+  uint64_t bytes[ES_KERNEL_KINDS] = {};
+  double ms[ES_KERNEL_KINDS] = {};
   int blocks_ov = 0, threads_ov = 0;
 
   ~es_ctx() {
@@ -231,6 +231,7 @@ es_status es_init(const es_config *cfg, void *workspace, size_t workspace_bytes,
     if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
       return set_err(ES_ECUDA, "cudaEventCreate failed");
   for (uint64_t n : h->plan.state_nbytes) h->max_state = std::max<uint64_t>(h->max_state, n);
+  if (cudaMemset(h->ws + h->plan.scratch_off, 0, 256) != cudaSuccess) return set_err(ES_ECUDA, "cudaMemset failed");
   if (h->plan.G > 1) {
     es::Transport *t = h->plan.transport == ES_TRANSPORT_NCCL
                            ? es::make_nccl_transport(h->plan.comm, h->plan.G, h->plan.rank, &err)
@@ -796,6 +797,32 @@ es_status es_import_context(es_handle h, int32_t est, const void *host_src, size
   // host_src may be released by the caller on return
   if (cudaStreamSynchronize(cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaStreamSynchronize failed");
   return ES_OK;
+}
+
+// ---- NEXT-4: per-EST dropout ---------------------------------------------------
+
+es_status es_dropout(es_handle h, const void *x, void *y, uint8_t *mask, uint64_t n, es_dtype dtype, float p,
+                     int32_t state_idx, es_stream stream) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  const es::Plan &pl = h->plan;
+  if (dtype != ES_F32 && dtype != ES_BF16) return set_err(ES_EINVAL, "bad dtype");
+  if (!(p >= 0.0f && p < 1.0f)) return set_err(ES_EINVAL, "p must be in [0, 1)");
+  if (n >= (1ull << 40)) return set_err(ES_EINVAL, "n too large");
+  if (n > 0 && (!x || !y)) return set_err(ES_EINVAL, "x / y are NULL");
+  if (state_idx < 0 || state_idx >= (int32_t)pl.state_nbytes.size() || pl.state_nbytes[state_idx] != 16)
+    return set_err(ES_EINVAL, "state_idx must name a registered 16-byte Philox record");
+  if (!h->state_registered) return set_err(ES_ESTATE, "es_register_state has not been called");
+  if (h->cur_local < 0) return set_err(ES_ESTATE, "no EST is running (call es_switch_context first)");
+  cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
+  const float scale = 1.0f / (1.0f - p);
+  const uint64_t nbytes = n * (2 * (uint64_t)es::dtype_size(dtype) + (mask ? 1 : 0));
+  return h->timed(ES_KERNEL_DROPOUT, nbytes, cs, [&](int *nl) {
+    *nl = 1;
+    return es::launch_dropout(dtype, x, y, mask, (int64_t)n, p, scale,
+                              reinterpret_cast<uint64_t *>(h->live_ptr[state_idx]),
+                              reinterpret_cast<unsigned int *>(h->ws + pl.scratch_off), cs);
+  });
 }
 
 // ---- instrumentation ---------------------------------------------------------

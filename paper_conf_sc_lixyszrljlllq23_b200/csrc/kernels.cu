@@ -581,6 +581,69 @@ __global__ void __launch_bounds__(256) k_swap(const __grid_constant__ SwapParams
   swap_entry(p.tab, (int)blockIdx.y, (int)blockIdx.x, (int)gridDim.x, p.cur, p.next);
 }
 
+// ---- k_dropout (NEXT-4) ------------------------------------------------------
+// Philox4x32-10 (Salmon et al., SC'11) -- element i: key = seed, counter =
+// (i/4, offset); word i % 4; u = (w >> 8) * 2^-24; keep = u >= p.
+
+__device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint2 k) {
+  const uint32_t M0 = 0xD2511F53u, M1 = 0xCD9E8D57u, W0 = 0x9E3779B9u, W1 = 0xBB67AE85u;
+#pragma unroll
+  for (int r = 0; r < 10; ++r) {
+    if (r > 0) {
+      k.x += W0;
+      k.y += W1;
+    }
+    const uint32_t hi0 = __umulhi(M0, c.x), lo0 = M0 * c.x;
+    const uint32_t hi1 = __umulhi(M1, c.z), lo1 = M1 * c.z;
+    c = make_uint4(hi1 ^ c.y ^ k.x, lo1, hi0 ^ c.w ^ k.y, lo0);
+  }
+  return c;
+}
+
+struct DropoutParams {
+  const void *x;
+  void *y;
+  uint8_t *mask;
+  int64_t n;
+  float p, scale;
+  uint64_t *record;
+  unsigned int *counter;
+};
+
+template <typename T>
+__global__ void __launch_bounds__(256) k_dropout(const __grid_constant__ DropoutParams p) {
+  pdl_enter();
+  const uint64_t seed = p.record[0], offset = p.record[1];
+  const uint2 key = make_uint2((uint32_t)seed, (uint32_t)(seed >> 32));
+  const int64_t nq = (p.n + 3) / 4;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < nq; q += stride) {
+    const uint4 w = philox4x32_10(
+        make_uint4((uint32_t)q, (uint32_t)((uint64_t)q >> 32), (uint32_t)offset, (uint32_t)(offset >> 32)), key);
+    const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const int64_t i = q * 4 + e;
+      if (i < p.n) {
+        const float u = __uint2float_rn(ws[e] >> 8) * (1.0f / 16777216.0f);   // exact: 24-bit integer
+        const bool keep = u >= p.p;
+        T::store1(p.y, i, keep ? __fmul_rn(T::load1(p.x, i), p.scale) : 0.0f);
+        if (p.mask) p.mask[i] = keep ? 1 : 0;
+      }
+    }
+  }
+  // Advance the EST's Philox offset once every block has read it.
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(p.counter, 1u) == gridDim.x - 1) {
+      p.record[1] = offset + 1;
+      *p.counter = 0;
+      __threadfence();
+    }
+  }
+}
+
 }  // namespace
 
 void set_pdl(bool on) { g_pdl = on; }
@@ -623,6 +686,15 @@ cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *s
   if (sdt == ES_F32 && ddt == ES_BF16)
     return launch_stash_t<F32T, BF16T, 4>(live.data(), n, s, bo, to, launches, swap);
   return launch_stash_t<BF16T, F32T, 4>(live.data(), n, s, bo, to, launches, swap);
+}
+
+cudaError_t launch_dropout(es_dtype dtype, const void *x, void *y, uint8_t *mask, int64_t n, float p, float scale,
+                           uint64_t *record, unsigned int *counter, cudaStream_t s) {
+  DropoutParams d{x, y, mask, n, p, scale, record, counter};
+  const int64_t nq = std::max<int64_t>((n + 3) / 4, 1);
+  const int blocks = (int)std::min<int64_t>((nq + 255) / 256, (int64_t)kSMs * 16);
+  if (dtype == ES_BF16) return launch(k_dropout<BF16T>, dim3(blocks), dim3(256), s, d);
+  return launch(k_dropout<F32T>, dim3(blocks), dim3(256), s, d);
 }
 
 cudaError_t launch_swap(const SwapEntry *table_dev, int32_t n, uint64_t max_nbytes, int32_t cur, int32_t next,

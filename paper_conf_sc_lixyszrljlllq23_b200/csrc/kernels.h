@@ -75,6 +75,14 @@ cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *s
 cudaError_t launch_swap(const SwapEntry *table_dev, int32_t n, uint64_t max_nbytes, int32_t cur, int32_t next,
                         cudaStream_t s);
 
+// NEXT-4 per-EST dropout: y = dropout(x, p)
+// driven by the Philox record {seed u64, offset u64} at `record` (the live
+// context buffer of the running EST); the kernel advances record.offset by
+// one when the whole grid has read it (`counter`: a zeroed u32 in the
+// workspace).  x / y 16-byte aligned; mask (nullable) gets 1 = kept.
+cudaError_t launch_dropout(es_dtype dtype, const void *x, void *y, uint8_t *mask, int64_t n, float p, float scale,
+                           uint64_t *record, unsigned int *counter, cudaStream_t s);
+
 // Programmatic dependent launch (on by default; ES_NO_PDL=1 disables).
 void set_pdl(bool on);
 

@@ -341,6 +341,8 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
   total += p->state_block * p->local_ests.size();
   p->table_off = total;
   total += align256(p->state_nbytes.size() * 32);
+  p->scratch_off = total;
+  total += 256;
   p->stage_off = total;
   total += max_stage;
   p->parts_off = total;

@@ -64,6 +64,7 @@ struct Plan {
   uint64_t state_block = 0;
   uint64_t state_area_off = 0;          // n_local state blocks
   uint64_t table_off = 0;               // swap table (n_state entries)
+  uint64_t scratch_off = 0;             // 256 B of zeroed scratch (dropout grid counter)
   uint64_t stage_off = 0;               // exchange staging (max over buckets)
   uint64_t parts_off = 0;               // chain partials (max over buckets)
   uint64_t total = 0;

@@ -18,7 +18,7 @@ ES_F32, ES_BF16 = 0, 1
 ES_STASH_COPY, ES_STASH_BORROW, ES_STASH_INPLACE = 0, 1, 2
 ES_SCHED_AUTO, ES_SCHED_DIRECT, ES_SCHED_CHAIN = 0, 1, 2
 ES_TRANSPORT_NONE, ES_TRANSPORT_NCCL, ES_TRANSPORT_LOOPBACK = 0, 1, 2
-ES_KERNEL_STASH, ES_KERNEL_FOLD, ES_KERNEL_SWAP = 0, 1, 2
+ES_KERNEL_STASH, ES_KERNEL_FOLD, ES_KERNEL_SWAP, ES_KERNEL_DROPOUT = 0, 1, 2, 3
 ES_OP_FIELDS = 10
 ES_OP_FOLD, ES_OP_SEND, ES_OP_RECV, ES_OP_GROUP_BEGIN, ES_OP_GROUP_END = 1, 2, 3, 4, 5
 ES_BUF_NONE, ES_BUF_SRC, ES_BUF_STAGE, ES_BUF_PART, ES_BUF_OUT = 0, 1, 2, 3, 4
@@ -28,7 +28,7 @@ EXPORTED = [
     "es_workspace_bytes", "es_init", "es_destroy", "es_sync", "es_register_state", "es_init_state",
     "es_read_state", "es_switch_context", "es_stash_grad", "es_stash_grads", "es_stash_and_switch", "es_allreduce",
     "es_allreduce_many", "es_chunk_elems", "es_slot_ptr", "es_context_bytes", "es_export_context",
-    "es_import_context",
+    "es_import_context", "es_dropout",
     "es_plan_ops", "es_loopback_create", "es_loopback_destroy", "es_profile_enable",
     "es_profile_reset", "es_profile_query", "es_set_launch_override", "es_status_string",
     "es_last_error", "es_abi_version",
@@ -94,6 +94,7 @@ def lib():
                                      ctypes.POINTER(ctypes.c_int), ctypes.c_int, i32, P]),
         "es_chunk_elems": (u64, [u64, i32, u32]),
         "es_slot_ptr": (st, [P, i32, i32, ctypes.POINTER(P)]),
+        "es_dropout": (st, [P, P, P, P, u64, ctypes.c_int, ctypes.c_float, i32, P]),
         "es_context_bytes": (st, [P, ctypes.POINTER(sz)]),
         "es_export_context": (st, [P, i32, P, sz, P]),
         "es_import_context": (st, [P, i32, P, sz, P]),
@@ -238,6 +239,11 @@ def es_export_context(h, est, stream):
 def es_import_context(h, est, blob, stream):
     buf = ctypes.create_string_buffer(bytes(blob), len(blob))
     _check(lib().es_import_context(h, est, buf, len(blob), ctypes.c_void_p(stream)), "es_import_context")
+
+
+def es_dropout(h, x_ptr, y_ptr, mask_ptr, n, dtype, p, state_idx, stream):
+    _check(lib().es_dropout(h, ctypes.c_void_p(x_ptr), ctypes.c_void_p(y_ptr), ctypes.c_void_p(mask_ptr), n, dtype,
+                            float(p), state_idx, ctypes.c_void_p(stream)), "es_dropout")
 
 
 def es_chunk_elems(L, N, A=16):

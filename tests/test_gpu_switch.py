@@ -351,3 +351,90 @@ def test_elastic_resume_mid_step_fig9():
     for a in aggs2:
         a.close()
     es.es_loopback_destroy(w2)
+
+
+# ---- NEXT-4: per-EST device Philox dropout --------------------------------------------------
+
+def _philox_state(seed, offset=0):
+    return int(seed).to_bytes(8, "little") + int(offset).to_bytes(8, "little")
+
+
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+def test_dropout_matches_oracle(dtype):
+    import oracle
+    from gpu_util import assert_bits_equal, from_dev, to_dev
+    agg = Aggregator(1, 1, 0, [0], [(64, "f32")], state_nbytes=[16])
+    live = [torch.zeros(16, dtype=torch.uint8, device="cuda")]
+    agg.register_state(live)
+    seed, off = 0x1234_5678_9ABC_DEF0, 41
+    agg.init_state(0, 0, _philox_state(seed, off))
+    agg.switch(0)
+    rng = np.random.default_rng(7)
+    for n, p in [(1, 0.5), (5, 0.1), (4099, 0.5), (100003, 0.9), (65536, 0.0)]:
+        x32 = rng.standard_normal(n).astype(np.float32)
+        x = x32 if dtype == "f32" else oracle.f32_to_bf16_bits(x32)
+        y, m = agg.dropout(to_dev(x), p, with_mask=True)
+        torch.cuda.synchronize()
+        wy, wm = oracle.dropout(x, dtype, p, seed, off)
+        assert np.array_equal(m.cpu().numpy(), wm), (n, p)
+        assert_bits_equal(from_dev(y), wy, f"n={n} p={p}")
+        off += 1                                                  # one offset unit per call
+        assert live[0].cpu().numpy().tobytes() == _philox_state(seed, off)
+    agg.close()
+
+
+def _dedicated_masks(seeds, steps, calls, n, p):
+    out = {}
+    for k, seed in enumerate(seeds):
+        a = Aggregator(1, 1, 0, [0], [(64, "f32")], state_nbytes=[16])
+        live = [torch.zeros(16, dtype=torch.uint8, device="cuda")]
+        a.register_state(live)
+        a.init_state(0, 0, _philox_state(seed))
+        a.switch(0)
+        x = torch.ones(n, device="cuda")
+        out[k] = [[a.dropout(x, p, with_mask=True)[1].clone() for _ in range(calls)] for _ in range(steps)]
+        torch.cuda.synchronize()
+        a.close()
+    return out
+
+
+def test_dropout_time_sliced_equals_dedicated_and_graph_safe():
+    """An EST's masks do not depend on how ESTs share a GPU -- eager and inside
+    a CUDA graph (where a host-side generator mirror could not follow)."""
+    N, steps, calls, n, p = 4, 3, 2, 20000, 0.3
+    seeds = [1000 + 7 * k for k in range(N)]
+    want = _dedicated_masks(seeds, steps, calls, n, p)
+    for use_graph in (False, True):
+        agg = Aggregator(N, 1, 0, [0] * N, [(64, "f32")], state_nbytes=[16])
+        live = [torch.zeros(16, dtype=torch.uint8, device="cuda")]
+        agg.register_state(live)
+        for k in range(N):
+            agg.init_state(k, 0, _philox_state(seeds[k]))
+        x = torch.ones(n, device="cuda")
+        masks = [[torch.empty(n, dtype=torch.uint8, device="cuda") for _ in range(calls)] for _ in range(N)]
+
+        def one_step():
+            for k in range(N):
+                agg.switch(k)
+                for c in range(calls):
+                    es.es_dropout(agg.h, x.data_ptr(), ybuf.data_ptr(),
+                                  masks[k][c].data_ptr(), n, es.ES_F32, p, 0, torch.cuda.current_stream().cuda_stream)
+        ybuf = torch.empty_like(x)
+        if use_graph:
+            s = torch.cuda.Stream()
+            g = torch.cuda.CUDAGraph()
+            agg.switch(N - 1)                      # the step starts with EST N-1 live, as after a step
+            torch.cuda.synchronize()
+            # capture consumes nothing: records only advance when the graph runs
+            with torch.cuda.graph(g, stream=s):
+                one_step()
+        for st in range(steps):
+            if use_graph:
+                g.replay()
+            else:
+                one_step()
+            torch.cuda.synchronize()
+            for k in range(N):
+                for c in range(calls):
+                    assert torch.equal(masks[k][c], want[k][st][c]), (use_graph, st, k, c)
+        agg.close()
