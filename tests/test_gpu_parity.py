@@ -256,38 +256,124 @@ def test_loopback_multi_step_reuse(sched, batched):
 
 # ---- full size, in the bench launch configuration: sampled windows -----------------------------
 
-@pytest.mark.parametrize("name", ["tiny", "resnet50"])
+def _bench_step(agg, local, grads, outs):
+    """Exactly bench.py's step: switch-in, fused stash+switch per EST, the last
+    local EST borrowed, one batched allreduce."""
+    B = len(outs)
+    agg.switch(local[0])
+    for i, k in enumerate(local):
+        if i == len(local) - 1:
+            agg.stash_many(k, range(B), grads[k], es.ES_STASH_BORROW)
+        else:
+            agg.stash_and_switch(k, range(B), grads[k], local[i + 1], es.ES_STASH_COPY)
+    agg.allreduce_many(range(B), outs)
+
+
+def _check_sampled(name, outs, fetch, buckets, N, seed=0):
+    from gpu_util import from_dev
+    rng = np.random.default_rng(seed)
+    for b, (L, d) in enumerate(buckets):
+        C = oracle.chunk_elems(L, N)
+        starts = [0, max(0, L - 4099), max(0, C - 2000), max(0, (N - 1) * C - 7)] + \
+            list(rng.integers(0, max(1, L - 4099), 3))
+        for s in starts:
+            s = int(min(s, L - 1))
+            n = min(4099, L - s)
+            want = oracle.reduce([fetch(k, b, s, n) for k in range(N)], d, L=L, first=s)
+            assert_bits_equal(from_dev(outs[b][s:s + n]), want, f"{name} b={b} s={s}")
+
+
+@pytest.mark.parametrize("name", ["tiny", "resnet50", "vgg19", "bert_base", "swin_b"])
 def test_full_size_sampled_parity(name):
+    """BASELINE.json's full sizes at G=1, in bench.py's launch configuration
+    (CUDA graph of the fused step, replayed), checked on sampled windows that
+    include chunk boundaries and the ragged end, plus a property at any size."""
     cfg = workloads.config(name)
     N = cfg["N"]
     from gpu_util import Aggregator, from_dev
     buckets = cfg["buckets"]
-    agg = Aggregator(N, 1, 0, [0] * N, buckets)
-    grads = [[workloads.est_bucket(name, k, b, device="cuda") for b in range(len(buckets))] for k in range(N)]
-    outs = [agg.new_out(b) for b in range(len(buckets))]
+    agg = Aggregator(N, 1, 0, [0] * N, buckets, state_nbytes=workloads.state_nbytes())
+    live = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in workloads.state_nbytes()]
+    agg.register_state(live)
     for k in range(N):
-        for b in range(len(buckets)):
-            agg.stash(k, b, grads[k][b], es.ES_STASH_BORROW if k == N - 1 else es.ES_STASH_COPY)
-    for b in range(len(buckets)):
-        agg.allreduce(b, outs[b])
+        for i, blob in enumerate(workloads.est_state(name, k)):
+            agg.init_state(k, i, blob)
+    grads = {k: [workloads.est_bucket(name, k, b, device="cuda") for b in range(len(buckets))] for k in range(N)}
+    outs = [agg.new_out(b) for b in range(len(buckets))]
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        _bench_step(agg, list(range(N)), grads, outs)        # eager warm-up
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        _bench_step(agg, list(range(N)), grads, outs)
+    for o in outs:
+        o.zero_()
+    for _ in range(2):
+        g.replay()
     torch.cuda.synchronize()
     agg.sync()
-    rng = np.random.default_rng(0)
-    for b, (L, d) in enumerate(buckets):
-        C = oracle.chunk_elems(L, N)
-        starts = [0, max(0, L - 4099), max(0, C - 2000)] + list(rng.integers(0, max(1, L - 4099), 3))
-        for s in starts:
-            s = int(s)
-            n = min(4099, L - s)
-            win = [from_dev(grads[k][b][s:s + n]) for k in range(N)]
-            want = oracle.reduce(win, d, L=L, first=s)
-            assert_bits_equal(from_dev(outs[b][s:s + n]), want, f"{name} b={b} s={s}")
-    # property at any size: every element finite and |out| <= max_k |x_k| (up to rounding)
-    for b in range(len(buckets)):
+    _check_sampled(name, outs, lambda k, b, st, n: from_dev(grads[k][b][st:st + n]), buckets, N)
+    for b in range(len(buckets)):         # property at any size: finite, |out| <= max_k |x_k| (+ rounding)
         o = outs[b].float()
-        mx = torch.stack([g[b].float().abs() for g in grads]).amax(0)
+        mx = grads[0][b].float().abs()
+        for k in range(1, N):
+            mx = torch.maximum(mx, grads[k][b].float().abs())
         assert torch.isfinite(o).all() and bool((o.abs() <= mx * 1.01).all())
     agg.close()
+
+
+@pytest.mark.parametrize("name,G,kind", [("resnet50", 8, "contiguous"), ("resnet50", 2, "contiguous"),
+                                         ("bert_base", 8, "contiguous"), ("bert_base", 8, "round_robin"),
+                                         ("vgg19", 4, "contiguous")])
+def test_full_size_multi_rank_loopback(name, G, kind):
+    """The configs' G > 1 shapes at full size over the loopback transport
+    (all G ranks on this GPU): every rank holds the oracle's bits."""
+    import threading
+    cfg = workloads.config(name)
+    N = cfg["N"]
+    from gpu_util import Aggregator, from_dev
+    buckets = cfg["buckets"]
+    m = workloads.mapping(N, G, kind)
+    world = es.es_loopback_create(G)
+    aggs = [Aggregator(N, G, r, m, buckets, state_nbytes=workloads.state_nbytes(),
+                       transport=es.ES_TRANSPORT_LOOPBACK, comm=world.value) for r in range(G)]
+    lives = []
+    for r, a in enumerate(aggs):
+        live = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in workloads.state_nbytes()]
+        a.register_state(live)
+        lives.append(live)
+        for k in a.local_ests:
+            for i, blob in enumerate(workloads.est_state(name, k)):
+                a.init_state(k, i, blob)
+    grads = {k: [workloads.est_bucket(name, k, b, device="cuda") for b in range(len(buckets))] for k in range(N)}
+    outs = [[a.new_out(b) for b in range(len(buckets))] for a in aggs]
+    streams = [torch.cuda.Stream() for _ in range(G)]
+    torch.cuda.synchronize()
+    errs = []
+
+    def run(r):
+        try:
+            with torch.cuda.stream(streams[r]):
+                _bench_step(aggs[r], aggs[r].local_ests, grads, outs[r])
+        except Exception as e:
+            errs.append(e)
+    ts = [threading.Thread(target=run, args=(r,)) for r in range(G)]
+    [t.start() for t in ts]
+    [t.join(timeout=600) for t in ts]
+    torch.cuda.synchronize()
+    if errs:
+        raise errs[0]
+    fetch = lambda k, b, st, n: from_dev(grads[k][b][st:st + n])  # noqa: E731
+    for r in (0, G - 1):
+        _check_sampled(f"{name} G={G} {kind} rank {r}", outs[r], fetch, buckets, N, seed=r)
+    for r in range(1, G):                 # every rank holds the same bits
+        for b in range(len(buckets)):
+            iv = torch.int16 if outs[r][b].dtype == torch.bfloat16 else torch.int32
+            assert torch.equal(outs[r][b].view(iv), outs[0][b].view(iv)), (r, b)
+    for a in aggs:
+        a.close()
+    es.es_loopback_destroy(world)
 
 
 # ---- NEXT-3 compatibility variants -------------------------------------------------------------
