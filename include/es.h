@@ -88,10 +88,18 @@ typedef enum { ES_STASH_COPY = 0, ES_STASH_BORROW = 1, ES_STASH_INPLACE = 2 } es
  *           EST c scales, rounds and owns chunk c; then all-gather.
  *   AUTO:   per bucket, the one with fewer max-per-GPU received bytes
  *           (ties -> DIRECT).  The choice is identical on every rank. */
-typedef enum { ES_SCHED_AUTO = 0, ES_SCHED_DIRECT = 1, ES_SCHED_CHAIN = 2 } es_sched;
+/*   PEER:   no transport library: rank g's fold kernel pulls the remote
+ *           ESTs' contributions for its shard straight out of the peers'
+ *           slots over NVLink (CUDA IPC-mapped workspaces, es_peer_*), writes
+ *           its shard result into its own workspace, and a gather kernel pulls
+ *           every other shard from its owner; device-side barriers (flags in
+ *           peer memory) order the phases.  No staging copy, no NCCL protocol.
+ *           Opt-in (never chosen by AUTO); BORROWed buckets are made
+ *           peer-visible by copying the parts peers read into the slot. */
+typedef enum { ES_SCHED_AUTO = 0, ES_SCHED_DIRECT = 1, ES_SCHED_CHAIN = 2, ES_SCHED_PEER = 3 } es_sched;
 
 /* How ranks exchange bytes when G > 1.
- *   NONE:     G == 1 only.
+ *   NONE:     G == 1, or G > 1 with sched PEER (no transport library needed).
  *   NCCL:     `comm` is a borrowed ncclComm_t over exactly the G ranks
  *             (e.g. torch ProcessGroupNCCL._comm_ptr()).  Only point-to-point
  *             ncclSend/ncclRecv inside ncclGroupStart/End are used -- never an
@@ -239,6 +247,22 @@ es_status es_allreduce(es_handle h, int32_t bucket, void *out, es_stream stream)
  * checked for every entry before anything is enqueued. */
 es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void *const *outs, es_stream stream);
 
+/* ---- peer memory (ES_SCHED_PEER) -------------------------------------------- */
+
+/* Opaque per-rank descriptor of this handle's workspace for peers: a CUDA
+ * IPC handle of the workspace's allocation plus offset, process id and raw
+ * address.  The caller all-gathers the G blobs with any collective it has
+ * (e.g. torch.distributed.all_gather_object) and passes them, in rank order,
+ * to es_peer_open, which maps every peer's workspace (cudaIpcOpenMemHandle
+ * with lazy peer access; the raw address when the peer lives in the same
+ * process, as with the loopback transport).  Required before the first
+ * es_allreduce of a handle whose schedule is PEER; ES_EUNSUPPORTED if the
+ * workspace cannot be IPC-exported (e.g. a VMM / expandable-segments
+ * allocation). */
+#define ES_PEER_BLOB_BYTES 128
+es_status es_peer_blob(es_handle h, void *blob, size_t bytes);
+es_status es_peer_open(es_handle h, const void *blobs, size_t bytes);
+
 /* ---- zero-copy slots and elastic resume -------------- */
 
 /* Device pointer of local EST `est`'s slot for `bucket` (bucket dtype,
@@ -303,14 +327,17 @@ enum {
   ES_OP_SEND = 2,        /* [1]=lo [2]=hi [3]=peer [4]=buf_kind [5]=buf_id                      */
   ES_OP_RECV = 3,        /* same fields as SEND                                                 */
   ES_OP_GROUP_BEGIN = 4,
-  ES_OP_GROUP_END = 5
+  ES_OP_GROUP_END = 5,
+  ES_OP_BARRIER = 6,     /* PEER: all G ranks reach this point (device flags)                  */
+  ES_OP_GATHER = 7       /* PEER: [1]=lo [2]=hi [3]=owner: out[lo,hi) <- owner's ES_BUF_RESULT  */
 };
 enum {
   ES_BUF_NONE = 0,
   ES_BUF_SRC = 1,        /* local EST buf_id's contribution (slot or borrowed), bucket dtype   */
   ES_BUF_STAGE = 2,      /* staging for remote EST buf_id's contribution, bucket dtype         */
   ES_BUF_PART = 3,       /* fp32 partial buffer buf_id                                         */
-  ES_BUF_OUT = 4         /* the caller's output, bucket dtype                                  */
+  ES_BUF_OUT = 4,        /* the caller's output, bucket dtype                                  */
+  ES_BUF_RESULT = 5      /* PEER: this rank's shard result area in its workspace, bucket dtype */
 };
 /* All [lo, hi) ranges are in bucket element coordinates. */
 es_status es_plan_ops(const es_config *cfg, int32_t bucket, int64_t *ops, size_t cap_ops,
@@ -324,7 +351,8 @@ es_status es_loopback_destroy(void *world);
 /* ---- instrumentation ------------------------------------------------------ */
 
 typedef enum {
-  ES_KERNEL_STASH = 0, ES_KERNEL_FOLD = 1, ES_KERNEL_SWAP = 2, ES_KERNEL_DROPOUT = 3, ES_KERNEL_KINDS = 4
+  ES_KERNEL_STASH = 0, ES_KERNEL_FOLD = 1, ES_KERNEL_SWAP = 2, ES_KERNEL_DROPOUT = 3, ES_KERNEL_GATHER = 4,
+  ES_KERNEL_BARRIER = 5, ES_KERNEL_KINDS = 6
 } es_kernel_kind;
 
 /* When enabled, every kernel launch of this handle is bracketed by CUDA

@@ -120,6 +120,21 @@ class Aggregator:
         n, d = self.buckets[bucket]
         return torch.empty(n, dtype=TORCH_DTYPES[d], device=self.device)
 
+    # ---- peer memory (ES_SCHED_PEER) ----------------------------------------------------
+    def peer_blob(self):
+        return es.es_peer_blob(self.h)
+
+    def peer_open(self, blobs):
+        """blobs: every rank's peer_blob(), in rank order."""
+        es.es_peer_open(self.h, list(blobs))
+
+    def peer_connect(self, group=None):
+        """All-gather the peer blobs over torch.distributed and map the peers."""
+        import torch.distributed as dist
+        blobs = [None] * self.G
+        dist.all_gather_object(blobs, self.peer_blob(), group=group)
+        self.peer_open(blobs)
+
     # ---- per-EST dropout (NEXT-4) ---------------------------------------------------------
     def dropout(self, x, p, state_idx=0, with_mask=False, stream=None):
         """Dropout of the running EST from its device Philox record."""

@@ -4,6 +4,8 @@
 // groups (transport_*.cpp) on the caller's stream.
 #include <cuda_runtime.h>
 
+#include <unistd.h>
+
 #include <algorithm>
 #include <cstring>
 #include <memory>
@@ -70,6 +72,12 @@ struct es_ctx {
   es_status sticky = ES_OK;
   std::string sticky_msg;
 
+  // ES_SCHED_PEER
+  std::vector<unsigned char *> peer_ws;   // [G] workspace base of every rank, mapped here
+  std::vector<void *> ipc_mapped;         // cudaIpcOpenMemHandle results to close
+  bool peer_open = false;
+  uint64_t barrier_epoch = 0;
+
   // instrumentation
   bool prof = false;
   struct Rec {
@@ -91,6 +99,7 @@ struct es_ctx {
     for (auto &r : recs) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
     for (auto e : pool) cudaEventDestroy(e);
     for (auto e : graph_events) cudaEventDestroy(e);
+    for (void *p : ipc_mapped) cudaIpcCloseMemHandle(p);
   }
   cudaEvent_t ev() {
     if (!pool.empty()) {
@@ -232,7 +241,9 @@ es_status es_init(const es_config *cfg, void *workspace, size_t workspace_bytes,
       return set_err(ES_ECUDA, "cudaEventCreate failed");
   for (uint64_t n : h->plan.state_nbytes) h->max_state = std::max<uint64_t>(h->max_state, n);
   if (cudaMemset(h->ws + h->plan.scratch_off, 0, 256) != cudaSuccess) return set_err(ES_ECUDA, "cudaMemset failed");
-  if (h->plan.G > 1) {
+  if (h->plan.peer && cudaMemset(h->ws + h->plan.flags_off, 0, 64 * 8) != cudaSuccess)
+    return set_err(ES_ECUDA, "cudaMemset of the peer flags failed");
+  if (h->plan.G > 1 && h->plan.transport != ES_TRANSPORT_NONE) {
     es::Transport *t = h->plan.transport == ES_TRANSPORT_NCCL
                            ? es::make_nccl_transport(h->plan.comm, h->plan.G, h->plan.rank, &err)
                            : es::make_loopback_transport(h->plan.comm, h->plan.G, h->plan.rank, &err);
@@ -467,6 +478,127 @@ es_status es_stash_grad(es_handle h, int32_t est, int32_t bucket, const void *gr
 
 // ---- aggregation --------------------------------------------------------------------
 
+namespace {
+es_status finish_allreduce(es_handle h, int32_t n, const int32_t *buckets, cudaStream_t cs, unsigned long long cap);
+
+es_status peer_barrier(es_handle h, cudaStream_t cs) {
+  const es::Plan &p = h->plan;
+  std::vector<uint64_t *> pf(p.G);
+  for (int32_t g = 0; g < p.G; ++g) pf[g] = reinterpret_cast<uint64_t *>(h->peer_ws[g] + p.flags_off);
+  const uint64_t epoch = ++h->barrier_epoch;
+  return h->timed(ES_KERNEL_BARRIER, 0, cs, [&](int *nl) {
+    *nl = 1;
+    return es::launch_peer_barrier(pf.data(), reinterpret_cast<uint64_t *>(h->ws + p.flags_off), p.G, p.rank, epoch,
+                                   cs);
+  });
+}
+
+// ES_SCHED_PEER, phase-merged over the batch: [peer-visible copies of
+// borrowed buckets] -> barrier -> one fold launch (own shards, remote
+// contributions read from the owners' slots over NVLink) -> barrier -> one
+// gather launch per dtype (every shard from its owner's RESULT area).
+es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *const *outs, cudaStream_t cs, float r) {
+  const es::Plan &p = h->plan;
+  if (!h->peer_open) return set_err(ES_ESTATE, "ES_SCHED_PEER needs es_peer_open before es_allreduce");
+  es_status s;
+  const int32_t g = p.rank;
+  auto slot_of = [&](int32_t rank, int32_t e, int32_t b) {
+    return h->peer_ws[rank] + p.grad_off + (uint64_t)p.owner_index[e] * p.slot_block + p.slot_off[b];
+  };
+  // 1. borrowed contributions: peers read the ranges outside our shard from the slot
+  for (int dd = 0; dd < 2; ++dd) {
+    std::vector<es::StashSegDesc> segs;
+    uint64_t nbytes = 0;
+    for (int32_t i = 0; i < n; ++i) {
+      const es::BucketPlan &b = p.bp[buckets[i]];
+      if ((int)b.dtype != dd || b.L == 0) continue;
+      for (int32_t li = 0; li < h->n_local; ++li) {
+        const void *bw = h->borrowed[(size_t)li * h->B + buckets[i]];
+        if (!bw) continue;
+        unsigned char *slot = h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[buckets[i]];
+        const unsigned char *src = reinterpret_cast<const unsigned char *>(bw);
+        if (b.shard_lo > 0) segs.push_back({src, slot, b.shard_lo});
+        if ((uint64_t)b.shard_hi < b.L)
+          segs.push_back({src + (uint64_t)b.shard_hi * b.esize, slot + (uint64_t)b.shard_hi * b.esize,
+                          (int64_t)(b.L - (uint64_t)b.shard_hi)});
+        nbytes += 2 * (b.L - (uint64_t)(b.shard_hi - b.shard_lo)) * b.esize;
+      }
+    }
+    if (segs.empty()) continue;
+    s = h->timed(ES_KERNEL_STASH, nbytes, cs, [&](int *nl) {
+      return es::launch_stash_multi((es_dtype)dd, (es_dtype)dd, segs.data(), (int)segs.size(), cs, h->blocks_ov,
+                                    h->threads_ov, nl);
+    });
+    if (s != ES_OK) return s;
+  }
+  // 2. every rank's slots hold this step's contributions
+  if ((s = peer_barrier(h, cs)) != ES_OK) return s;
+  // 3. fold of the own shards
+  for (int dd = 0; dd < 2; ++dd) {
+    std::vector<es::FoldSegDesc> segs;
+    std::vector<std::vector<const void *>> srcs;
+    uint64_t nbytes = 0;
+    for (int32_t i = 0; i < n; ++i) {
+      const int32_t bk = buckets[i];
+      const es::BucketPlan &b = p.bp[bk];
+      if ((int)b.dtype != dd || b.shard_hi <= b.shard_lo) continue;
+      std::vector<const void *> src(p.N);
+      for (int32_t e = 0; e < p.N; ++e) {
+        const int32_t li = p.local_index[e];
+        const void *bw = li >= 0 ? h->borrowed[(size_t)li * h->B + bk] : nullptr;
+        const unsigned char *base = bw ? reinterpret_cast<const unsigned char *>(bw) : slot_of(p.est_to_gpu[e], e, bk);
+        src[e] = base + (uint64_t)b.shard_lo * b.esize;
+      }
+      es::FoldSegDesc d;
+      d.lo = b.shard_lo;
+      d.n = b.shard_hi - b.shard_lo;
+      d.C = (uint32_t)b.C;
+      d.rot = true;
+      d.out = h->ws + p.result_off + p.slot_off[bk] + (uint64_t)b.shard_lo * b.esize;
+      nbytes += (uint64_t)d.n * ((uint64_t)p.N + 1) * b.esize;
+      segs.push_back(d);
+      srcs.push_back(std::move(src));
+    }
+    if (segs.empty()) continue;
+    for (size_t i = 0; i < segs.size(); ++i) segs[i].src = srcs[i].data();
+    s = h->timed(ES_KERNEL_FOLD, nbytes, cs, [&](int *nl) {
+      return es::launch_fold_multi((es_dtype)dd, p.N, r, p.compat, segs.data(), (int)segs.size(), cs, h->blocks_ov,
+                                   h->threads_ov, nl);
+    });
+    if (s != ES_OK) return s;
+  }
+  // 4. every shard result is ready; every slot has been read
+  if ((s = peer_barrier(h, cs)) != ES_OK) return s;
+  // 5. gather every shard from its owner
+  for (int dd = 0; dd < 2; ++dd) {
+    std::vector<es::StashSegDesc> segs;
+    uint64_t nbytes = 0;
+    for (int32_t i = 0; i < n; ++i) {
+      const int32_t bk = buckets[i];
+      const es::BucketPlan &b = p.bp[bk];
+      if ((int)b.dtype != dd || b.L == 0) continue;
+      unsigned char *outp = reinterpret_cast<unsigned char *>(outs[i]);
+      const uint64_t S = es::chunk_elems(b.L, p.G, p.A);
+      for (int32_t o = 0; o < p.G; ++o) {
+        const uint64_t lo = std::min<uint64_t>(b.L, S * o), hi = std::min<uint64_t>(b.L, S * (o + 1));
+        if (hi <= lo) continue;
+        segs.push_back({h->peer_ws[o] + p.result_off + p.slot_off[bk] + lo * b.esize, outp + lo * b.esize,
+                        (int64_t)(hi - lo)});
+        nbytes += 2 * (hi - lo) * b.esize;
+      }
+    }
+    if (segs.empty()) continue;
+    s = h->timed(ES_KERNEL_GATHER, nbytes, cs, [&](int *nl) {
+      return es::launch_stash_multi((es_dtype)dd, (es_dtype)dd, segs.data(), (int)segs.size(), cs, h->blocks_ov,
+                                    h->threads_ov, nl);
+    });
+    if (s != ES_OK) return s;
+  }
+  (void)g;
+  return ES_OK;
+}
+}  // namespace
+
 es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void *const *outs, es_stream stream) {
   es_status s = check_handle(h);
   if (s != ES_OK) return s;
@@ -502,6 +634,11 @@ es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void
     return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
 
   const float r = 1.0f / (float)p.N;   // R5: fl32(1/N), correctly rounded fp32 division
+
+  if (p.peer) {
+    if ((s = peer_allreduce(h, n, buckets, outs, cs, r)) != ES_OK) return s;
+    return finish_allreduce(h, n, buckets, cs, cap);
+  }
 
   // Pending FOLD ops: consecutive folds (across buckets for G == 1, within a
   // chain round for G > 1) are independent and go out as one multi-segment
@@ -601,6 +738,12 @@ es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void
     }
   }
   if ((s = flush()) != ES_OK) return s;
+  return finish_allreduce(h, n, buckets, cs, cap);
+}
+
+namespace {
+
+es_status finish_allreduce(es_handle h, int32_t n, const int32_t *buckets, cudaStream_t cs, unsigned long long cap) {
   for (int32_t i = 0; i < n; ++i) {
     const int32_t bucket = buckets[i];
     if (cudaEventRecord(h->ar_ev[bucket], cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaEventRecord failed");
@@ -616,8 +759,118 @@ es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void
   return ES_OK;
 }
 
+}  // namespace
+
 es_status es_allreduce(es_handle h, int32_t bucket, void *out, es_stream stream) {
   return es_allreduce_many(h, 1, &bucket, &out, stream);
+}
+
+// ---- peer memory ---------------------------------------------------------------------
+
+namespace {
+
+struct PeerBlob {
+  char magic[8];            // "ESPEER01"
+  int32_t rank, pid;
+  uint64_t raw;             // workspace address in the owner's process
+  uint64_t offset;          // workspace - allocation base
+  uint64_t ws_bytes;
+  int32_t ipc_ok, pad;
+  cudaIpcMemHandle_t handle;
+};
+static_assert(sizeof(PeerBlob) <= ES_PEER_BLOB_BYTES, "peer blob too large");
+
+// Base of the allocation that contains p (driver cuMemGetAddressRange,
+// resolved through the runtime so libes has no link-time libcuda dependency).
+bool allocation_base(void *p, void **base) {
+  typedef int (*Fn)(unsigned long long *, size_t *, unsigned long long);
+  static Fn fn = nullptr;
+  if (!fn) {
+    void *sym = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &sym, cudaEnableDefault, &q) != cudaSuccess || !sym) {
+      cudaGetLastError();
+      return false;
+    }
+    fn = reinterpret_cast<Fn>(sym);
+  }
+  unsigned long long b = 0;
+  size_t sz = 0;
+  if (fn(&b, &sz, (unsigned long long)(uintptr_t)p) != 0) return false;
+  *base = reinterpret_cast<void *>((uintptr_t)b);
+  return true;
+}
+
+}  // namespace
+
+es_status es_peer_blob(es_handle h, void *blob, size_t bytes) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  if (!blob || bytes < ES_PEER_BLOB_BYTES) return set_err(ES_EINVAL, "blob must hold ES_PEER_BLOB_BYTES");
+  PeerBlob b;
+  std::memset(&b, 0, sizeof b);
+  std::memcpy(b.magic, "ESPEER01", 8);
+  b.rank = h->plan.rank;
+  b.pid = (int32_t)getpid();
+  b.raw = (uint64_t)(uintptr_t)h->ws;
+  b.ws_bytes = h->ws_bytes;
+  void *base = nullptr;
+  if (allocation_base(h->ws, &base) && cudaIpcGetMemHandle(&b.handle, base) == cudaSuccess) {
+    b.ipc_ok = 1;
+    b.offset = (uint64_t)((uintptr_t)h->ws - (uintptr_t)base);
+  } else {
+    cudaGetLastError();
+  }
+  std::memset(blob, 0, ES_PEER_BLOB_BYTES);
+  std::memcpy(blob, &b, sizeof b);
+  return ES_OK;
+}
+
+es_status es_peer_open(es_handle h, const void *blobs, size_t bytes) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  const es::Plan &p = h->plan;
+  if (!blobs || bytes < (size_t)p.G * ES_PEER_BLOB_BYTES) return set_err(ES_EINVAL, "need G blobs");
+  if (h->peer_open) return set_err(ES_ESTATE, "peers already open");
+  std::vector<unsigned char *> ws(p.G, nullptr);
+  std::vector<void *> mapped;
+  const int32_t me = (int32_t)getpid();
+  for (int32_t g = 0; g < p.G; ++g) {
+    PeerBlob b;
+    std::memcpy(&b, reinterpret_cast<const unsigned char *>(blobs) + (size_t)g * ES_PEER_BLOB_BYTES, sizeof b);
+    if (std::memcmp(b.magic, "ESPEER01", 8) != 0 || b.rank != g) {
+      for (void *m : mapped) cudaIpcCloseMemHandle(m);
+      return set_err(ES_EINVAL, "blob g is not rank g's es_peer_blob");
+    }
+    int32_t n_g = 0;
+    for (int32_t e = 0; e < p.N; ++e) n_g += p.est_to_gpu[e] == g;
+    if (b.ws_bytes < p.grad_off + (uint64_t)n_g * p.slot_block) {
+      for (void *m : mapped) cudaIpcCloseMemHandle(m);
+      return set_err(ES_EINVAL, "peer workspace smaller than this layout");
+    }
+    if (g == p.rank) {
+      ws[g] = h->ws;
+    } else if (b.pid == me) {
+      ws[g] = reinterpret_cast<unsigned char *>((uintptr_t)b.raw);     // same process (loopback)
+    } else {
+      if (!b.ipc_ok) {
+        for (void *m : mapped) cudaIpcCloseMemHandle(m);
+        return set_err(ES_EUNSUPPORTED, "peer workspace is not IPC-exportable");
+      }
+      void *ptr = nullptr;
+      if (cudaIpcOpenMemHandle(&ptr, b.handle, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+        cudaGetLastError();
+        for (void *m : mapped) cudaIpcCloseMemHandle(m);
+        return set_err(ES_ECUDA, "cudaIpcOpenMemHandle failed");
+      }
+      mapped.push_back(ptr);
+      ws[g] = reinterpret_cast<unsigned char *>(ptr) + b.offset;
+    }
+  }
+  h->peer_ws = ws;
+  h->ipc_mapped = mapped;
+  h->peer_open = true;
+  return ES_OK;
 }
 
 // ---- zero-copy slots and elastic resume ------------------------------------------

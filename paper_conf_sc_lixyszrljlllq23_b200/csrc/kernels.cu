@@ -644,6 +644,39 @@ __global__ void __launch_bounds__(256) k_dropout(const __grid_constant__ Dropout
   }
 }
 
+// ---- k_peer_barrier (ES_SCHED_PEER) -------------------------------------------
+
+struct BarrierParams {
+  uint64_t *peer_flags[64];
+  uint64_t *my_flags;
+  int32_t G, rank;
+  uint64_t epoch;
+};
+
+__global__ void __launch_bounds__(64) k_peer_barrier(const __grid_constant__ BarrierParams p) {
+  pdl_enter();
+  const int t = threadIdx.x;
+  __threadfence_system();                       // this GPU's completed writes before the arrival
+  if (t < p.G) {
+    uint64_t *dst = p.peer_flags[t] + p.rank;
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(dst), "l"(p.epoch) : "memory");
+  }
+  if (t < p.G) {
+    const uint64_t *src = p.my_flags + t;
+    uint64_t v = 0, t0 = 0, now = 0;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+    do {
+      asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(src) : "memory");
+      if (v >= p.epoch) break;
+      __nanosleep(256);
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now));
+      if (now - t0 > 60ull * 1000000000ull) __trap();   // a peer never arrived: fail loudly, never hang the GPU
+    } while (true);
+  }
+  __syncthreads();
+  __threadfence_system();
+}
+
 }  // namespace
 
 void set_pdl(bool on) { g_pdl = on; }
@@ -695,6 +728,18 @@ cudaError_t launch_dropout(es_dtype dtype, const void *x, void *y, uint8_t *mask
   const int blocks = (int)std::min<int64_t>((nq + 255) / 256, (int64_t)kSMs * 16);
   if (dtype == ES_BF16) return launch(k_dropout<BF16T>, dim3(blocks), dim3(256), s, d);
   return launch(k_dropout<F32T>, dim3(blocks), dim3(256), s, d);
+}
+
+cudaError_t launch_peer_barrier(uint64_t *const *peer_flags, uint64_t *my_flags, int32_t G, int32_t rank,
+                                uint64_t epoch, cudaStream_t s) {
+  if (G < 1 || G > 64) return cudaErrorInvalidValue;
+  BarrierParams b;
+  for (int i = 0; i < 64; ++i) b.peer_flags[i] = i < G ? peer_flags[i] : nullptr;
+  b.my_flags = my_flags;
+  b.G = G;
+  b.rank = rank;
+  b.epoch = epoch;
+  return launch(k_peer_barrier, dim3(1), dim3(64), s, b);
 }
 
 cudaError_t launch_swap(const SwapEntry *table_dev, int32_t n, uint64_t max_nbytes, int32_t cur, int32_t next,

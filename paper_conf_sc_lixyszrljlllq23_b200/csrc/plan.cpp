@@ -141,6 +141,28 @@ void plan_direct(const Plan &p, BucketPlan *b) {
   b->ops.push_back(make_op(ES_OP_GROUP_END));
 }
 
+// PEER (fused pull over peer memory): barrier (every rank's slots hold
+// this step's contributions) -> fold of the own shard reading remote
+// contributions from the owners' slots, result into the own RESULT area ->
+// barrier (every shard result is ready; every slot has been read) -> gather
+// of every shard from its owner's RESULT area into out.
+void plan_peer(const Plan &p, BucketPlan *b) {
+  const int32_t g = p.rank;
+  b->sched = ES_SCHED_PEER;
+  if (b->L == 0) return;
+  Range own = shard_range(b->L, p.G, p.A, g);
+  b->shard_lo = own.lo;
+  b->shard_hi = own.hi;
+  b->ops.push_back(make_op(ES_OP_BARRIER, 0));
+  if (own.hi > own.lo)
+    b->ops.push_back(make_op(ES_OP_FOLD, own.lo, own.hi, -1, p.N, ES_BUF_NONE, 0, ES_BUF_RESULT, 0));
+  b->ops.push_back(make_op(ES_OP_BARRIER, 1));
+  for (int32_t h = 0; h < p.G; ++h) {
+    Range s = shard_range(b->L, p.G, p.A, h);
+    if (s.hi > s.lo) b->ops.push_back(make_op(ES_OP_GATHER, s.lo, s.hi, h));
+  }
+}
+
 void plan_chain(const Plan &p, BucketPlan *b) {
   const int32_t g = p.rank;
   b->sched = ES_SCHED_CHAIN;
@@ -253,13 +275,14 @@ bool validate(const es_config *cfg, std::string *err, bool need_comm) {
   for (int32_t i = 0; i < cfg->n_state; ++i)
     if (cfg->state_nbytes[i] == 0 || cfg->state_nbytes[i] > (1ull << 31))
       return fail(err, "state_nbytes must be in [1, 2^31]");
-  if (cfg->sched != ES_SCHED_AUTO && cfg->sched != ES_SCHED_DIRECT && cfg->sched != ES_SCHED_CHAIN)
+  if (cfg->sched != ES_SCHED_AUTO && cfg->sched != ES_SCHED_DIRECT && cfg->sched != ES_SCHED_CHAIN &&
+      cfg->sched != ES_SCHED_PEER)
     return fail(err, "bad sched");
   if (cfg->compat & ~(uint32_t)(ES_COMPAT_PREDIV | ES_COMPAT_PREMUL | ES_COMPAT_BF16_HOP))
     return fail(err, "unknown compat bits");
   if ((cfg->compat & ES_COMPAT_PREDIV) && (cfg->compat & ES_COMPAT_PREMUL))
     return fail(err, "compat PREDIV and PREMUL are exclusive");
-  if (cfg->G > 1 && need_comm) {
+  if (cfg->G > 1 && need_comm && cfg->sched != ES_SCHED_PEER) {
     if (cfg->transport != ES_TRANSPORT_NCCL && cfg->transport != ES_TRANSPORT_LOOPBACK)
       return fail(err, "G > 1 needs transport NCCL or LOOPBACK");
     if (!cfg->comm) return fail(err, "G > 1 needs comm");
@@ -314,6 +337,7 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
         s = ch < d ? ES_SCHED_CHAIN : ES_SCHED_DIRECT;
       }
       if (s == ES_SCHED_CHAIN) plan_chain(*p, &b);
+      else if (s == ES_SCHED_PEER) plan_peer(*p, &b);
       else plan_direct(*p, &b);
     }
     max_stage = std::max(max_stage, b.stage_bytes);
@@ -328,8 +352,18 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
     off += align256(p->bp[bi].L * p->bp[bi].esize);
   }
   p->slot_block = off;
-  p->grad_off = 0;
-  uint64_t total = p->slot_block * p->local_ests.size();
+  // PEER: the regions peers address (flags, shard results, gradient slots)
+  // come first, at offsets that depend only on the layout -- identical on
+  // every rank whatever its number of local ESTs.
+  p->peer = p->G > 1 && p->sched_req == ES_SCHED_PEER;
+  uint64_t head = 0;
+  if (p->peer) {
+    p->flags_off = 0;
+    p->result_off = align256(64 * 8);
+    head = p->result_off + p->slot_block;   // one bucket-layout block: shard results at bucket offsets
+  }
+  p->grad_off = head;
+  uint64_t total = head + p->slot_block * p->local_ests.size();
   off = 0;
   p->state_off.resize(p->state_nbytes.size());
   for (size_t i = 0; i < p->state_nbytes.size(); ++i) {
@@ -347,6 +381,11 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
   total += max_stage;
   p->parts_off = total;
   total += max_parts;
+  p->owner_index.assign(p->N, 0);
+  {
+    std::vector<int32_t> cnt(p->G, 0);
+    for (int32_t e = 0; e < p->N; ++e) p->owner_index[e] = cnt[p->est_to_gpu[e]]++;
+  }
   p->total = align256(total);
   return ES_OK;
 }

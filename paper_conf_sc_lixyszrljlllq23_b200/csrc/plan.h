@@ -67,6 +67,10 @@ struct Plan {
   uint64_t scratch_off = 0;             // 256 B of zeroed scratch (dropout grid counter)
   uint64_t stage_off = 0;               // exchange staging (max over buckets)
   uint64_t parts_off = 0;               // chain partials (max over buckets)
+  uint64_t flags_off = 0;               // PEER: G barrier flags (u64) written by peers
+  uint64_t result_off = 0;              // PEER: per-bucket shard results (slot-block layout)
+  bool peer = false;                    // some bucket uses ES_SCHED_PEER
+  std::vector<int32_t> owner_index;     // [N]: EST's index among its owner's local ESTs
   uint64_t total = 0;
 };
 

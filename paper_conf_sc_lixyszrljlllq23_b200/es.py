@@ -16,19 +16,20 @@ from . import _build
 ES_OK, ES_EINVAL, ES_ESTATE, ES_ENOMEM, ES_ECUDA, ES_ENCCL, ES_EUNSUPPORTED = range(7)
 ES_F32, ES_BF16 = 0, 1
 ES_STASH_COPY, ES_STASH_BORROW, ES_STASH_INPLACE = 0, 1, 2
-ES_SCHED_AUTO, ES_SCHED_DIRECT, ES_SCHED_CHAIN = 0, 1, 2
+ES_SCHED_AUTO, ES_SCHED_DIRECT, ES_SCHED_CHAIN, ES_SCHED_PEER = 0, 1, 2, 3
 ES_TRANSPORT_NONE, ES_TRANSPORT_NCCL, ES_TRANSPORT_LOOPBACK = 0, 1, 2
-ES_KERNEL_STASH, ES_KERNEL_FOLD, ES_KERNEL_SWAP, ES_KERNEL_DROPOUT = 0, 1, 2, 3
+ES_KERNEL_STASH, ES_KERNEL_FOLD, ES_KERNEL_SWAP, ES_KERNEL_DROPOUT, ES_KERNEL_GATHER, ES_KERNEL_BARRIER = range(6)
 ES_OP_FIELDS = 10
-ES_OP_FOLD, ES_OP_SEND, ES_OP_RECV, ES_OP_GROUP_BEGIN, ES_OP_GROUP_END = 1, 2, 3, 4, 5
-ES_BUF_NONE, ES_BUF_SRC, ES_BUF_STAGE, ES_BUF_PART, ES_BUF_OUT = 0, 1, 2, 3, 4
+ES_OP_FOLD, ES_OP_SEND, ES_OP_RECV, ES_OP_GROUP_BEGIN, ES_OP_GROUP_END, ES_OP_BARRIER, ES_OP_GATHER = range(1, 8)
+ES_BUF_NONE, ES_BUF_SRC, ES_BUF_STAGE, ES_BUF_PART, ES_BUF_OUT, ES_BUF_RESULT = range(6)
+ES_PEER_BLOB_BYTES = 128
 ES_COMPAT_PREDIV, ES_COMPAT_PREMUL, ES_COMPAT_BF16_HOP = 1, 2, 4
 
 EXPORTED = [
     "es_workspace_bytes", "es_init", "es_destroy", "es_sync", "es_register_state", "es_init_state",
     "es_read_state", "es_switch_context", "es_stash_grad", "es_stash_grads", "es_stash_and_switch", "es_allreduce",
     "es_allreduce_many", "es_chunk_elems", "es_slot_ptr", "es_context_bytes", "es_export_context",
-    "es_import_context", "es_dropout",
+    "es_import_context", "es_dropout", "es_peer_blob", "es_peer_open",
     "es_plan_ops", "es_loopback_create", "es_loopback_destroy", "es_profile_enable",
     "es_profile_reset", "es_profile_query", "es_set_launch_override", "es_status_string",
     "es_last_error", "es_abi_version",
@@ -95,6 +96,8 @@ def lib():
         "es_chunk_elems": (u64, [u64, i32, u32]),
         "es_slot_ptr": (st, [P, i32, i32, ctypes.POINTER(P)]),
         "es_dropout": (st, [P, P, P, P, u64, ctypes.c_int, ctypes.c_float, i32, P]),
+        "es_peer_blob": (st, [P, P, sz]),
+        "es_peer_open": (st, [P, P, sz]),
         "es_context_bytes": (st, [P, ctypes.POINTER(sz)]),
         "es_export_context": (st, [P, i32, P, sz, P]),
         "es_import_context": (st, [P, i32, P, sz, P]),
@@ -244,6 +247,18 @@ def es_import_context(h, est, blob, stream):
 def es_dropout(h, x_ptr, y_ptr, mask_ptr, n, dtype, p, state_idx, stream):
     _check(lib().es_dropout(h, ctypes.c_void_p(x_ptr), ctypes.c_void_p(y_ptr), ctypes.c_void_p(mask_ptr), n, dtype,
                             float(p), state_idx, ctypes.c_void_p(stream)), "es_dropout")
+
+
+def es_peer_blob(h):
+    buf = ctypes.create_string_buffer(ES_PEER_BLOB_BYTES)
+    _check(lib().es_peer_blob(h, buf, ES_PEER_BLOB_BYTES), "es_peer_blob")
+    return buf.raw
+
+
+def es_peer_open(h, blobs):
+    data = b"".join(blobs)
+    buf = ctypes.create_string_buffer(data, len(data))
+    _check(lib().es_peer_open(h, buf, len(data)), "es_peer_open")
 
 
 def es_chunk_elems(L, N, A=16):

@@ -37,7 +37,10 @@ class RankExec:
         cfg = es.Config(N, G, rank, mapping, [(L, es.ES_F32 if d == "f32" else es.ES_BF16) for L, d in buckets], A,
                         sched=sched)
         self.plans = [es.es_plan_ops(cfg, b) for b in range(len(buckets))]
+        self.sched = sched
         self.out = [np.zeros(L, np.float32 if d == "f32" else np.uint16) for L, d in buckets]
+        self.result = [np.zeros(L, np.float32 if d == "f32" else np.uint16) for L, d in buckets]   # PEER
+        self.nbar = 0
         self.b = 0
         self.pc = 0
         self.stage = {}
@@ -50,8 +53,8 @@ class RankExec:
 
     def _src(self, e, lo, hi):
         b = self.b
-        if self.map[e] == self.g:
-            return self.xs[b][e][lo:hi]
+        if self.map[e] == self.g or self.sched == es.ES_SCHED_PEER:
+            return self.xs[b][e][lo:hi]          # local slot, or (PEER) the owner's slot over NVLink
         slo, arr = self.stage[e]
         assert slo <= lo and hi <= slo + arr.size, "staging does not cover the fold range"
         return arr[lo - slo:hi - slo]
@@ -85,7 +88,10 @@ class RankExec:
                 rest = order[1:]
             for e in rest:
                 acc = (acc + widen(self._src(e, a, z))).astype(np.float32)
-            if outk == es.ES_BUF_PART:
+            if outk == es.ES_BUF_RESULT:
+                r = np.float32(1) / np.float32(self.N)
+                self.result[self.b][a:z] = narrow(acc * r, d)
+            elif outk == es.ES_BUF_PART:
                 if outid not in self.parts:
                     self.parts[outid] = (lo, np.zeros(hi - lo, np.float32))
                 plo, parr = self.parts[outid]
@@ -135,6 +141,14 @@ class RankExec:
             if op == es.ES_OP_FOLD:
                 self._fold(f)
                 self.pc += 1
+            elif op == es.ES_OP_BARRIER:
+                if not transport.barrier(self):
+                    return progressed
+                self.pc += 1
+            elif op == es.ES_OP_GATHER:
+                lo, hi, owner = int(f[1]), int(f[2]), int(f[3])
+                self.out[self.b][lo:hi] = transport.ranks[owner].result[self.b][lo:hi]
+                self.pc += 1
             elif op == es.ES_OP_GROUP_BEGIN:
                 end = self.pc + 1
                 while int(ops[end][0]) != es.ES_OP_GROUP_END:
@@ -152,9 +166,23 @@ class RankExec:
 class Mailbox:
     """In-process transport: NCCL-like per-(src, dst) FIFO matching."""
 
-    def __init__(self):
+    def __init__(self, ranks=()):
         self.q = collections.defaultdict(collections.deque)
         self.posted = {}
+        self.ranks = list(ranks)
+        self.arrived = collections.Counter()
+
+    def barrier(self, ex):
+        """PEER barrier: passes once every rank has arrived at its n-th barrier."""
+        key = ex.nbar
+        if not getattr(ex, "_at_barrier", False):
+            self.arrived[key] += 1
+            ex._at_barrier = True
+        if self.arrived[key] < len(self.ranks):
+            return False
+        ex._at_barrier = False
+        ex.nbar += 1
+        return True
 
     def group(self, ex, body):
         key = (ex.g, ex.b, ex.pc)
@@ -181,7 +209,7 @@ class Mailbox:
 
 def simulate(N, G, mapping, buckets, xs, A=16, sched=es.ES_SCHED_AUTO):
     ranks = [RankExec(N, G, g, mapping, buckets, xs, A, sched) for g in range(G)]
-    box = Mailbox()
+    box = Mailbox(ranks)
     while not all(r.done() for r in ranks):
         if not any(r.run(box) for r in ranks if not r.done()):
             raise AssertionError("deadlock: no rank can progress")
