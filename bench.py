@@ -44,6 +44,8 @@ def parse():
                    help="one es_stash_grad / es_allreduce call per bucket (DDP-style) instead of the batched calls")
     p.add_argument("--no-fuse", action="store_true",
                    help="separate es_switch_context and es_stash_grads launches instead of es_stash_and_switch")
+    p.add_argument("--incremental", action="store_true",
+                   help="NEXT-1: fold each EST into running partials at its switch (es_stash_fold_grads, G == 1)")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     p.add_argument("--cpu-seconds", type=float, default=10.0)
@@ -228,7 +230,7 @@ def main():
     snb = workloads.state_nbytes()
     agg = Aggregator(N, G, rank, mapping, buckets, state_nbytes=snb,
                      transport=es.ES_TRANSPORT_NONE if G == 1 else es.ES_TRANSPORT_NCCL, comm=comm, sched=sched,
-                     device=dev)
+                     device=dev, options=es.ES_OPT_INCREMENTAL if args.incremental else 0)
     if G > 1 and sched == es.ES_SCHED_PEER:
         agg.peer_connect()                       # CUDA IPC map of every peer's workspace (NVLink)
     live = [torch.zeros(n, dtype=torch.uint8, device=dev) for n in snb]
@@ -243,9 +245,15 @@ def main():
     flush = None if in_bytes > 2 * L2_BYTES else torch.empty(4 * L2_BYTES, dtype=torch.uint8, device=dev)
     torch.cuda.synchronize()
 
-    fuse = not (args.per_bucket or args.no_fuse)
+    fuse = not (args.per_bucket or args.no_fuse or args.incremental)
 
     def step():
+        if args.incremental:
+            for i, k in enumerate(local):
+                agg.switch(k)
+                agg.stash_fold(k, range(B), grads[k], es.ES_STASH_BORROW if i == len(local) - 1 else es.ES_STASH_COPY)
+            agg.allreduce_many(range(B), outs)
+            return
         if fuse:
             # switch-in of the first local EST, then per EST: stash its
             # buckets + switch to the next EST in one launch
@@ -348,7 +356,7 @@ def main():
     per_launch = fl_bytes / max(fl_n, 1)
     traffic = None
     tfile = os.path.join(ROOT, "profiles", f"traffic_{name}_g{G}.json")
-    if os.path.exists(tfile):
+    if os.path.exists(tfile) and not (args.incremental or args.per_bucket or args.no_fuse or args.no_graph):
         with open(tfile) as f:
             traffic = json.load(f).get("fold_dram_bytes_per_launch")
 
@@ -358,7 +366,8 @@ def main():
         "vs_baseline": None, "dtype": cfg["dtype"], "data": "synthetic",
         "config": {"workload": name, "N": N, "G": G, "mapping": args.mapping, "sched": args.sched,
                    "buckets": B, "elements": sum(n for n, _ in buckets), "graph": graph is not None,
-                   "api": "per-bucket" if args.per_bucket else ("batched" if args.no_fuse else "batched+fused-switch"),
+                   "api": "per-bucket" if args.per_bucket else ("incremental" if args.incremental else
+                                                               ("batched" if args.no_fuse else "batched+fused-switch")),
                    "l2": ("inputs larger than L2 (%.1f MB of EST gradients per GPU per step)" % (in_bytes / 1e6))
                    if flush is None else "L2 flushed between timed steps (512 MB write)",
                    "desc": cfg["desc"]},

@@ -137,7 +137,12 @@ typedef struct {
   es_sched sched;
   uint32_t compat;                /* 0 = the canonical definition (R1-R6, R13); else ES_COMPAT_*
                                      bits.  Part of the persisted definition. */
+  uint32_t options;               /* ES_OPT_* bits (execution choices; never change bits)      */
 } es_config;
+
+/* ES_OPT_INCREMENTAL: reserve fp32 partials so that es_stash_fold_grads can
+ * fold each EST into the running partials at its switch (NEXT-1, G == 1). */
+#define ES_OPT_INCREMENTAL 1u
 
 /* NEXT-3 compatibility variants -- same canonical order, different step
  * arithmetic:
@@ -228,6 +233,23 @@ es_status es_stash_grads(es_handle h, int32_t est, int32_t n, const int32_t *buc
  * be a valid local EST (ES_EINVAL / ES_ESTATE otherwise). */
 es_status es_stash_and_switch(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
                               const es_dtype *grad_dtypes, es_stash_mode mode, int32_t next_est, es_stream stream);
+
+/* NEXT-1 incremental canonical fold (PAPER.md:599-606 overlaps
+ * the gradient swap with the next EST's compute): at EST `est`'s switch,
+ * fold its contribution straight into the running unrounded fp32 partials of
+ * the chunks c < est -- for them `est` comes after c+1..est-1 in canonical
+ * order (R2), and ESTs run in index order -- and stash only chunks >= est,
+ * which wait for the wrap.  es_allreduce of the bucket then folds the
+ * partials with the stashed 0..c of each chunk: the end-of-step critical
+ * path reads ~(N+3)/2 contributions per element instead of N+1, with the
+ * same bits (segmentability, R14) and about the same total bytes.
+ * Requirements: G == 1, cfg.options has ES_OPT_INCREMENTAL, every EST of the
+ * step calls this for the bucket in order 0, 1, ..., N-1 (ES_ESTATE
+ * otherwise; mixing with es_stash_grad for the same bucket and step is an
+ * ES_ESTATE error).  mode: COPY (the stashed part is copied) or BORROW (the
+ * buffer is kept until es_allreduce completes). */
+es_status es_stash_fold_grads(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
+                              const es_dtype *grad_dtypes, es_stash_mode mode, es_stream stream);
 
 /* ---- aggregation ---------------------------------------------------------- */
 

@@ -37,12 +37,12 @@ class Aggregator:
     """
 
     def __init__(self, N, G, rank, est_to_gpu, buckets, chunk_align=16, state_nbytes=(),
-                 transport=None, comm=None, sched=es.ES_SCHED_AUTO, device=None, compat=0):
+                 transport=None, comm=None, sched=es.ES_SCHED_AUTO, device=None, compat=0, options=0):
         if transport is None:
             transport = es.ES_TRANSPORT_NONE if G == 1 else es.ES_TRANSPORT_NCCL
         self.buckets = [(int(n), DTYPES[d]) for n, d in buckets]
         self.cfg = es.Config(N, G, rank, est_to_gpu, self.buckets, chunk_align, tuple(state_nbytes),
-                             transport, comm, sched, compat)
+                             transport, comm, sched, compat, options)
         self.N, self.G, self.rank = N, G, rank
         self.local_ests = [e for e in range(N) if est_to_gpu[e] == rank]
         self.device = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
@@ -107,6 +107,11 @@ class Aggregator:
         es.es_stash_and_switch(self.h, est, list(buckets), [g.data_ptr() for g in grads],
                                [DTYPES[g.dtype] for g in grads], mode, next_est, _stream(stream))
         self._mirror_generator(next_est)
+
+    def stash_fold(self, est, buckets, grads, mode=es.ES_STASH_COPY, stream=None):
+        """NEXT-1: fold EST `est` into the running partials now, stash the rest."""
+        es.es_stash_fold_grads(self.h, est, list(buckets), [g.data_ptr() for g in grads],
+                               [DTYPES[g.dtype] for g in grads], mode, _stream(stream))
 
     def allreduce_many(self, buckets, outs, stream=None):
         es.es_allreduce_many(self.h, list(buckets), [o.data_ptr() for o in outs], _stream(stream))

@@ -72,6 +72,9 @@ struct es_ctx {
   es_status sticky = ES_OK;
   std::string sticky_msg;
 
+  // NEXT-1 incremental fold: next EST expected per bucket (0: none folded yet)
+  std::vector<int32_t> inc_next;
+
   // ES_SCHED_PEER
   std::vector<unsigned char *> peer_ws;   // [G] workspace base of every rank, mapped here
   std::vector<void *> ipc_mapped;         // cudaIpcOpenMemHandle results to close
@@ -233,6 +236,7 @@ es_status es_init(const es_config *cfg, void *workspace, size_t workspace_bytes,
   h->ar_ev.assign(h->B, nullptr);
   h->ar_cap.assign(h->B, 0);
   h->ar_recorded.assign(h->B, 0);
+  h->inc_next.assign(h->B, 0);
   for (auto &e : h->stash_ev)
     if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
       return set_err(ES_ECUDA, "cudaEventCreate failed");
@@ -383,6 +387,9 @@ es_status stash_impl(es_handle h, int32_t est, int32_t n, const int32_t *buckets
   }
   const int32_t li = p.local_index[est];
   if (li < 0) return set_err(ES_ESTATE, "est is not mapped to this rank");
+  for (int32_t i = 0; i < n; ++i)
+    if (h->inc_next[buckets[i]] > 0)
+      return set_err(ES_ESTATE, "bucket is being folded incrementally this step (es_stash_fold_grads)");
   if (mode == ES_STASH_INPLACE)
     for (int32_t i = 0; i < n; ++i)
       if (p.bp[buckets[i]].L > 0 &&
@@ -463,6 +470,108 @@ es_status stash_impl(es_handle h, int32_t est, int32_t n, const int32_t *buckets
 es_status es_stash_grads(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
                          const es_dtype *gdts, es_stash_mode mode, es_stream stream) {
   return stash_impl(h, est, n, buckets, grads, gdts, mode, -1, stream);
+}
+
+es_status es_stash_fold_grads(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
+                              const es_dtype *gdts, es_stash_mode mode, es_stream stream) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  const es::Plan &p = h->plan;
+  if (!(p.options & ES_OPT_INCREMENTAL) || p.G != 1)
+    return set_err(ES_EUNSUPPORTED, "es_stash_fold_grads needs G == 1 and ES_OPT_INCREMENTAL");
+  if (n < 0 || (n > 0 && (!buckets || !grads || !gdts))) return set_err(ES_EINVAL, "bad bucket/grad arrays");
+  if (est < 0 || est >= p.N) return set_err(ES_EINVAL, "est out of range");
+  if (mode != ES_STASH_COPY && mode != ES_STASH_BORROW) return set_err(ES_EINVAL, "mode must be COPY or BORROW");
+  for (int32_t i = 0; i < n; ++i) {
+    const int32_t bk = buckets[i];
+    if (bk < 0 || bk >= h->B) return set_err(ES_EINVAL, "bucket out of range");
+    const es::BucketPlan &b = p.bp[bk];
+    if (gdts[i] != b.dtype) return set_err(ES_EINVAL, "incremental fold needs grad dtype == bucket dtype");
+    if (b.L > 0 && (!grads[i] || !aligned16(grads[i])))
+      return set_err(ES_EINVAL, "grad must be a 16-byte aligned device pointer");
+    for (int32_t j = 0; j < i; ++j)
+      if (buckets[j] == bk) return set_err(ES_EINVAL, "bucket listed twice");
+    if (h->inc_next[bk] != est)
+      return set_err(ES_ESTATE, "incremental fold expects the ESTs of a bucket in order 0, 1, ..., N-1");
+    if (est == 0)
+      for (int32_t li = 0; li < h->n_local; ++li)
+        if (h->stashed[(size_t)li * h->B + bk])
+          return set_err(ES_ESTATE, "bucket already stashed this step with es_stash_grad(s)");
+  }
+  const int32_t li = p.local_index[est];
+  cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
+  const unsigned long long cap = capture_id(cs);
+  for (int32_t i = 0; i < n; ++i) {
+    const int32_t bk = buckets[i];
+    if (h->ar_recorded[bk] && h->ar_cap[bk] == cap && cudaStreamWaitEvent(cs, h->ar_ev[bk], 0) != cudaSuccess)
+      return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
+  }
+  const float r = 1.0f / (float)p.N;
+  for (int dd = 0; dd < 2; ++dd) {
+    // (i) fold x_est into the partials of chunks c < est (R2: est follows c+1..est-1)
+    std::vector<es::FoldSegDesc> segs;
+    std::vector<std::vector<const void *>> srcs;
+    uint64_t fbytes = 0;
+    // (ii) stash chunks >= est (they wait for the wrap)
+    std::vector<es::StashSegDesc> st;
+    uint64_t sbytes = 0;
+    for (int32_t i = 0; i < n; ++i) {
+      const int32_t bk = buckets[i];
+      const es::BucketPlan &b = p.bp[bk];
+      if ((int)b.dtype != dd || b.L == 0) continue;
+      const unsigned char *x = reinterpret_cast<const unsigned char *>(grads[i]);
+      float *part = reinterpret_cast<float *>(h->ws + p.inc_off + p.inc_bucket_off[bk]);
+      const int64_t L = (int64_t)b.L, C = (int64_t)b.C;
+      const int64_t cont_hi = std::min<int64_t>(L, (int64_t)std::max(est - 1, 0) * C);   // chunks < est-1
+      const int64_t inc_hi = std::min<int64_t>(L, (int64_t)est * C);                     // chunks < est
+      auto add = [&](int64_t lo, int64_t hi, bool cont) {
+        if (hi <= lo) return;
+        es::FoldSegDesc d;
+        d.lo = lo;
+        d.n = hi - lo;
+        d.C = (uint32_t)b.C;
+        d.rot = false;
+        d.m = 1;
+        d.part_in = cont ? part + lo : nullptr;
+        d.out_partial = true;
+        d.out = part + lo;
+        segs.push_back(d);
+        srcs.push_back({x + (uint64_t)lo * b.esize});
+        fbytes += (uint64_t)(hi - lo) * (b.esize + (cont ? 8 : 4));
+      };
+      add(0, cont_hi, true);           // partial continues
+      add(cont_hi, inc_hi, false);     // chunk est-1: est is its first EST (c+1)
+      if (mode == ES_STASH_COPY && inc_hi < L) {
+        unsigned char *slot = h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[bk];
+        st.push_back({x + (uint64_t)inc_hi * b.esize, slot + (uint64_t)inc_hi * b.esize, L - inc_hi});
+        sbytes += 2 * (uint64_t)(L - inc_hi) * b.esize;
+      }
+    }
+    if (!segs.empty()) {
+      for (size_t j = 0; j < segs.size(); ++j) segs[j].src = srcs[j].data();
+      s = h->timed(ES_KERNEL_FOLD, fbytes, cs, [&](int *nl) {
+        return es::launch_fold_multi((es_dtype)dd, p.N, r, p.compat, segs.data(), (int)segs.size(), cs, h->blocks_ov,
+                                     h->threads_ov, nl);
+      });
+      if (s != ES_OK) return s;
+    }
+    if (!st.empty()) {
+      s = h->timed(ES_KERNEL_STASH, sbytes, cs, [&](int *nl) {
+        return es::launch_stash_multi((es_dtype)dd, (es_dtype)dd, st.data(), (int)st.size(), cs, h->blocks_ov,
+                                      h->threads_ov, nl);
+      });
+      if (s != ES_OK) return s;
+    }
+  }
+  for (int32_t i = 0; i < n; ++i) {
+    const size_t k = (size_t)li * h->B + buckets[i];
+    h->borrowed[k] = mode == ES_STASH_BORROW ? grads[i] : nullptr;
+    if (cudaEventRecord(h->stash_ev[k], cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaEventRecord failed");
+    h->stash_cap[k] = cap;
+    h->stashed[k] = 1;
+    h->inc_next[buckets[i]] = est + 1;
+  }
+  return ES_OK;
 }
 
 es_status es_stash_and_switch(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
@@ -618,10 +727,13 @@ es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void
       if (!h->stashed[(size_t)li * h->B + bk])
         return set_err(ES_ESTATE, "es_allreduce before every local EST stashed this bucket");
   }
-  for (int32_t i = 0; i < n; ++i)
+  for (int32_t i = 0; i < n; ++i) {
     for (int32_t li = 0; li < h->n_local; ++li)
       if (!h->stashed[(size_t)li * h->B + buckets[i]])
         return set_err(ES_ESTATE, "es_allreduce before every local EST stashed this bucket");
+    if (h->inc_next[buckets[i]] != 0 && h->inc_next[buckets[i]] != p.N)
+      return set_err(ES_ESTATE, "incremental fold of this bucket is incomplete");
+  }
   cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
   const unsigned long long cap = capture_id(cs);
   for (int32_t i = 0; i < n; ++i)
@@ -679,6 +791,33 @@ es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void
       return h->ws + p.parts_off + pt.off + (uint64_t)(lo - pt.lo) * 4;
     };
     unsigned char *outp = reinterpret_cast<unsigned char *>(outs[i]);
+    if (h->inc_next[bucket] == p.N && b.L > 0) {
+      // NEXT-1 end of step: chunk c < N-1 continues from its partial (ESTs
+      // c+1..N-1) over the stashed ESTs 0..c; chunk N-1 folds 0..N-1.
+      if (!pend.empty() && pend_dt != b.dtype && (s = flush()) != ES_OK) return s;
+      pend_dt = b.dtype;
+      const float *part = reinterpret_cast<const float *>(h->ws + p.inc_off + p.inc_bucket_off[bucket]);
+      for (int32_t c = 0; c < p.N; ++c) {
+        const int64_t lo = std::min<int64_t>((int64_t)b.L, (int64_t)c * (int64_t)b.C);
+        const int64_t hi = std::min<int64_t>((int64_t)b.L, (int64_t)(c + 1) * (int64_t)b.C);
+        if (hi <= lo) continue;
+        es::FoldSegDesc d;
+        d.lo = lo;
+        d.n = hi - lo;
+        d.C = (uint32_t)b.C;
+        d.rot = false;
+        const bool cont = c < p.N - 1;
+        d.m = cont ? c + 1 : p.N;
+        d.part_in = cont ? part + lo : nullptr;
+        d.out = outp + (uint64_t)lo * esz;
+        std::vector<const void *> src;
+        for (int32_t e = 0; e < d.m; ++e) src.push_back(src_base(e) + (uint64_t)lo * esz);
+        pend_bytes += (uint64_t)d.n * ((uint64_t)d.m * esz + (cont ? 4 : 0) + esz);
+        pend.push_back(d);
+        pend_src.push_back(std::move(src));
+      }
+      continue;
+    }
     for (const es::Op &op : b.ops) {
       const int64_t *f = op.f;
       switch (f[0]) {
@@ -755,6 +894,7 @@ es_status finish_allreduce(es_handle h, int32_t n, const int32_t *buckets, cudaS
       h->stashed[(size_t)li * h->B + bucket] = 0;
       h->borrowed[(size_t)li * h->B + bucket] = nullptr;
     }
+    h->inc_next[bucket] = 0;
   }
   return ES_OK;
 }

@@ -282,6 +282,8 @@ bool validate(const es_config *cfg, std::string *err, bool need_comm) {
     return fail(err, "unknown compat bits");
   if ((cfg->compat & ES_COMPAT_PREDIV) && (cfg->compat & ES_COMPAT_PREMUL))
     return fail(err, "compat PREDIV and PREMUL are exclusive");
+  if (cfg->options & ~(uint32_t)ES_OPT_INCREMENTAL) return fail(err, "unknown option bits");
+  if ((cfg->options & ES_OPT_INCREMENTAL) && cfg->G != 1) return fail(err, "ES_OPT_INCREMENTAL needs G == 1");
   if (cfg->G > 1 && need_comm && cfg->sched != ES_SCHED_PEER) {
     if (cfg->transport != ES_TRANSPORT_NCCL && cfg->transport != ES_TRANSPORT_LOOPBACK)
       return fail(err, "G > 1 needs transport NCCL or LOOPBACK");
@@ -315,6 +317,7 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
   p->comm = cfg->G > 1 ? cfg->comm : nullptr;
   p->sched_req = cfg->sched;
   p->compat = cfg->compat;
+  p->options = cfg->options;
 
   p->bp.resize(cfg->n_buckets);
   uint64_t max_stage = 0, max_parts = 0;
@@ -381,6 +384,16 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
   total += max_stage;
   p->parts_off = total;
   total += max_parts;
+  if (p->options & ES_OPT_INCREMENTAL) {
+    p->inc_off = align256(total);
+    uint64_t o = 0;
+    p->inc_bucket_off.resize(p->bp.size());
+    for (size_t bi = 0; bi < p->bp.size(); ++bi) {
+      p->inc_bucket_off[bi] = o;
+      o += align256(p->bp[bi].L * 4);
+    }
+    total = p->inc_off + o;
+  }
   p->owner_index.assign(p->N, 0);
   {
     std::vector<int32_t> cnt(p->G, 0);

@@ -54,6 +54,9 @@ struct Plan {
   void *comm = nullptr;
   es_sched sched_req = ES_SCHED_AUTO;
   uint32_t compat = 0;                  // NEXT-3 variant bits
+  uint32_t options = 0;                 // ES_OPT_* bits
+  uint64_t inc_off = 0;                 // NEXT-1: fp32 partials, bucket-major (inc_block bytes)
+  std::vector<uint64_t> inc_bucket_off; // [n_buckets]
   std::vector<BucketPlan> bp;
 
   // Workspace layout (byte offsets from the workspace base, 256-aligned).

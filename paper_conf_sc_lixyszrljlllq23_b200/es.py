@@ -24,10 +24,11 @@ ES_OP_FOLD, ES_OP_SEND, ES_OP_RECV, ES_OP_GROUP_BEGIN, ES_OP_GROUP_END, ES_OP_BA
 ES_BUF_NONE, ES_BUF_SRC, ES_BUF_STAGE, ES_BUF_PART, ES_BUF_OUT, ES_BUF_RESULT = range(6)
 ES_PEER_BLOB_BYTES = 128
 ES_COMPAT_PREDIV, ES_COMPAT_PREMUL, ES_COMPAT_BF16_HOP = 1, 2, 4
+ES_OPT_INCREMENTAL = 1
 
 EXPORTED = [
     "es_workspace_bytes", "es_init", "es_destroy", "es_sync", "es_register_state", "es_init_state",
-    "es_read_state", "es_switch_context", "es_stash_grad", "es_stash_grads", "es_stash_and_switch", "es_allreduce",
+    "es_read_state", "es_switch_context", "es_stash_grad", "es_stash_grads", "es_stash_and_switch", "es_stash_fold_grads", "es_allreduce",
     "es_allreduce_many", "es_chunk_elems", "es_slot_ptr", "es_context_bytes", "es_export_context",
     "es_import_context", "es_dropout", "es_peer_blob", "es_peer_open",
     "es_plan_ops", "es_loopback_create", "es_loopback_destroy", "es_profile_enable",
@@ -54,7 +55,7 @@ class es_config(ctypes.Structure):
         ("chunk_align", ctypes.c_uint32),
         ("n_state", ctypes.c_int32), ("state_nbytes", ctypes.POINTER(ctypes.c_uint64)),
         ("transport", ctypes.c_int), ("comm", ctypes.c_void_p), ("sched", ctypes.c_int),
-        ("compat", ctypes.c_uint32),
+        ("compat", ctypes.c_uint32), ("options", ctypes.c_uint32),
     ]
 
 
@@ -93,6 +94,8 @@ def lib():
         "es_allreduce_many": (st, [P, i32, ctypes.POINTER(i32), ctypes.POINTER(P), P]),
         "es_stash_and_switch": (st, [P, i32, i32, ctypes.POINTER(i32), ctypes.POINTER(P),
                                      ctypes.POINTER(ctypes.c_int), ctypes.c_int, i32, P]),
+        "es_stash_fold_grads": (st, [P, i32, i32, ctypes.POINTER(i32), ctypes.POINTER(P),
+                                     ctypes.POINTER(ctypes.c_int), ctypes.c_int, P]),
         "es_chunk_elems": (u64, [u64, i32, u32]),
         "es_slot_ptr": (st, [P, i32, i32, ctypes.POINTER(P)]),
         "es_dropout": (st, [P, P, P, P, u64, ctypes.c_int, ctypes.c_float, i32, P]),
@@ -130,7 +133,7 @@ class Config:
     """Owns an es_config and the host arrays it points to."""
 
     def __init__(self, N, G, rank, est_to_gpu, buckets, chunk_align=16, state_nbytes=(),
-                 transport=ES_TRANSPORT_NONE, comm=None, sched=ES_SCHED_AUTO, compat=0):
+                 transport=ES_TRANSPORT_NONE, comm=None, sched=ES_SCHED_AUTO, compat=0, options=0):
         self.N, self.G, self.rank = int(N), int(G), int(rank)
         self.est_to_gpu = list(int(g) for g in est_to_gpu)
         self.buckets = [(int(n), int(d)) for n, d in buckets]
@@ -139,7 +142,8 @@ class Config:
         self._sn = (ctypes.c_uint64 * max(len(state_nbytes), 1))(*state_nbytes)
         self.state_nbytes = list(state_nbytes)
         self.c = es_config(self.N, self.G, self.rank, self._map, self._bk, len(self.buckets), int(chunk_align),
-                           len(state_nbytes), self._sn, int(transport), comm, int(sched), int(compat))
+                           len(state_nbytes), self._sn, int(transport), comm, int(sched), int(compat),
+                           int(options))
 
     def ptr(self):
         return ctypes.byref(self.c)
@@ -211,6 +215,14 @@ def es_stash_and_switch(h, est, buckets, grad_ptrs, grad_dtypes, mode, next_est,
     d = (ctypes.c_int * max(n, 1))(*grad_dtypes)
     _check(lib().es_stash_and_switch(h, est, n, b, g, d, mode, next_est, ctypes.c_void_p(stream)),
            "es_stash_and_switch")
+
+
+def es_stash_fold_grads(h, est, buckets, grad_ptrs, grad_dtypes, mode, stream):
+    n = len(buckets)
+    b = (ctypes.c_int32 * max(n, 1))(*buckets)
+    g = (ctypes.c_void_p * max(n, 1))(*grad_ptrs)
+    d = (ctypes.c_int * max(n, 1))(*grad_dtypes)
+    _check(lib().es_stash_fold_grads(h, est, n, b, g, d, mode, ctypes.c_void_p(stream)), "es_stash_fold_grads")
 
 
 def es_allreduce_many(h, buckets, out_ptrs, stream):

@@ -448,3 +448,67 @@ def _loopback_compat(xs_per_bucket, G, mapping, sched, compat):
         a.close()
     es.es_loopback_destroy(world)
     return res
+
+
+# ---- NEXT-1 incremental canonical fold ---------------------------------------------------------
+
+@pytest.mark.parametrize("N", [1, 2, 3, 8, 12, 32])
+def test_incremental_fold_matches_oracle(N):
+    from gpu_util import Aggregator, from_dev, to_dev
+    rng = np.random.default_rng(900 + N)
+    Ls, dts = [100003, 40, 4099, 1], ["f32", "bf16", "f32", "bf16"]     # 40 < N*C for N >= 3: empty chunks
+    agg = Aggregator(N, 1, 0, [0] * N, list(zip(Ls, dts)), options=es.ES_OPT_INCREMENTAL)
+    outs = [agg.new_out(b) for b in range(len(Ls))]
+    for step in range(2):
+        xs = [_gauss(rng, N, L, d) for L, d in zip(Ls, dts)]
+        devs = [[to_dev(xs[b][k]) for b in range(len(Ls))] for k in range(N)]
+        for k in range(N):
+            agg.stash_fold(k, range(len(Ls)), devs[k], es.ES_STASH_BORROW if k == N - 1 else es.ES_STASH_COPY)
+        agg.allreduce_many(range(len(Ls)), outs)
+        torch.cuda.synchronize()
+        for b, d in enumerate(dts):
+            assert_bits_equal(from_dev(outs[b]), oracle.reduce(xs[b], d), f"step {step} N={N} b={b}")
+    agg.close()
+
+
+def test_incremental_fold_protocol_and_graph():
+    from gpu_util import Aggregator, from_dev, to_dev
+    N, L = 4, 5000
+    rng = np.random.default_rng(901)
+    xs = _gauss(rng, N, L)
+    devs = [to_dev(x) for x in xs]
+    agg = Aggregator(N, 1, 0, [0] * N, [(L, "f32")], options=es.ES_OPT_INCREMENTAL)
+    out = agg.new_out(0)
+    with pytest.raises(es.EsError) as e:              # must start with EST 0
+        agg.stash_fold(1, [0], [devs[1]])
+    assert e.value.status == es.ES_ESTATE
+    agg.stash_fold(0, [0], [devs[0]])
+    with pytest.raises(es.EsError) as e:              # no mixing with the plain stash
+        agg.stash(1, 0, devs[1])
+    assert e.value.status == es.ES_ESTATE
+    agg.stash_fold(1, [0], [devs[1]])
+    agg.stash_fold(2, [0], [devs[2]])
+    with pytest.raises(es.EsError) as e:              # incomplete: EST 3 has not run
+        agg.allreduce(0, out)
+    assert e.value.status == es.ES_ESTATE
+    agg.stash_fold(3, [0], [devs[3]])
+    agg.allreduce(0, out)
+    torch.cuda.synchronize()
+    assert_bits_equal(from_dev(out), oracle.reduce(xs, "f32"))
+    # the whole incremental step as a CUDA graph
+    s = torch.cuda.Stream()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        for k in range(N):
+            agg.stash_fold(k, [0], [devs[k]])
+        agg.allreduce(0, out)
+    out.zero_()
+    g.replay()
+    g.replay()
+    torch.cuda.synchronize()
+    assert_bits_equal(from_dev(out), oracle.reduce(xs, "f32"))
+    agg.close()
+    with pytest.raises(es.EsError) as e:              # G > 1 is refused at init
+        Aggregator(4, 2, 0, [0, 0, 1, 1], [(L, "f32")], options=es.ES_OPT_INCREMENTAL,
+                   transport=es.ES_TRANSPORT_LOOPBACK, comm=es.es_loopback_create(2).value)
+    assert e.value.status == es.ES_EINVAL
