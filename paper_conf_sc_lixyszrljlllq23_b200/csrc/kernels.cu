@@ -569,6 +569,158 @@ cudaError_t launch_stash_t(const StashSegDesc *segs, int nseg, cudaStream_t s, i
   return cudaSuccess;
 }
 
+// ---- k_copy_tma: TMA bulk-copy stash for same-dtype segments ------------------
+// One elected thread per CTA streams a contiguous, equal share of the bytes
+// through an S-stage shared-memory ring: cp.async.bulk global->shared
+// (completion on an mbarrier with expect_tx), then cp.async.bulk
+// shared->global.  Chosen with ES_STASH_TMA=1 (S=4 x 32 KB, 1 CTA/SM) or 2
+// (S=6 x 16 KB, 2 CTAs/SM); the default is the SM copy (k_stash), which
+// measured faster (profiles/).
+
+struct CopySeg {
+  const unsigned char *src;
+  unsigned char *dst;
+  uint64_t bytes;
+};
+
+struct CopyTmaParams {
+  int32_t nseg;
+  uint64_t total16;            // sum of floor16(bytes)
+  uint64_t per_cta;            // multiple of 16
+  CopySeg seg[32];
+};
+
+__device__ __forceinline__ uint32_t smem_addr(const void *p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+template <int S, int T>
+__global__ void __launch_bounds__(32) k_copy_tma(const __grid_constant__ CopyTmaParams p) {
+  extern __shared__ __align__(128) unsigned char ring[];
+  __shared__ __align__(8) uint64_t bars[S];
+  pdl_enter();
+  if (threadIdx.x != 0) return;
+  for (int st = 0; st < S; ++st)
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_addr(&bars[st])) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  uint64_t pos = (uint64_t)blockIdx.x * p.per_cta;
+  const uint64_t end = min(pos + p.per_cta, p.total16);
+  // cursor over the concatenated floor16 space
+  int si = 0;
+  uint64_t seg_base = 0;
+  auto next_tile = [&](const unsigned char *&src, unsigned char *&dst, uint32_t &n) -> bool {
+    while (pos < end) {
+      const uint64_t len = p.seg[si].bytes & ~uint64_t(15);
+      if (pos >= seg_base + len) {
+        seg_base += len;
+        ++si;
+        continue;
+      }
+      const uint64_t off = pos - seg_base;
+      const uint64_t take = min(min((uint64_t)T, end - pos), len - off);
+      src = p.seg[si].src + off;
+      dst = p.seg[si].dst + off;
+      n = (uint32_t)take;
+      pos += take;
+      return true;
+    }
+    return false;
+  };
+  const unsigned char *tsrc[S] = {};
+  unsigned char *tdst[S] = {};
+  uint32_t tn[S] = {};
+  auto load = [&](int st) {
+    const uint32_t bar = smem_addr(&bars[st]);
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(tn[st]) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_addr(ring + (size_t)st * T)), "l"(tsrc[st]), "r"(tn[st]), "r"(bar)
+                 : "memory");
+  };
+  int loaded = 0;
+  for (int st = 0; st < S && next_tile(tsrc[st], tdst[st], tn[st]); ++st) {
+    load(st);
+    ++loaded;
+  }
+  for (int i = 0; i < loaded; ++i) {
+    const int st = i % S;
+    const uint32_t bar = smem_addr(&bars[st]);
+    const uint32_t parity = (uint32_t)((i / S) & 1);
+    uint32_t ok = 0;
+    do {
+      asm volatile("{\n .reg .pred q;\n mbarrier.try_wait.parity.shared::cta.b64 q, [%1], %2;\n selp.u32 %0, 1, 0, q;\n}"
+                   : "=r"(ok)
+                   : "r"(bar), "r"(parity)
+                   : "memory");
+    } while (!ok);
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(tdst[st]),
+                 "r"(smem_addr(ring + (size_t)st * T)), "r"(tn[st])
+                 : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    const unsigned char *ns;
+    unsigned char *nd;
+    uint32_t nn;
+    if (next_tile(ns, nd, nn)) {
+      asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // stage st has been read out
+      tsrc[st] = ns;
+      tdst[st] = nd;
+      tn[st] = nn;
+      load(st);
+      ++loaded;
+    }
+  }
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+  // sub-16-byte tails of the segments: CTA (segment index % grid)
+  for (int k = 0; k < p.nseg; ++k) {
+    if ((uint32_t)k % gridDim.x != blockIdx.x) continue;
+    const uint64_t len = p.seg[k].bytes & ~uint64_t(15);
+    for (uint64_t b = len; b < p.seg[k].bytes; ++b) p.seg[k].dst[b] = p.seg[k].src[b];
+  }
+}
+
+template <int S, int T>
+cudaError_t launch_copy_tma(const StashSegDesc *segs, int nseg, int esize, cudaStream_t s, int ctas_per_sm,
+                            int *launches) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_copy_tma<S, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, S * T);
+    attr = true;
+  }
+  for (int i = 0; i < nseg; i += 32) {
+    const int k = std::min(32, nseg - i);
+    CopyTmaParams p;
+    p.nseg = k;
+    p.total16 = 0;
+    for (int j = 0; j < k; ++j) {
+      p.seg[j].src = reinterpret_cast<const unsigned char *>(segs[i + j].src);
+      p.seg[j].dst = reinterpret_cast<unsigned char *>(segs[i + j].dst);
+      p.seg[j].bytes = (uint64_t)segs[i + j].n * esize;
+      p.total16 += p.seg[j].bytes & ~uint64_t(15);
+    }
+    const int grid = kSMs * ctas_per_sm;
+    p.per_cta = ((p.total16 + grid - 1) / grid + 15) & ~uint64_t(15);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(32);
+    cfg.dynamicSmemBytes = S * T;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = g_pdl ? 1 : 0;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, k_copy_tma<S, T>, p);
+    if (e == cudaSuccess) e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+    ++*launches;
+  }
+  return cudaSuccess;
+}
+
+int g_stash_tma = [] {
+  const char *e = std::getenv("ES_STASH_TMA");
+  return e ? std::atoi(e) : 0;
+}();
+
 // ---- k_swap -----------------------------------------------------------------
 
 struct SwapParams {
@@ -713,6 +865,11 @@ cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *s
     return cudaSuccess;
   }
   const int n = (int)live.size();
+  if (sdt == ddt && g_stash_tma > 0 && !(swap && swap->n > 0)) {
+    const int es_ = sdt == ES_BF16 ? 2 : 4;
+    return g_stash_tma == 1 ? launch_copy_tma<4, 32768>(live.data(), n, es_, s, 1, launches)
+                            : launch_copy_tma<6, 16384>(live.data(), n, es_, s, 2, launches);
+  }
   if (sdt == ES_F32 && ddt == ES_F32) return launch_stash_t<F32T, F32T, 4>(live.data(), n, s, bo, to, launches, swap);
   if (sdt == ES_BF16 && ddt == ES_BF16)
     return launch_stash_t<BF16T, BF16T, 8>(live.data(), n, s, bo, to, launches, swap);
