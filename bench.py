@@ -46,6 +46,9 @@ def parse():
                    help="separate es_switch_context and es_stash_grads launches instead of es_stash_and_switch")
     p.add_argument("--incremental", action="store_true",
                    help="NEXT-1: fold each EST into running partials at its switch (es_stash_fold_grads, G == 1)")
+    p.add_argument("--inplace", action="store_true",
+                   help="NEXT-2 zero-copy stash: each EST's gradients are produced in its slot (es_slot_ptr) and "
+                        "stashed with ES_STASH_INPLACE")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     p.add_argument("--cpu-seconds", type=float, default=10.0)
@@ -238,16 +241,29 @@ def main():
     for k in local:
         for i, blob in enumerate(workloads.est_state(name, k)):
             agg.init_state(k, i, blob)
-    grads = {k: [workloads.est_bucket(name, k, b, device=dev) for b in range(B)] for k in local}
+    if args.inplace:       # the synthetic "backward" writes straight into the EST's slots
+        grads = {k: [workloads.est_bucket(name, k, b, device=dev, out=agg.slot(k, b)) for b in range(B)]
+                 for k in local}
+    else:
+        grads = {k: [workloads.est_bucket(name, k, b, device=dev) for b in range(B)] for k in local}
     outs = [agg.new_out(b) for b in range(B)]
     esz = 2 if cfg["dtype"] == "bf16" else 4
     in_bytes = len(local) * sum(n for n, _ in buckets) * esz
     flush = None if in_bytes > 2 * L2_BYTES else torch.empty(4 * L2_BYTES, dtype=torch.uint8, device=dev)
     torch.cuda.synchronize()
 
-    fuse = not (args.per_bucket or args.no_fuse or args.incremental)
+    fuse = not (args.per_bucket or args.no_fuse or args.incremental or args.inplace)
 
     def step():
+        if args.inplace:
+            agg.switch(local[0])
+            for i, k in enumerate(local):
+                if i == len(local) - 1:
+                    agg.stash_many(k, range(B), grads[k], es.ES_STASH_INPLACE)
+                else:
+                    agg.stash_and_switch(k, range(B), grads[k], local[i + 1], es.ES_STASH_INPLACE)
+            agg.allreduce_many(range(B), outs)
+            return
         if args.incremental:
             for i, k in enumerate(local):
                 agg.switch(k)
@@ -343,7 +359,8 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
 
-    kinds = {"stash": es.ES_KERNEL_STASH, "fold": es.ES_KERNEL_FOLD, "swap": es.ES_KERNEL_SWAP}
+    kinds = {"stash": es.ES_KERNEL_STASH, "fold": es.ES_KERNEL_FOLD, "swap": es.ES_KERNEL_SWAP,
+             "gather": es.ES_KERNEL_GATHER, "barrier": es.ES_KERNEL_BARRIER}
     prof = {k: agg.profile_query(v) for k, v in kinds.items()}   # (launches, ms, bytes)
     agg.profile(False)
     steps_profiled = 1 if graph is not None else args.steps
@@ -356,7 +373,8 @@ def main():
     per_launch = fl_bytes / max(fl_n, 1)
     traffic = None
     tfile = os.path.join(ROOT, "profiles", f"traffic_{name}_g{G}.json")
-    if os.path.exists(tfile) and not (args.incremental or args.per_bucket or args.no_fuse or args.no_graph):
+    if os.path.exists(tfile) and not (args.incremental or args.per_bucket or args.no_fuse or args.no_graph
+                                      or args.inplace):
         with open(tfile) as f:
             traffic = json.load(f).get("fold_dram_bytes_per_launch")
 
@@ -367,7 +385,8 @@ def main():
         "config": {"workload": name, "N": N, "G": G, "mapping": args.mapping, "sched": args.sched,
                    "buckets": B, "elements": sum(n for n, _ in buckets), "graph": graph is not None,
                    "api": "per-bucket" if args.per_bucket else ("incremental" if args.incremental else
-                                                               ("batched" if args.no_fuse else "batched+fused-switch")),
+                                                               ("zero-copy-inplace" if args.inplace else
+                                                                ("batched" if args.no_fuse else "batched+fused-switch"))),
                    "l2": ("inputs larger than L2 (%.1f MB of EST gradients per GPU per step)" % (in_bytes / 1e6))
                    if flush is None else "L2 flushed between timed steps (512 MB write)",
                    "desc": cfg["desc"]},
@@ -377,6 +396,9 @@ def main():
                      "launches_per_step": int(fl_n / steps_profiled),
                      "avg_launch_us": round(fl_ms / max(fl_n, 1) * 1e3, 2), "peak_source": peak_src},
         "breakdown_ms_per_step": {k: round(v[1] / steps_profiled, 4) for k, v in prof.items()},
+        "per_kernel": {k: {"launches_per_step": int(v[0] / steps_profiled),
+                           "algorithmic_GBps": round(v[2] / (v[1] / 1e3) / 1e9, 1) if v[1] > 0 else None,
+                           "us_per_launch": round(v[1] / max(v[0], 1) * 1e3, 2)} for k, v in prof.items()},
         # SURVEY 8(d)'s narrower metric: es_allreduce time only (stashes already done)
         "allreduce_only": {"ms": round(fl_ms / steps_profiled, 4),
                            "GBps": round(payload / (fl_ms / steps_profiled / 1e3) / 1e9, 1) if fl_ms > 0 else None},
