@@ -1,0 +1,331 @@
+// api_allreduce.cpp -- C ABI: es_allreduce(_many), the executor that walks the
+// planner's op list (plan.cpp) launching multi-segment folds and transport
+// groups, and the phase-merged ES_SCHED_PEER executor.
+#include <unistd.h>
+
+#include "handle.h"
+
+extern "C" {
+
+// ---- aggregation --------------------------------------------------------------------
+
+namespace {
+es_status finish_allreduce(es_handle h, int32_t n, const int32_t *buckets, cudaStream_t cs, unsigned long long cap);
+
+es_status peer_barrier(es_handle h, cudaStream_t cs) {
+  const es::Plan &p = h->plan;
+  std::vector<uint64_t *> pf(p.G);
+  for (int32_t g = 0; g < p.G; ++g) pf[g] = reinterpret_cast<uint64_t *>(h->peer_ws[g] + p.flags_off);
+  const uint64_t epoch = ++h->barrier_epoch;
+  return h->timed(ES_KERNEL_BARRIER, 0, cs, [&](int *nl) {
+    *nl = 1;
+    return es::launch_peer_barrier(pf.data(), reinterpret_cast<uint64_t *>(h->ws + p.flags_off), p.G, p.rank, epoch,
+                                   cs);
+  });
+}
+
+// ES_SCHED_PEER, phase-merged over the batch: [peer-visible copies of
+// borrowed buckets] -> barrier -> one fold launch (own shards, remote
+// contributions read from the owners' slots over NVLink) -> barrier -> one
+// gather launch per dtype (every shard from its owner's RESULT area).
+es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *const *outs, cudaStream_t cs, float r) {
+  const es::Plan &p = h->plan;
+  if (!h->peer_open) return set_err(ES_ESTATE, "ES_SCHED_PEER needs es_peer_open before es_allreduce");
+  es_status s;
+  const int32_t g = p.rank;
+  auto slot_of = [&](int32_t rank, int32_t e, int32_t b) {
+    return h->peer_ws[rank] + p.grad_off + (uint64_t)p.owner_index[e] * p.slot_block + p.slot_off[b];
+  };
+  // 1. borrowed contributions: peers read the ranges outside our shard from the slot
+  for (int dd = 0; dd < 2; ++dd) {
+    std::vector<es::StashSegDesc> segs;
+    uint64_t nbytes = 0;
+    for (int32_t i = 0; i < n; ++i) {
+      const es::BucketPlan &b = p.bp[buckets[i]];
+      if ((int)b.dtype != dd || b.L == 0) continue;
+      for (int32_t li = 0; li < h->n_local; ++li) {
+        const void *bw = h->borrowed[(size_t)li * h->B + buckets[i]];
+        if (!bw) continue;
+        unsigned char *slot = h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[buckets[i]];
+        const unsigned char *src = reinterpret_cast<const unsigned char *>(bw);
+        if (b.shard_lo > 0) segs.push_back({src, slot, b.shard_lo});
+        if ((uint64_t)b.shard_hi < b.L)
+          segs.push_back({src + (uint64_t)b.shard_hi * b.esize, slot + (uint64_t)b.shard_hi * b.esize,
+                          (int64_t)(b.L - (uint64_t)b.shard_hi)});
+        nbytes += 2 * (b.L - (uint64_t)(b.shard_hi - b.shard_lo)) * b.esize;
+      }
+    }
+    if (segs.empty()) continue;
+    s = h->timed(ES_KERNEL_STASH, nbytes, cs, [&](int *nl) {
+      return es::launch_stash_multi((es_dtype)dd, (es_dtype)dd, segs.data(), (int)segs.size(), cs, h->blocks_ov,
+                                    h->threads_ov, nl);
+    });
+    if (s != ES_OK) return s;
+  }
+  // 2. every rank's slots hold this step's contributions
+  if ((s = peer_barrier(h, cs)) != ES_OK) return s;
+  // 3. fold of the own shards
+  for (int dd = 0; dd < 2; ++dd) {
+    std::vector<es::FoldSegDesc> segs;
+    std::vector<std::vector<const void *>> srcs;
+    uint64_t nbytes = 0;
+    for (int32_t i = 0; i < n; ++i) {
+      const int32_t bk = buckets[i];
+      const es::BucketPlan &b = p.bp[bk];
+      if ((int)b.dtype != dd || b.shard_hi <= b.shard_lo) continue;
+      std::vector<const void *> src(p.N);
+      for (int32_t e = 0; e < p.N; ++e) {
+        const int32_t li = p.local_index[e];
+        const void *bw = li >= 0 ? h->borrowed[(size_t)li * h->B + bk] : nullptr;
+        const unsigned char *base = bw ? reinterpret_cast<const unsigned char *>(bw) : slot_of(p.est_to_gpu[e], e, bk);
+        src[e] = base + (uint64_t)b.shard_lo * b.esize;
+      }
+      es::FoldSegDesc d;
+      d.lo = b.shard_lo;
+      d.n = b.shard_hi - b.shard_lo;
+      d.C = (uint32_t)b.C;
+      d.rot = true;
+      d.out = h->ws + p.result_off + p.slot_off[bk] + (uint64_t)b.shard_lo * b.esize;
+      nbytes += (uint64_t)d.n * ((uint64_t)p.N + 1) * b.esize;
+      segs.push_back(d);
+      srcs.push_back(std::move(src));
+    }
+    if (segs.empty()) continue;
+    for (size_t i = 0; i < segs.size(); ++i) segs[i].src = srcs[i].data();
+    s = h->timed(ES_KERNEL_FOLD, nbytes, cs, [&](int *nl) {
+      return es::launch_fold_multi((es_dtype)dd, p.N, r, p.compat, segs.data(), (int)segs.size(), cs, h->blocks_ov,
+                                   h->threads_ov, nl);
+    });
+    if (s != ES_OK) return s;
+  }
+  // 4. every shard result is ready; every slot has been read
+  if ((s = peer_barrier(h, cs)) != ES_OK) return s;
+  // 5. gather every shard from its owner
+  for (int dd = 0; dd < 2; ++dd) {
+    std::vector<es::StashSegDesc> segs;
+    uint64_t nbytes = 0;
+    for (int32_t i = 0; i < n; ++i) {
+      const int32_t bk = buckets[i];
+      const es::BucketPlan &b = p.bp[bk];
+      if ((int)b.dtype != dd || b.L == 0) continue;
+      unsigned char *outp = reinterpret_cast<unsigned char *>(outs[i]);
+      const uint64_t S = es::chunk_elems(b.L, p.G, p.A);
+      for (int32_t o = 0; o < p.G; ++o) {
+        const uint64_t lo = std::min<uint64_t>(b.L, S * o), hi = std::min<uint64_t>(b.L, S * (o + 1));
+        if (hi <= lo) continue;
+        segs.push_back({h->peer_ws[o] + p.result_off + p.slot_off[bk] + lo * b.esize, outp + lo * b.esize,
+                        (int64_t)(hi - lo)});
+        nbytes += 2 * (hi - lo) * b.esize;
+      }
+    }
+    if (segs.empty()) continue;
+    s = h->timed(ES_KERNEL_GATHER, nbytes, cs, [&](int *nl) {
+      return es::launch_stash_multi((es_dtype)dd, (es_dtype)dd, segs.data(), (int)segs.size(), cs, h->blocks_ov,
+                                    h->threads_ov, nl);
+    });
+    if (s != ES_OK) return s;
+  }
+  (void)g;
+  return ES_OK;
+}
+}  // namespace
+
+es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void *const *outs, es_stream stream) {
+  es_status s = check_handle(h);
+  if (s != ES_OK) return s;
+  const es::Plan &p = h->plan;
+  if (n < 0 || (n > 0 && (!buckets || !outs))) return set_err(ES_EINVAL, "bad bucket/out arrays");
+  for (int32_t i = 0; i < n; ++i) {
+    const int32_t bk = buckets[i];
+    if (bk < 0 || bk >= h->B) return set_err(ES_EINVAL, "bucket out of range");
+    for (int32_t j = 0; j < i; ++j)
+      if (buckets[j] == bk) return set_err(ES_EINVAL, "bucket listed twice");
+    const es::BucketPlan &b = p.bp[bk];
+    if (b.L == 0) continue;
+    if (!outs[i] || !aligned16(outs[i])) return set_err(ES_EINVAL, "out must be a 16-byte aligned device pointer");
+    const unsigned char *o = reinterpret_cast<const unsigned char *>(outs[i]);
+    if (o < h->ws + h->ws_bytes && h->ws < o + b.L * b.esize) return set_err(ES_EINVAL, "out overlaps the workspace");
+    for (int32_t li = 0; li < h->n_local; ++li)
+      if (!h->stashed[(size_t)li * h->B + bk])
+        return set_err(ES_ESTATE, "es_allreduce before every local EST stashed this bucket");
+  }
+  for (int32_t i = 0; i < n; ++i) {
+    for (int32_t li = 0; li < h->n_local; ++li)
+      if (!h->stashed[(size_t)li * h->B + buckets[i]])
+        return set_err(ES_ESTATE, "es_allreduce before every local EST stashed this bucket");
+    if (h->inc_next[buckets[i]] != 0 && h->inc_next[buckets[i]] != p.N)
+      return set_err(ES_ESTATE, "incremental fold of this bucket is incomplete");
+  }
+  cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
+  const unsigned long long cap = capture_id(cs);
+  for (int32_t i = 0; i < n; ++i)
+    for (int32_t li = 0; li < h->n_local; ++li) {
+      const size_t k = (size_t)li * h->B + buckets[i];
+      if (h->stash_cap[k] == cap && cudaStreamWaitEvent(cs, h->stash_ev[k], 0) != cudaSuccess)
+        return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
+    }
+  if (h->last_ar && h->last_ar_cap == cap && cudaStreamWaitEvent(cs, h->last_ar, 0) != cudaSuccess)
+    return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
+
+  const float r = 1.0f / (float)p.N;   // R5: fl32(1/N), correctly rounded fp32 division
+
+  if (p.peer) {
+    if ((s = peer_allreduce(h, n, buckets, outs, cs, r)) != ES_OK) return s;
+    return finish_allreduce(h, n, buckets, cs, cap);
+  }
+
+  // Pending FOLD ops: consecutive folds (across buckets for G == 1, within a
+  // chain round for G > 1) are independent and go out as one multi-segment
+  // launch; a transport group flushes them first.
+  std::vector<es::FoldSegDesc> pend;
+  std::vector<std::vector<const void *>> pend_src;
+  es_dtype pend_dt = ES_F32;
+  uint64_t pend_bytes = 0;
+  auto flush = [&]() -> es_status {
+    if (pend.empty()) return ES_OK;
+    for (size_t i = 0; i < pend.size(); ++i) pend[i].src = pend_src[i].data();
+    es_status st = h->timed(ES_KERNEL_FOLD, pend_bytes, cs, [&](int *nl) {
+      return es::launch_fold_multi(pend_dt, p.N, r, p.compat, pend.data(), (int)pend.size(), cs, h->blocks_ov,
+                                   h->threads_ov, nl);
+    });
+    pend.clear();
+    pend_src.clear();
+    pend_bytes = 0;
+    return st;
+  };
+
+  for (int32_t i = 0; i < n; ++i) {
+    const int32_t bucket = buckets[i];
+    const es::BucketPlan &b = p.bp[bucket];
+    const uint32_t esz = b.esize;
+    auto src_base = [&](int32_t e) -> unsigned char * {   // element 0 of local EST e's contribution
+      const int32_t li = p.local_index[e];
+      const void *bw = h->borrowed[(size_t)li * h->B + bucket];
+      if (bw) return reinterpret_cast<unsigned char *>(const_cast<void *>(bw));
+      return h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[bucket];
+    };
+    auto contrib_at = [&](int32_t e, int64_t lo) -> unsigned char * {
+      if (p.local_index[e] >= 0) return src_base(e) + (uint64_t)lo * esz;
+      return h->ws + p.stage_off + (uint64_t)b.stage_index[e] * b.stage_stride + (uint64_t)(lo - b.shard_lo) * esz;
+    };
+    auto part_at = [&](int64_t id, int64_t lo) -> unsigned char * {
+      const es::Part &pt = b.parts[id];
+      return h->ws + p.parts_off + pt.off + (uint64_t)(lo - pt.lo) * 4;
+    };
+    unsigned char *outp = reinterpret_cast<unsigned char *>(outs[i]);
+    if (h->inc_next[bucket] == p.N && b.L > 0) {
+      // NEXT-1 end of step: chunk c < N-1 continues from its partial (ESTs
+      // c+1..N-1) over the stashed ESTs 0..c; chunk N-1 folds 0..N-1.
+      if (!pend.empty() && pend_dt != b.dtype && (s = flush()) != ES_OK) return s;
+      pend_dt = b.dtype;
+      const float *part = reinterpret_cast<const float *>(h->ws + p.inc_off + p.inc_bucket_off[bucket]);
+      for (int32_t c = 0; c < p.N; ++c) {
+        const int64_t lo = std::min<int64_t>((int64_t)b.L, (int64_t)c * (int64_t)b.C);
+        const int64_t hi = std::min<int64_t>((int64_t)b.L, (int64_t)(c + 1) * (int64_t)b.C);
+        if (hi <= lo) continue;
+        es::FoldSegDesc d;
+        d.lo = lo;
+        d.n = hi - lo;
+        d.C = (uint32_t)b.C;
+        d.rot = false;
+        const bool cont = c < p.N - 1;
+        d.m = cont ? c + 1 : p.N;
+        d.part_in = cont ? part + lo : nullptr;
+        d.out = outp + (uint64_t)lo * esz;
+        std::vector<const void *> src;
+        for (int32_t e = 0; e < d.m; ++e) src.push_back(src_base(e) + (uint64_t)lo * esz);
+        pend_bytes += (uint64_t)d.n * ((uint64_t)d.m * esz + (cont ? 4 : 0) + esz);
+        pend.push_back(d);
+        pend_src.push_back(std::move(src));
+      }
+      continue;
+    }
+    for (const es::Op &op : b.ops) {
+      const int64_t *f = op.f;
+      switch (f[0]) {
+        case ES_OP_FOLD: {
+          if (!pend.empty() && pend_dt != b.dtype && (s = flush()) != ES_OK) return s;
+          pend_dt = b.dtype;
+          const int64_t lo = f[1], hi = f[2];
+          es::FoldSegDesc d;
+          d.lo = lo;
+          d.n = hi - lo;
+          d.C = (uint32_t)b.C;
+          std::vector<const void *> src;
+          if (f[3] < 0) {
+            d.rot = true;
+            for (int32_t e = 0; e < p.N; ++e) src.push_back(contrib_at(e, lo));
+          } else {
+            d.rot = false;
+            d.m = (int32_t)f[4];
+            for (int32_t t = 0; t < d.m; ++t) src.push_back(contrib_at((int32_t)((f[3] + t) % p.N), lo));
+          }
+          d.part_in = f[5] == ES_BUF_PART ? reinterpret_cast<const float *>(part_at(f[6], lo)) : nullptr;
+          d.out_partial = f[7] == ES_BUF_PART;
+          d.out = d.out_partial ? (void *)part_at(f[8], lo) : (void *)(outp + (uint64_t)lo * esz);
+          pend_bytes += (uint64_t)d.n * ((uint64_t)src.size() * esz + (d.part_in ? 4 : 0) + (d.out_partial ? 4 : esz));
+          pend.push_back(d);
+          pend_src.push_back(std::move(src));
+          break;
+        }
+        case ES_OP_GROUP_BEGIN:
+          if ((s = flush()) != ES_OK) return s;
+          if ((s = h->tp->group_begin()) != ES_OK) return h->poison(s, h->tp->err);
+          break;
+        case ES_OP_GROUP_END:
+          if ((s = h->tp->group_end(cs)) != ES_OK) return h->poison(s, h->tp->err);
+          break;
+        case ES_OP_SEND:
+        case ES_OP_RECV: {
+          const int64_t lo = f[1], hi = f[2];
+          const int peer = (int)f[3];
+          unsigned char *ptr = nullptr;
+          uint64_t w = esz;
+          switch (f[4]) {
+            case ES_BUF_SRC:
+            case ES_BUF_STAGE: ptr = contrib_at((int32_t)f[5], lo); break;
+            case ES_BUF_PART: ptr = part_at(f[5], lo); w = 4; break;
+            case ES_BUF_OUT: ptr = outp + (uint64_t)lo * esz; break;
+            default: return h->poison(ES_ESTATE, "corrupt plan: bad buffer kind");
+          }
+          const size_t nbytes = (size_t)(hi - lo) * w;
+          s = f[0] == ES_OP_SEND ? h->tp->send(ptr, nbytes, peer) : h->tp->recv(ptr, nbytes, peer);
+          if (s != ES_OK) return h->poison(s, h->tp->err);
+          break;
+        }
+        default:
+          return h->poison(ES_ESTATE, "corrupt plan: bad opcode");
+      }
+    }
+  }
+  if ((s = flush()) != ES_OK) return s;
+  return finish_allreduce(h, n, buckets, cs, cap);
+}
+
+namespace {
+
+es_status finish_allreduce(es_handle h, int32_t n, const int32_t *buckets, cudaStream_t cs, unsigned long long cap) {
+  for (int32_t i = 0; i < n; ++i) {
+    const int32_t bucket = buckets[i];
+    if (cudaEventRecord(h->ar_ev[bucket], cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaEventRecord failed");
+    h->ar_recorded[bucket] = 1;
+    h->ar_cap[bucket] = cap;
+    h->last_ar = h->ar_ev[bucket];
+    h->last_ar_cap = cap;
+    for (int32_t li = 0; li < h->n_local; ++li) {
+      h->stashed[(size_t)li * h->B + bucket] = 0;
+      h->borrowed[(size_t)li * h->B + bucket] = nullptr;
+    }
+    h->inc_next[bucket] = 0;
+  }
+  return ES_OK;
+}
+
+}  // namespace
+
+es_status es_allreduce(es_handle h, int32_t bucket, void *out, es_stream stream) {
+  return es_allreduce_many(h, 1, &bucket, &out, stream);
+}
+
+
+}  // extern "C"
