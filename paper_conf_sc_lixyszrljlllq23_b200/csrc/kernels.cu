@@ -78,6 +78,10 @@ __device__ __forceinline__ void st_stream(uint2 *p, const uint2 &v) {
 }
 __device__ __forceinline__ void st_stream(int4 *p, const int4 &v) { st_stream(static_cast<void *>(p), v); }
 
+__device__ __forceinline__ uint32_t smem_addr(const void *p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
 template <typename K, typename P>
 cudaError_t launch(K kernel, dim3 grid, dim3 block, cudaStream_t s, const P &params) {
   cudaLaunchConfig_t cfg = {};
@@ -343,6 +347,100 @@ __global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams
   }
 }
 
+// ---- k_fold_tma: TMA / shared-memory staged fold (experiment) -------------------
+// The north star's "pulls the N EST contributions through TMA/shared-memory
+// staging": per tile of 256*V elements one elected thread issues N
+// cp.async.bulk copies (one per source row, completion on the stage's
+// mbarrier), all threads fold from shared memory in canonical order and
+// store.  S-stage ring, tiles prefetched S-1 ahead.  Canonical (rot)
+// segments without partials only, N <= 16.  Selected with ES_FOLD_TMA=1;
+// the LDG kernel above is the default (profiles/: it measured as fast).
+
+template <typename T, int MAXSEG, int MAXSRC, int S>
+__global__ void __launch_bounds__(256) k_fold_tma(const __grid_constant__ FoldParams<MAXSEG, MAXSRC> p) {
+  constexpr int V = T::kVec;
+  constexpr int TILE = 256 * V;                 // elements per tile
+  constexpr int TILEB = TILE * T::kSize;        // 4096 bytes per source row
+  extern __shared__ __align__(128) unsigned char ring[];
+  __shared__ __align__(8) uint64_t full[S];
+  pdl_enter();
+  const int si = find_seg(p.seg, p.nseg, (int)blockIdx.x);
+  const FoldSeg &g = p.seg[si];
+  const int nb = (si + 1 < p.nseg ? p.seg[si + 1].block0 : p.nblocks) - g.block0;
+  const int lb = (int)blockIdx.x - g.block0;
+  const void *const *src = p.src + g.src0;
+  const int N = p.N;
+  const int64_t ntiles = (g.n + TILE - 1) / TILE;
+  const int tid = threadIdx.x;
+  if (tid == 0) {
+    for (int st = 0; st < S; ++st)
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_addr(&full[st])) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  auto issue = [&](int64_t i) {                 // thread 0: tile number i of this block
+    const int64_t tile = lb + i * nb;
+    const int st = (int)(i % S);
+    const int64_t t0 = tile * TILE;
+    const int64_t cnt = min((int64_t)TILE, g.n - t0);
+    const uint32_t bytes = (uint32_t)((cnt * T::kSize) & ~int64_t(15));
+    const uint32_t bar = smem_addr(&full[st]);
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes * (uint32_t)N)
+                 : "memory");
+    if (bytes == 0) return;
+    for (int k = 0; k < N; ++k)
+      asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                   ::"r"(smem_addr(ring + ((size_t)st * N + k) * TILEB)),
+                   "l"(reinterpret_cast<const char *>(src[k]) + t0 * T::kSize), "r"(bytes), "r"(bar)
+                   : "memory");
+  };
+  int64_t mine = lb < ntiles ? (ntiles - lb + nb - 1) / nb : 0;
+  if (tid == 0)
+    for (int64_t i = 0; i < S - 1 && i < mine; ++i) issue(i);
+  for (int64_t i = 0; i < mine; ++i) {
+    if (tid == 0 && i + S - 1 < mine) issue(i + S - 1);
+    const int st = (int)(i % S);
+    const uint32_t bar = smem_addr(&full[st]);
+    const uint32_t parity = (uint32_t)((i / S) & 1);
+    uint32_t ok = 0;
+    do {
+      asm volatile("{\n .reg .pred q;\n mbarrier.try_wait.parity.shared::cta.b64 q, [%1], %2;\n selp.u32 %0, 1, 0, q;\n}"
+                   : "=r"(ok)
+                   : "r"(bar), "r"(parity)
+                   : "memory");
+    } while (!ok);
+    const int64_t t0 = (lb + i * nb) * TILE;
+    const int64_t cnt = min((int64_t)TILE, g.n - t0);
+    const int e0 = tid * V;
+    if (e0 + V <= cnt) {
+      const uint32_t c = (uint32_t)(g.lo + t0 + e0) / g.C;    // R1
+      int k = (int)(c + 1u == (uint32_t)N ? 0u : c + 1u);      // R2
+      float acc[V];
+      const unsigned char *row0 = ring + (size_t)st * N * TILEB + (size_t)e0 * T::kSize;
+      T::widen(*reinterpret_cast<const int4 *>(row0 + (size_t)k * TILEB), acc);   // R3
+      for (int j = 1; j < N; ++j) {
+        k = (k + 1 == N) ? 0 : k + 1;
+        float x[V];
+        T::widen(*reinterpret_cast<const int4 *>(row0 + (size_t)k * TILEB), x);
+#pragma unroll
+        for (int e = 0; e < V; ++e) acc[e] = __fadd_rn(acc[e], x[e]);
+      }
+#pragma unroll
+      for (int e = 0; e < V; ++e) acc[e] = __fmul_rn(acc[e], p.r);                  // R5
+      st_stream(reinterpret_cast<char *>(g.out) + (t0 + e0) * T::kSize, T::narrow(acc));
+    } else if (e0 < cnt) {                                      // ragged tail of the segment
+      for (int64_t t = t0 + e0; t < t0 + cnt; ++t)
+        T::store1(g.out, t, __fmul_rn(fold_scalar<T, false>(g, src, N, t, 0u, p.r), p.r));
+    }
+    __syncthreads();                                            // stage free for the refill
+  }
+}
+
+int g_fold_tma = [] {
+  const char *e = std::getenv("ES_FOLD_TMA");
+  return e ? std::atoi(e) : 0;
+}();
+
 template <typename T, int MAXSEG, int MAXSRC>
 cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSegDesc *d, int nseg, cudaStream_t s,
                               int bo, int to) {
@@ -378,6 +476,36 @@ cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSeg
   std::vector<int32_t> block0;
   split_blocks(work, total, &block0, &p.nblocks);
   for (int i = 0; i < nseg; ++i) p.seg[i].block0 = block0[i];
+  bool tma_ok = g_fold_tma > 0 && !compat && N <= 16 && bo == 0 && to == 0;
+  for (int i = 0; i < nseg && tma_ok; ++i) tma_ok = d[i].rot && !d[i].part_in && !d[i].out_partial;
+  if (tma_ok) {
+    constexpr int kS = 3;
+    const int stage = N * 256 * T::kVec * T::kSize;
+    static bool attr = false;
+    if (!attr) {
+      cudaFuncSetAttribute(k_fold_tma<T, MAXSEG, MAXSRC, kS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           kS * 16 * 4096);
+      attr = true;
+    }
+    const int per_sm = std::max(1, (227 * 1024) / (kS * stage + 1024));
+    int64_t tiles = 0;
+    for (int i = 0; i < nseg; ++i) tiles += (d[i].n + 256 * T::kVec - 1) / (256 * T::kVec);
+    const int grid = (int)std::max<int64_t>(nseg, std::min<int64_t>(tiles, (int64_t)kSMs * per_sm));
+    split_blocks(work, grid, &block0, &p.nblocks);
+    for (int i = 0; i < nseg; ++i) p.seg[i].block0 = block0[i];
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(p.nblocks);
+    cfg.blockDim = dim3(256);
+    cfg.dynamicSmemBytes = kS * stage;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = g_pdl ? 1 : 0;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, k_fold_tma<T, MAXSEG, MAXSRC, kS>, p);
+    return e != cudaSuccess ? e : cudaGetLastError();
+  }
   if (compat) return launch(k_fold<T, MAXSEG, MAXSRC, true>, dim3(p.nblocks), dim3(threads), s, p);
   return launch(k_fold<T, MAXSEG, MAXSRC, false>, dim3(p.nblocks), dim3(threads), s, p);
 }
@@ -589,10 +717,6 @@ struct CopyTmaParams {
   uint64_t per_cta;            // multiple of 16
   CopySeg seg[32];
 };
-
-__device__ __forceinline__ uint32_t smem_addr(const void *p) {
-  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
 
 template <int S, int T>
 __global__ void __launch_bounds__(32) k_copy_tma(const __grid_constant__ CopyTmaParams p) {
