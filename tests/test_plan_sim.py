@@ -103,3 +103,35 @@ def test_auto_picks_fewer_bytes():
     assert sched_of("swin_b", 4) == es.ES_SCHED_CHAIN
     assert sched_of("resnet50", 8) == es.ES_SCHED_DIRECT
     assert sched_of("bert_base", 8, "round_robin") == es.ES_SCHED_DIRECT
+
+
+def test_random_configs_property():
+    """Property test over random (N, G, mapping, ragged L, A, schedule): every
+    rank of the replayed plan holds the oracle's bits."""
+    from hypothesis import given, settings, HealthCheck
+    from hypothesis import strategies as st
+
+    @st.composite
+    def cfgs(draw):
+        N = draw(st.integers(1, 12))
+        G = draw(st.integers(1, min(N, 6)))
+        base = list(range(G)) + [draw(st.integers(0, G - 1)) for _ in range(N - G)]
+        perm = draw(st.permutations(base))
+        nb = draw(st.integers(1, 3))
+        Ls = [draw(st.integers(0, 700)) for _ in range(nb)]
+        dts = [draw(st.sampled_from(["f32", "bf16"])) for _ in range(nb)]
+        A = draw(st.sampled_from([8, 16, 32]))
+        sched = draw(st.sampled_from([es.ES_SCHED_AUTO, es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_PEER]))
+        seed = draw(st.integers(0, 2 ** 31))
+        return N, G, list(perm), Ls, dts, A, sched, seed
+
+    @settings(max_examples=150, deadline=None, suppress_health_check=list(HealthCheck))
+    @given(cfgs())
+    def run(c):
+        N, G, m, Ls, dts, A, sched, seed = c
+        xs = _data(N, [max(L, 1) for L in Ls], dts, seed)
+        xs = [[x[:L] for x in row] for row, L in zip(xs, Ls)]
+        want = [oracle.reduce(x, d, A=A) for x, d in zip(xs, dts)]
+        _check(N, G, m, Ls, dts, sched, A=A, xs=xs, want=want)
+
+    run()
