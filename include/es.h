@@ -208,10 +208,13 @@ es_status es_switch_context(es_handle h, int32_t est, es_stream stream);
 /* Stashes local EST `est`'s gradient for `bucket`.
  * grad: device pointer, 16-byte aligned, `numel` elements of grad_dtype.
  * COPY: one vectorised kernel copies/casts into the EST's slot (RNE when
- * narrowing fp32->bf16, exact when widening).  BORROW: grad_dtype must
- * equal the bucket dtype; the pointer is recorded.  Either way an event on
- * `stream` orders the stash before the bucket's next es_allreduce.
- * ES_ESTATE if `est` is not mapped to this rank. */
+ * narrowing fp32->bf16, exact when widening); the copy waits (on `stream`)
+ * for the bucket's previous es_allreduce, which may still read the slot.
+ * BORROW: grad_dtype must equal the bucket dtype; the pointer is recorded.
+ * INPLACE: grad must be es_slot_ptr(est, bucket); nothing is copied.  In
+ * every mode an event on `stream` orders the stash before the bucket's
+ * next es_allreduce.  ES_ESTATE if `est` is not mapped to this rank or the
+ * bucket is being folded incrementally this step. */
 es_status es_stash_grad(es_handle h, int32_t est, int32_t bucket, const void *grad,
                         es_dtype grad_dtype, es_stash_mode mode, es_stream stream);
 
@@ -378,10 +381,13 @@ typedef enum {
 } es_kernel_kind;
 
 /* When enabled, every kernel launch of this handle is bracketed by CUDA
- * events on its own stream.  es_profile_query synchronises on those events
- * and returns, per kind since the last reset: launches, summed device ms,
- * and algorithmic bytes (reads + writes the method needs, DESIGN.md
- * "Roofline").  Launch counts are kept even when timing is off. */
+ * events on its own stream (event-record nodes when the stream is being
+ * captured into a CUDA graph).  es_profile_query synchronises on those
+ * events and returns, per kind since the last reset: launches, summed device
+ * ms, and algorithmic bytes (reads + writes the method needs, DESIGN.md
+ * "Kernels and their rooflines").  For captured launches the ms are those of
+ * the graph's most recent replay and launches/bytes count the capture once.
+ * Launch counts are kept even when timing is off. */
 es_status es_profile_enable(es_handle h, int32_t on);
 es_status es_profile_reset(es_handle h);
 es_status es_profile_query(es_handle h, es_kernel_kind kind, uint64_t *launches, double *ms,
