@@ -38,7 +38,7 @@ def parse():
     p.add_argument("--config", default="resnet50",
                    choices=["tiny", "resnet50", "vgg19", "bert_base", "swin_b"])
     p.add_argument("--mapping", default="contiguous", choices=["contiguous", "round_robin", "random"])
-    p.add_argument("--sched", default="auto", choices=["auto", "direct", "chain", "peer"])
+    p.add_argument("--sched", default="auto", choices=["auto", "direct", "chain", "peer", "peer_chain", "peer_auto"])
     p.add_argument("--no-graph", action="store_true", help="eager launches instead of one CUDA graph per step")
     p.add_argument("--per-bucket", action="store_true",
                    help="one es_stash_grad / es_allreduce call per bucket (DDP-style) instead of the batched calls")
@@ -229,12 +229,12 @@ def main():
     buckets = cfg["buckets"]
     B = len(buckets)
     sched = {"auto": es.ES_SCHED_AUTO, "direct": es.ES_SCHED_DIRECT, "chain": es.ES_SCHED_CHAIN,
-             "peer": es.ES_SCHED_PEER}[args.sched]
+             "peer": es.ES_SCHED_PEER, "peer_chain": es.ES_SCHED_PEER_CHAIN, "peer_auto": es.ES_SCHED_PEER_AUTO}[args.sched]
     snb = workloads.state_nbytes()
     agg = Aggregator(N, G, rank, mapping, buckets, state_nbytes=snb,
                      transport=es.ES_TRANSPORT_NONE if G == 1 else es.ES_TRANSPORT_NCCL, comm=comm, sched=sched,
                      device=dev, options=es.ES_OPT_INCREMENTAL if args.incremental else 0)
-    if G > 1 and sched == es.ES_SCHED_PEER:
+    if G > 1 and sched in es.PEER_SCHEDS:
         agg.peer_connect()                       # CUDA IPC map of every peer's workspace (NVLink)
     live = [torch.zeros(n, dtype=torch.uint8, device=dev) for n in snb]
     agg.register_state(live)

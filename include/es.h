@@ -96,7 +96,18 @@ typedef enum { ES_STASH_COPY = 0, ES_STASH_BORROW = 1, ES_STASH_INPLACE = 2 } es
  *           peer memory) order the phases.  No staging copy, no NCCL protocol.
  *           Opt-in (never chosen by AUTO); BORROWed buckets are made
  *           peer-visible by copying the parts peers read into the slot. */
-typedef enum { ES_SCHED_AUTO = 0, ES_SCHED_DIRECT = 1, ES_SCHED_CHAIN = 2, ES_SCHED_PEER = 3 } es_sched;
+/*   PEER_CHAIN: the CHAIN schedule without a transport: the GPU of segment r
+ *           of chunk c reads the incoming unrounded fp32 partial directly from
+ *           the producer's workspace over NVLink inside its fold kernel (the
+ *           partial's transfer and the local fold are one kernel); a device
+ *           barrier separates rounds; chunk c is gathered from the RESULT area
+ *           of the GPU of EST c.
+ *   PEER_AUTO: per bucket PEER_CHAIN where CHAIN would move fewer bytes,
+ *           else PEER (the AUTO rule over the peer-memory schedules). */
+typedef enum {
+  ES_SCHED_AUTO = 0, ES_SCHED_DIRECT = 1, ES_SCHED_CHAIN = 2, ES_SCHED_PEER = 3, ES_SCHED_PEER_CHAIN = 4,
+  ES_SCHED_PEER_AUTO = 5
+} es_sched;
 
 /* How ranks exchange bytes when G > 1.
  *   NONE:     G == 1, or G > 1 with sched PEER (no transport library needed).
@@ -346,9 +357,12 @@ uint64_t es_chunk_elems(uint64_t L, int32_t N, uint32_t A);
 #define ES_OP_FIELDS 10
 enum {
   ES_OP_FOLD = 1,        /* [1]=lo [2]=hi [3]=e0 (-1: per-element rotation (c+1)%N) [4]=m (#ESTs)
-                            [5]=in_kind (0 none / ES_BUF_PART) [6]=in_id
+                            [5]=in_kind (0 none / ES_BUF_PART / ES_BUF_PEER_PART) [6]=in_id
+                                (PEER_PART: the producer rank)
                             [7]=out_kind (ES_BUF_PART: unscaled fp32 partial /
-                                          ES_BUF_OUT: scaled, rounded) [8]=out_id              */
+                                          ES_BUF_OUT / ES_BUF_RESULT: scaled, rounded) [8]=out_id
+                                (PEER_CHAIN: byte offset of the own partial)
+                            [9]=PEER_PART: byte offset in the producer's partials area       */
   ES_OP_SEND = 2,        /* [1]=lo [2]=hi [3]=peer [4]=buf_kind [5]=buf_id                      */
   ES_OP_RECV = 3,        /* same fields as SEND                                                 */
   ES_OP_GROUP_BEGIN = 4,
@@ -362,7 +376,8 @@ enum {
   ES_BUF_STAGE = 2,      /* staging for remote EST buf_id's contribution, bucket dtype         */
   ES_BUF_PART = 3,       /* fp32 partial buffer buf_id                                         */
   ES_BUF_OUT = 4,        /* the caller's output, bucket dtype                                  */
-  ES_BUF_RESULT = 5      /* PEER: this rank's shard result area in its workspace, bucket dtype */
+  ES_BUF_RESULT = 5,     /* PEER: this rank's shard result area in its workspace, bucket dtype */
+  ES_BUF_PEER_PART = 6   /* PEER_CHAIN: another rank's fp32 partial, read over NVLink          */
 };
 /* All [lo, hi) ranges are in bucket element coordinates. */
 es_status es_plan_ops(const es_config *cfg, int32_t bucket, int64_t *ops, size_t cap_ops,

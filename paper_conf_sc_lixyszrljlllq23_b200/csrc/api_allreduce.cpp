@@ -24,25 +24,26 @@ es_status peer_barrier(es_handle h, cudaStream_t cs) {
   });
 }
 
-// ES_SCHED_PEER, phase-merged over the batch: [peer-visible copies of
-// borrowed buckets] -> barrier -> one fold launch (own shards, remote
-// contributions read from the owners' slots over NVLink) -> barrier -> one
-// gather launch per dtype (every shard from its owner's RESULT area).
+// Peer-memory schedules (PEER, PEER_CHAIN), phase-merged over the batch.
+// Every bucket's op list is cut at its BARRIER ops into phases; phase k of
+// all buckets runs as one fold launch and one gather launch per dtype, then
+// one device barrier.  All ranks plan the same barrier count per bucket, so
+// the merged sequence of barriers matches across ranks.
 es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *const *outs, cudaStream_t cs, float r) {
   const es::Plan &p = h->plan;
-  if (!h->peer_open) return set_err(ES_ESTATE, "ES_SCHED_PEER needs es_peer_open before es_allreduce");
+  if (!h->peer_open) return set_err(ES_ESTATE, "peer-memory schedules need es_peer_open before es_allreduce");
   es_status s;
-  const int32_t g = p.rank;
   auto slot_of = [&](int32_t rank, int32_t e, int32_t b) {
     return h->peer_ws[rank] + p.grad_off + (uint64_t)p.owner_index[e] * p.slot_block + p.slot_off[b];
   };
-  // 1. borrowed contributions: peers read the ranges outside our shard from the slot
+  // 1. PEER buckets: peers read the ranges of BORROWed contributions outside
+  //    our shard from the slot (PEER_CHAIN reads only local contributions).
   for (int dd = 0; dd < 2; ++dd) {
     std::vector<es::StashSegDesc> segs;
     uint64_t nbytes = 0;
     for (int32_t i = 0; i < n; ++i) {
       const es::BucketPlan &b = p.bp[buckets[i]];
-      if ((int)b.dtype != dd || b.L == 0) continue;
+      if ((int)b.dtype != dd || b.L == 0 || b.sched != ES_SCHED_PEER) continue;
       for (int32_t li = 0; li < h->n_local; ++li) {
         const void *bw = h->borrowed[(size_t)li * h->B + buckets[i]];
         if (!bw) continue;
@@ -62,70 +63,89 @@ es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *c
     });
     if (s != ES_OK) return s;
   }
-  // 2. every rank's slots hold this step's contributions
-  if ((s = peer_barrier(h, cs)) != ES_OK) return s;
-  // 3. fold of the own shards
-  for (int dd = 0; dd < 2; ++dd) {
-    std::vector<es::FoldSegDesc> segs;
-    std::vector<std::vector<const void *>> srcs;
-    uint64_t nbytes = 0;
-    for (int32_t i = 0; i < n; ++i) {
-      const int32_t bk = buckets[i];
-      const es::BucketPlan &b = p.bp[bk];
-      if ((int)b.dtype != dd || b.shard_hi <= b.shard_lo) continue;
-      std::vector<const void *> src(p.N);
-      for (int32_t e = 0; e < p.N; ++e) {
-        const int32_t li = p.local_index[e];
-        const void *bw = li >= 0 ? h->borrowed[(size_t)li * h->B + bk] : nullptr;
-        const unsigned char *base = bw ? reinterpret_cast<const unsigned char *>(bw) : slot_of(p.est_to_gpu[e], e, bk);
-        src[e] = base + (uint64_t)b.shard_lo * b.esize;
-      }
-      es::FoldSegDesc d;
-      d.lo = b.shard_lo;
-      d.n = b.shard_hi - b.shard_lo;
-      d.C = (uint32_t)b.C;
-      d.rot = true;
-      d.out = h->ws + p.result_off + p.slot_off[bk] + (uint64_t)b.shard_lo * b.esize;
-      nbytes += (uint64_t)d.n * ((uint64_t)p.N + 1) * b.esize;
-      segs.push_back(d);
-      srcs.push_back(std::move(src));
-    }
-    if (segs.empty()) continue;
-    for (size_t i = 0; i < segs.size(); ++i) segs[i].src = srcs[i].data();
-    s = h->timed(ES_KERNEL_FOLD, nbytes, cs, [&](int *nl) {
-      return es::launch_fold_multi((es_dtype)dd, p.N, r, p.compat, segs.data(), (int)segs.size(), cs, h->blocks_ov,
-                                   h->threads_ov, nl);
-    });
-    if (s != ES_OK) return s;
+  // 2. phases
+  int32_t phases = 0;
+  for (int32_t i = 0; i < n; ++i) {
+    int32_t k = 0;
+    for (const es::Op &op : p.bp[buckets[i]].ops) k += op.f[0] == ES_OP_BARRIER;
+    phases = std::max(phases, k + 1);
   }
-  // 4. every shard result is ready; every slot has been read
-  if ((s = peer_barrier(h, cs)) != ES_OK) return s;
-  // 5. gather every shard from its owner
-  for (int dd = 0; dd < 2; ++dd) {
-    std::vector<es::StashSegDesc> segs;
-    uint64_t nbytes = 0;
-    for (int32_t i = 0; i < n; ++i) {
-      const int32_t bk = buckets[i];
-      const es::BucketPlan &b = p.bp[bk];
-      if ((int)b.dtype != dd || b.L == 0) continue;
-      unsigned char *outp = reinterpret_cast<unsigned char *>(outs[i]);
-      const uint64_t S = es::chunk_elems(b.L, p.G, p.A);
-      for (int32_t o = 0; o < p.G; ++o) {
-        const uint64_t lo = std::min<uint64_t>(b.L, S * o), hi = std::min<uint64_t>(b.L, S * (o + 1));
-        if (hi <= lo) continue;
-        segs.push_back({h->peer_ws[o] + p.result_off + p.slot_off[bk] + lo * b.esize, outp + lo * b.esize,
-                        (int64_t)(hi - lo)});
-        nbytes += 2 * (hi - lo) * b.esize;
+  for (int32_t ph = 0; ph < phases; ++ph) {
+    for (int dd = 0; dd < 2; ++dd) {
+      std::vector<es::FoldSegDesc> folds;
+      std::vector<std::vector<const void *>> srcs;
+      std::vector<es::StashSegDesc> gathers;
+      uint64_t fbytes = 0, gbytes = 0;
+      for (int32_t i = 0; i < n; ++i) {
+        const int32_t bk = buckets[i];
+        const es::BucketPlan &b = p.bp[bk];
+        if ((int)b.dtype != dd) continue;
+        const uint32_t esz = b.esize;
+        int32_t k = 0;
+        for (const es::Op &op : b.ops) {
+          const int64_t *f = op.f;
+          if (f[0] == ES_OP_BARRIER) {
+            ++k;
+            continue;
+          }
+          if (k != ph) continue;
+          const int64_t lo = f[1], hi = f[2];
+          if (f[0] == ES_OP_GATHER) {
+            gathers.push_back({h->peer_ws[f[3]] + p.result_off + p.slot_off[bk] + (uint64_t)lo * esz,
+                               reinterpret_cast<unsigned char *>(outs[i]) + (uint64_t)lo * esz, hi - lo});
+            gbytes += 2 * (uint64_t)(hi - lo) * esz;
+            continue;
+          }
+          // ES_OP_FOLD
+          es::FoldSegDesc d;
+          d.lo = lo;
+          d.n = hi - lo;
+          d.C = (uint32_t)b.C;
+          std::vector<const void *> src;
+          auto contrib = [&](int32_t e) -> const unsigned char * {
+            const int32_t li = p.local_index[e];
+            const void *bw = li >= 0 ? h->borrowed[(size_t)li * h->B + bk] : nullptr;
+            const unsigned char *base = bw ? reinterpret_cast<const unsigned char *>(bw)
+                                           : slot_of(p.est_to_gpu[e], e, bk);   // local or peer slot
+            return base + (uint64_t)lo * esz;
+          };
+          if (f[3] < 0) {
+            d.rot = true;
+            for (int32_t e = 0; e < p.N; ++e) src.push_back(contrib(e));
+          } else {
+            d.rot = false;
+            d.m = (int32_t)f[4];
+            for (int32_t t = 0; t < d.m; ++t) src.push_back(contrib((int32_t)((f[3] + t) % p.N)));
+          }
+          if (f[5] == ES_BUF_PEER_PART)         // the previous GPU's partial, over NVLink
+            d.part_in = reinterpret_cast<const float *>(h->peer_ws[f[6]] + p.peer_parts_off + b.peer_part_base +
+                                                        (uint64_t)f[9]);
+          d.out_partial = f[7] == ES_BUF_PART;
+          d.out = d.out_partial ? (void *)(h->ws + p.peer_parts_off + b.peer_part_base + (uint64_t)f[8])
+                                : (void *)(h->ws + p.result_off + p.slot_off[bk] + (uint64_t)lo * esz);
+          fbytes += (uint64_t)d.n * ((uint64_t)src.size() * esz + (d.part_in ? 4 : 0) + (d.out_partial ? 4 : esz));
+          folds.push_back(d);
+          srcs.push_back(std::move(src));
+        }
+      }
+      if (!folds.empty()) {
+        for (size_t j = 0; j < folds.size(); ++j) folds[j].src = srcs[j].data();
+        s = h->timed(ES_KERNEL_FOLD, fbytes, cs, [&](int *nl) {
+          return es::launch_fold_multi((es_dtype)dd, p.N, r, p.compat, folds.data(), (int)folds.size(), cs,
+                                       h->blocks_ov, h->threads_ov, nl);
+        });
+        if (s != ES_OK) return s;
+      }
+      if (!gathers.empty()) {
+        s = h->timed(ES_KERNEL_GATHER, gbytes, cs, [&](int *nl) {
+          return es::launch_stash_multi((es_dtype)dd, (es_dtype)dd, gathers.data(), (int)gathers.size(), cs,
+                                        h->blocks_ov, h->threads_ov, nl);
+        });
+        if (s != ES_OK) return s;
       }
     }
-    if (segs.empty()) continue;
-    s = h->timed(ES_KERNEL_GATHER, nbytes, cs, [&](int *nl) {
-      return es::launch_stash_multi((es_dtype)dd, (es_dtype)dd, segs.data(), (int)segs.size(), cs, h->blocks_ov,
-                                    h->threads_ov, nl);
-    });
-    if (s != ES_OK) return s;
+    if (ph + 1 < phases && (s = peer_barrier(h, cs)) != ES_OK) return s;
   }
-  (void)g;
   return ES_OK;
 }
 }  // namespace

@@ -241,6 +241,83 @@ void plan_chain(const Plan &p, BucketPlan *b) {
   b->ops.push_back(make_op(ES_OP_GROUP_END));
 }
 
+// ---- PEER_CHAIN ----------------------------------------------------------------
+// The CHAIN schedule without a transport: the GPU of segment r of chunk c
+// reads the incoming unrounded fp32 partial directly out of the producer's
+// workspace over NVLink (part_in = a peer pointer) inside its fold kernel, so
+// the partial's transfer and the local fold are one kernel.  A device barrier
+// separates rounds; chunk c ends in the RESULT area of the GPU of EST c and
+// is gathered from there.
+
+struct ChainShape {
+  std::vector<std::vector<Seg>> segs;
+  std::vector<Range> rng;
+  int32_t R = 0;
+};
+
+ChainShape chain_shape(const Plan &p, const BucketPlan &b) {
+  ChainShape sh;
+  sh.segs.resize(p.N);
+  sh.rng.resize(p.N);
+  for (int32_t c = 0; c < p.N; ++c) {
+    sh.rng[c] = chunk_range(b.L, b.C, c);
+    if (sh.rng[c].hi <= sh.rng[c].lo) continue;
+    chunk_segments(p, c, &sh.segs[c]);
+    sh.R = std::max<int32_t>(sh.R, (int32_t)sh.segs[c].size());
+  }
+  return sh;
+}
+
+// Byte offsets (inside the uniform peer partials area) of rank h's outgoing
+// partials, off[c][r] (-1: none), allocated in (round, chunk) order; returns
+// the bytes rank h needs.
+uint64_t chain_out_parts(const ChainShape &sh, int32_t h, std::vector<std::vector<int64_t>> *off) {
+  const int32_t N = (int32_t)sh.segs.size();
+  off->assign(N, {});
+  for (int32_t c = 0; c < N; ++c) (*off)[c].assign(sh.segs[c].size(), -1);
+  uint64_t o = 0;
+  for (int32_t r = 0; r < sh.R; ++r)
+    for (int32_t c = 0; c < N; ++c) {
+      const int32_t m = (int32_t)sh.segs[c].size();
+      if (r >= m - 1 || sh.segs[c][r].gpu != h) continue;
+      (*off)[c][r] = (int64_t)o;
+      o += align256((uint64_t)(sh.rng[c].hi - sh.rng[c].lo) * 4);
+    }
+  return o;
+}
+
+void plan_peer_chain(const Plan &p, BucketPlan *b) {
+  const int32_t g = p.rank;
+  b->sched = ES_SCHED_PEER_CHAIN;
+  if (b->L == 0) return;
+  const ChainShape sh = chain_shape(p, *b);
+  std::vector<std::vector<std::vector<int64_t>>> offs(p.G);
+  for (int32_t h = 0; h < p.G; ++h) b->peer_part_bytes = std::max(b->peer_part_bytes, chain_out_parts(sh, h, &offs[h]));
+  b->part_bytes = 0;
+  b->ops.push_back(make_op(ES_OP_BARRIER, 0));
+  for (int32_t r = 0; r < sh.R; ++r) {
+    for (int32_t c = 0; c < p.N; ++c) {
+      const int32_t m = (int32_t)sh.segs[c].size();
+      if (r >= m || sh.segs[c][r].gpu != g) continue;
+      const Seg &s = sh.segs[c][r];
+      Op o = make_op(ES_OP_FOLD, sh.rng[c].lo, sh.rng[c].hi, s.e0, s.m, ES_BUF_NONE, 0,
+                     r == m - 1 ? ES_BUF_RESULT : ES_BUF_PART, 0);
+      if (r > 0) {                       // incoming partial: the producer's buffer, over NVLink
+        const int32_t prod = sh.segs[c][r - 1].gpu;
+        o.f[5] = ES_BUF_PEER_PART;
+        o.f[6] = prod;
+        o.f[9] = offs[prod][c][r - 1];
+      }
+      if (r < m - 1) o.f[8] = offs[g][c][r];   // own outgoing partial (byte offset)
+      b->ops.push_back(o);
+    }
+    b->ops.push_back(make_op(ES_OP_BARRIER, r + 1));
+  }
+  for (int32_t c = 0; c < p.N; ++c)
+    if (sh.rng[c].hi > sh.rng[c].lo)
+      b->ops.push_back(make_op(ES_OP_GATHER, sh.rng[c].lo, sh.rng[c].hi, p.est_to_gpu[c]));
+}
+
 bool fail(std::string *err, const char *msg) {
   if (err) *err = msg;
   return false;
@@ -276,7 +353,7 @@ bool validate(const es_config *cfg, std::string *err, bool need_comm) {
     if (cfg->state_nbytes[i] == 0 || cfg->state_nbytes[i] > (1ull << 31))
       return fail(err, "state_nbytes must be in [1, 2^31]");
   if (cfg->sched != ES_SCHED_AUTO && cfg->sched != ES_SCHED_DIRECT && cfg->sched != ES_SCHED_CHAIN &&
-      cfg->sched != ES_SCHED_PEER)
+      cfg->sched != ES_SCHED_PEER && cfg->sched != ES_SCHED_PEER_CHAIN && cfg->sched != ES_SCHED_PEER_AUTO)
     return fail(err, "bad sched");
   if (cfg->compat & ~(uint32_t)(ES_COMPAT_PREDIV | ES_COMPAT_PREMUL | ES_COMPAT_BF16_HOP))
     return fail(err, "unknown compat bits");
@@ -284,7 +361,9 @@ bool validate(const es_config *cfg, std::string *err, bool need_comm) {
     return fail(err, "compat PREDIV and PREMUL are exclusive");
   if (cfg->options & ~(uint32_t)ES_OPT_INCREMENTAL) return fail(err, "unknown option bits");
   if ((cfg->options & ES_OPT_INCREMENTAL) && cfg->G != 1) return fail(err, "ES_OPT_INCREMENTAL needs G == 1");
-  if (cfg->G > 1 && need_comm && cfg->sched != ES_SCHED_PEER) {
+  const bool peer_sched = cfg->sched == ES_SCHED_PEER || cfg->sched == ES_SCHED_PEER_CHAIN ||
+                          cfg->sched == ES_SCHED_PEER_AUTO;
+  if (cfg->G > 1 && need_comm && !peer_sched) {
     if (cfg->transport != ES_TRANSPORT_NCCL && cfg->transport != ES_TRANSPORT_LOOPBACK)
       return fail(err, "G > 1 needs transport NCCL or LOOPBACK");
     if (!cfg->comm) return fail(err, "G > 1 needs comm");
@@ -320,7 +399,7 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
   p->options = cfg->options;
 
   p->bp.resize(cfg->n_buckets);
-  uint64_t max_stage = 0, max_parts = 0;
+  uint64_t max_stage = 0, max_parts = 0, sum_peer_parts = 0;
   for (int32_t bi = 0; bi < cfg->n_buckets; ++bi) {
     BucketPlan &b = p->bp[bi];
     b.L = p->buckets[bi].numel;
@@ -331,20 +410,25 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
       plan_single(*p, &b);
     } else {
       es_sched s = p->sched_req;
-      if (s == ES_SCHED_AUTO) {
+      if (s == ES_SCHED_AUTO || s == ES_SCHED_PEER_AUTO) {
         uint64_t d = 0, ch = 0;
         for (int32_t g = 0; g < p->G; ++g) {
           d = std::max(d, direct_recv_bytes(*p, b, g));
           ch = std::max(ch, chain_recv_bytes(*p, b, g));
         }
-        s = ch < d ? ES_SCHED_CHAIN : ES_SCHED_DIRECT;
+        const bool chain = ch < d;
+        if (s == ES_SCHED_AUTO) s = chain ? ES_SCHED_CHAIN : ES_SCHED_DIRECT;
+        else s = chain ? ES_SCHED_PEER_CHAIN : ES_SCHED_PEER;
       }
       if (s == ES_SCHED_CHAIN) plan_chain(*p, &b);
       else if (s == ES_SCHED_PEER) plan_peer(*p, &b);
+      else if (s == ES_SCHED_PEER_CHAIN) plan_peer_chain(*p, &b);
       else plan_direct(*p, &b);
     }
     max_stage = std::max(max_stage, b.stage_bytes);
     max_parts = std::max(max_parts, b.part_bytes);
+    b.peer_part_base = sum_peer_parts;   // buckets of one batched call run their rounds together
+    sum_peer_parts += align256(b.peer_part_bytes);
   }
 
   // Workspace layout.
@@ -358,12 +442,15 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
   // PEER: the regions peers address (flags, shard results, gradient slots)
   // come first, at offsets that depend only on the layout -- identical on
   // every rank whatever its number of local ESTs.
-  p->peer = p->G > 1 && p->sched_req == ES_SCHED_PEER;
+  p->peer = p->G > 1 && (p->sched_req == ES_SCHED_PEER || p->sched_req == ES_SCHED_PEER_CHAIN ||
+                          p->sched_req == ES_SCHED_PEER_AUTO);
   uint64_t head = 0;
   if (p->peer) {
     p->flags_off = 0;
     p->result_off = align256(64 * 8);
     head = p->result_off + p->slot_block;   // one bucket-layout block: shard results at bucket offsets
+    p->peer_parts_off = head;               // PEER_CHAIN partials: per bucket, max over ranks
+    head += align256(sum_peer_parts);
   }
   p->grad_off = head;
   uint64_t total = head + p->slot_block * p->local_ests.size();

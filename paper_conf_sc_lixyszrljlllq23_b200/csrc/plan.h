@@ -39,6 +39,8 @@ struct BucketPlan {
   uint64_t stage_bytes = 0;
   std::vector<Part> parts;
   uint64_t part_bytes = 0;
+  uint64_t peer_part_bytes = 0;         // PEER_CHAIN: max over ranks of their outgoing partials
+  uint64_t peer_part_base = 0;          // PEER_CHAIN: this bucket's base in the peer partials area
   std::vector<Op> ops;
 };
 
@@ -72,6 +74,7 @@ struct Plan {
   uint64_t parts_off = 0;               // chain partials (max over buckets)
   uint64_t flags_off = 0;               // PEER: G barrier flags (u64) written by peers
   uint64_t result_off = 0;              // PEER: per-bucket shard results (slot-block layout)
+  uint64_t peer_parts_off = 0;          // PEER_CHAIN: partials read by the next GPU (uniform offset)
   bool peer = false;                    // some bucket uses ES_SCHED_PEER
   std::vector<int32_t> owner_index;     // [N]: EST's index among its owner's local ESTs
   uint64_t total = 0;

@@ -16,12 +16,13 @@ from . import _build
 ES_OK, ES_EINVAL, ES_ESTATE, ES_ENOMEM, ES_ECUDA, ES_ENCCL, ES_EUNSUPPORTED = range(7)
 ES_F32, ES_BF16 = 0, 1
 ES_STASH_COPY, ES_STASH_BORROW, ES_STASH_INPLACE = 0, 1, 2
-ES_SCHED_AUTO, ES_SCHED_DIRECT, ES_SCHED_CHAIN, ES_SCHED_PEER = 0, 1, 2, 3
+ES_SCHED_AUTO, ES_SCHED_DIRECT, ES_SCHED_CHAIN, ES_SCHED_PEER, ES_SCHED_PEER_CHAIN, ES_SCHED_PEER_AUTO = range(6)
+PEER_SCHEDS = (ES_SCHED_PEER, ES_SCHED_PEER_CHAIN, ES_SCHED_PEER_AUTO)
 ES_TRANSPORT_NONE, ES_TRANSPORT_NCCL, ES_TRANSPORT_LOOPBACK = 0, 1, 2
 ES_KERNEL_STASH, ES_KERNEL_FOLD, ES_KERNEL_SWAP, ES_KERNEL_DROPOUT, ES_KERNEL_GATHER, ES_KERNEL_BARRIER = range(6)
 ES_OP_FIELDS = 10
 ES_OP_FOLD, ES_OP_SEND, ES_OP_RECV, ES_OP_GROUP_BEGIN, ES_OP_GROUP_END, ES_OP_BARRIER, ES_OP_GATHER = range(1, 8)
-ES_BUF_NONE, ES_BUF_SRC, ES_BUF_STAGE, ES_BUF_PART, ES_BUF_OUT, ES_BUF_RESULT = range(6)
+ES_BUF_NONE, ES_BUF_SRC, ES_BUF_STAGE, ES_BUF_PART, ES_BUF_OUT, ES_BUF_RESULT, ES_BUF_PEER_PART = range(7)
 ES_PEER_BLOB_BYTES = 128
 ES_COMPAT_PREDIV, ES_COMPAT_PREMUL, ES_COMPAT_BF16_HOP = 1, 2, 4
 ES_OPT_INCREMENTAL = 1

@@ -72,7 +72,7 @@ def multi(rng, sched):
     world = es.es_loopback_create(G)
     aggs = [Aggregator(N, G, g, m, list(zip(Ls, dts)), transport=es.ES_TRANSPORT_LOOPBACK, comm=world.value,
                        sched=sched) for g in range(G)]
-    if sched == es.ES_SCHED_PEER:
+    if sched in es.PEER_SCHEDS:
         blobs = [a.peer_blob() for a in aggs]
         for a in aggs:
             a.peer_open(blobs)
@@ -109,6 +109,6 @@ def multi(rng, sched):
 if __name__ == "__main__":
     rng = np.random.default_rng(0)
     g1(rng)
-    for sched in (es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_PEER):
+    for sched in (es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_PEER, es.ES_SCHED_PEER_CHAIN):
         multi(rng, sched)
     print("sanitize_step ok")

@@ -105,7 +105,7 @@ def reduce_loopback(xs_per_bucket, G, mapping, sched=es.ES_SCHED_AUTO, A=16, bor
     world = es.es_loopback_create(G)
     aggs = [Aggregator(N, G, g, mapping, buckets, chunk_align=A, transport=es.ES_TRANSPORT_LOOPBACK,
                        comm=world.value, sched=sched) for g in range(G)]
-    if sched == es.ES_SCHED_PEER:                 # same process: peers map by raw address
+    if sched in es.PEER_SCHEDS:                   # same process: peers map by raw address
         blobs = [a.peer_blob() for a in aggs]
         for a in aggs:
             a.peer_open(blobs)

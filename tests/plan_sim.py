@@ -40,6 +40,8 @@ class RankExec:
         self.sched = sched
         self.out = [np.zeros(L, np.float32 if d == "f32" else np.uint16) for L, d in buckets]
         self.result = [np.zeros(L, np.float32 if d == "f32" else np.uint16) for L, d in buckets]   # PEER
+        self.peer_parts = {}        # PEER_CHAIN: byte offset -> (lo, fp32 partial), read by the next GPU
+        self.world = [self]
         self.nbar = 0
         self.b = 0
         self.pc = 0
@@ -53,7 +55,7 @@ class RankExec:
 
     def _src(self, e, lo, hi):
         b = self.b
-        if self.map[e] == self.g or self.sched == es.ES_SCHED_PEER:
+        if self.map[e] == self.g or self.plans[b][1] in (es.ES_SCHED_PEER, es.ES_SCHED_PEER_CHAIN):
             return self.xs[b][e][lo:hi]          # local slot, or (PEER) the owner's slot over NVLink
         slo, arr = self.stage[e]
         assert slo <= lo and hi <= slo + arr.size, "staging does not cover the fold range"
@@ -83,6 +85,10 @@ class RankExec:
                 plo, parr = self.parts[inid]
                 acc = parr[a - plo:z - plo].copy()
                 rest = order
+            elif ink == es.ES_BUF_PEER_PART:      # producer rank inid, byte offset f[9]
+                plo, parr = self.world[inid].peer_parts[int(f[9])]
+                acc = parr[a - plo:z - plo].copy()
+                rest = order
             else:
                 acc = widen(self._src(order[0], a, z)).copy()
                 rest = order[1:]
@@ -91,6 +97,8 @@ class RankExec:
             if outk == es.ES_BUF_RESULT:
                 r = np.float32(1) / np.float32(self.N)
                 self.result[self.b][a:z] = narrow(acc * r, d)
+            elif outk == es.ES_BUF_PART and self.plans[self.b][1] == es.ES_SCHED_PEER_CHAIN:
+                self.peer_parts[outid] = (lo, acc.copy())
             elif outk == es.ES_BUF_PART:
                 if outid not in self.parts:
                     self.parts[outid] = (lo, np.zeros(hi - lo, np.float32))
@@ -134,6 +142,8 @@ class RankExec:
                 self.b += 1
                 self.pc = 0
                 self.stage, self.parts = {}, {}
+                # peer_parts survive until every rank passed the next barrier; keep them (offsets are reused
+                # per bucket, and a bucket's consumers read them before the bucket's next barrier)
                 progressed = True
                 continue
             f = ops[self.pc]
@@ -209,6 +219,8 @@ class Mailbox:
 
 def simulate(N, G, mapping, buckets, xs, A=16, sched=es.ES_SCHED_AUTO):
     ranks = [RankExec(N, G, g, mapping, buckets, xs, A, sched) for g in range(G)]
+    for r in ranks:
+        r.world = ranks
     box = Mailbox(ranks)
     while not all(r.done() for r in ranks):
         if not any(r.run(box) for r in ranks if not r.done()):

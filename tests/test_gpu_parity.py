@@ -206,7 +206,7 @@ def test_all_mappings_n4_loopback(G):
     xs = [_gauss(rng, 4, 1001), _gauss(rng, 4, 64, "bf16"), _gauss(rng, 4, 3)]
     want = [oracle.reduce(xs[0], "f32"), oracle.reduce(xs[1], "bf16"), oracle.reduce(xs[2], "f32")]
     for m in _surjections(4, G):
-        for sched in (es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_PEER):
+        for sched in (es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_PEER, es.ES_SCHED_PEER_CHAIN):
             res = reduce_loopback(xs, G, m, sched)
             for g in range(G):
                 for b in range(3):
@@ -215,7 +215,8 @@ def test_all_mappings_n4_loopback(G):
 
 @pytest.mark.parametrize("G,kind", [(2, "contiguous"), (4, "contiguous"), (8, "contiguous"), (8, "round_robin"),
                                     (4, "random"), (8, "random"), (3, "random")])
-@pytest.mark.parametrize("sched", [es.ES_SCHED_AUTO, es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_PEER])
+@pytest.mark.parametrize("sched", [es.ES_SCHED_AUTO, es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_PEER,
+                                   es.ES_SCHED_PEER_CHAIN, es.ES_SCHED_PEER_AUTO])
 def test_mappings_n8_loopback(G, kind, sched):
     rng = np.random.default_rng(G * 10 + len(kind))
     xs = [_gauss(rng, 8, 200003), _gauss(rng, 8, 4096 + 5, "bf16")]
@@ -241,7 +242,7 @@ def test_bert_uneven_n12_g8_loopback(kind):
             assert_bits_equal(res[g][b], want[b], f"{kind} rank={g} b={b}")
 
 
-@pytest.mark.parametrize("sched", [es.ES_SCHED_CHAIN, es.ES_SCHED_DIRECT, es.ES_SCHED_PEER])
+@pytest.mark.parametrize("sched", [es.ES_SCHED_CHAIN, es.ES_SCHED_DIRECT, es.ES_SCHED_PEER, es.ES_SCHED_PEER_CHAIN])
 @pytest.mark.parametrize("batched", [False, True])
 def test_loopback_multi_step_reuse(sched, batched):
     """Three global steps on the same handles: slot / staging / partial reuse is ordered."""

@@ -49,7 +49,8 @@ def test_all_surjections_n4(G):
     xs = _data(4, Ls, dts, G)
     want = [oracle.reduce(x, d) for x, d in zip(xs, dts)]
     for m in _surjections(4, G):
-        for sched in (es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_AUTO, es.ES_SCHED_PEER):
+        for sched in (es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_AUTO, es.ES_SCHED_PEER,
+                      es.ES_SCHED_PEER_CHAIN, es.ES_SCHED_PEER_AUTO):
             _check(4, G, m, Ls, dts, sched, xs=xs, want=want)
 
 
@@ -60,7 +61,7 @@ def test_all_surjections_n6_g3():
     want = [oracle.reduce(x, d) for x, d in zip(xs, dts)]
     n = 0
     for m in _surjections(6, 3):
-        for sched in (es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_PEER):
+        for sched in (es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_PEER, es.ES_SCHED_PEER_CHAIN):
             _check(6, 3, m, Ls, dts, sched, xs=xs, want=want)
         n += 1
     assert n == 540
@@ -75,7 +76,8 @@ def test_config_shapes_small_buckets(name, G, kind):
     N = workloads.config(name)["N"]
     d = workloads.config(name)["dtype"]
     m = workloads.mapping(N, G, kind)
-    for sched in (es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_AUTO, es.ES_SCHED_PEER):
+    for sched in (es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_AUTO, es.ES_SCHED_PEER,
+                      es.ES_SCHED_PEER_CHAIN, es.ES_SCHED_PEER_AUTO):
         _check(N, G, m, [997, 4096 + 24, 13], [d, d, d], sched, seed=G)
 
 
@@ -121,7 +123,8 @@ def test_random_configs_property():
         Ls = [draw(st.integers(0, 700)) for _ in range(nb)]
         dts = [draw(st.sampled_from(["f32", "bf16"])) for _ in range(nb)]
         A = draw(st.sampled_from([8, 16, 32]))
-        sched = draw(st.sampled_from([es.ES_SCHED_AUTO, es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_PEER]))
+        sched = draw(st.sampled_from([es.ES_SCHED_AUTO, es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_PEER,
+                                      es.ES_SCHED_PEER_CHAIN, es.ES_SCHED_PEER_AUTO]))
         seed = draw(st.integers(0, 2 ** 31))
         return N, G, list(perm), Ls, dts, A, sched, seed
 
