@@ -158,6 +158,12 @@ def oracle_windows(name, fetch, budget_s, seed=0):
     return gbs, sample, windows
 
 
+def workload_config(args, cfg, G):
+    """The `config` keys both arms share (the same workload)."""
+    return {"workload": args.config, "N": cfg["N"], "G": G, "mapping": args.mapping, "sched": args.sched,
+            "buckets": len(cfg["buckets"]), "elements": sum(n for n, _ in cfg["buckets"]), "desc": cfg["desc"]}
+
+
 def run_reference(args, rank, world):
     if rank != 0:
         return
@@ -187,7 +193,8 @@ def run_reference(args, rank, world):
         "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GB/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 3), "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": cfg["dtype"], "data": "synthetic",
-        "config": {"workload": name, "N": cfg["N"], "G": world, "desc": cfg["desc"]},
+        "config": dict(workload_config(args, cfg, world), graph=False, api="C oracle (single thread)",
+                       l2="host memory"),
         "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
                          "sample": sample + "; ms_per_step extrapolates the full step"},
         "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -382,14 +389,12 @@ def main():
         "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": cfg["dtype"], "data": "synthetic",
-        "config": {"workload": name, "N": N, "G": G, "mapping": args.mapping, "sched": args.sched,
-                   "buckets": B, "elements": sum(n for n, _ in buckets), "graph": graph is not None,
+        "config": {**workload_config(args, cfg, G), "graph": graph is not None,
                    "api": "per-bucket" if args.per_bucket else ("incremental" if args.incremental else
                                                                ("zero-copy-inplace" if args.inplace else
                                                                 ("batched" if args.no_fuse else "batched+fused-switch"))),
                    "l2": ("inputs larger than L2 (%.1f MB of EST gradients per GPU per step)" % (in_bytes / 1e6))
-                   if flush is None else "L2 flushed between timed steps (512 MB write)",
-                   "desc": cfg["desc"]},
+                   if flush is None else "L2 flushed between timed steps (512 MB write)"},
         "roofline": {"bound": "hbm", "kernel": "k_fold", "achieved": round(achieved, 1) if achieved else None,
                      "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4) if achieved else None,
                      "traffic": traffic, "algorithmic_bytes_per_launch": int(per_launch),
