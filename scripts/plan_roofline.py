@@ -1,0 +1,110 @@
+"""Multi-GPU roofline of the ACTUAL plans (host-only, no GPU).
+
+For every BASELINE config, G and schedule, export each rank's op list through
+the C ABI (es_plan_ops) and count, per rank: bytes received over NVLink
+(RECV ops, peer reads of PEER folds / chain partials, GATHER of remote
+shards) and HBM bytes (fold reads/writes, staging writes, gathers).  The step
+time bound is the slowest rank's max(HBM / 6.54 TB/s, NVLink / 0.77 TB/s);
+chain rounds are separated by barriers, so for CHAIN / PEER_CHAIN the bound
+is summed over rounds.  Stash bytes are excluded (allreduce
+only).  Writes profiles/r01_plan_roofline.md.
+
+  python scripts/plan_roofline.py [out.md]
+"""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+from paper_conf_sc_lixyszrljlllq23_b200 import es, workloads  # noqa: E402
+
+HBM = 6541.5e9          # MEASURED_PEAKS hbm_gbs (copy)
+NVL = 770e9             # B200_PROFILING.md measured peer copy per direction
+SCHEDS = {"direct": es.ES_SCHED_DIRECT, "chain": es.ES_SCHED_CHAIN, "peer": es.ES_SCHED_PEER,
+          "peer_chain": es.ES_SCHED_PEER_CHAIN}
+
+
+def rank_costs(name, G, kind, sched):
+    """-> list over ranks of list over phases of (hbm_bytes, nvlink_in_bytes)."""
+    c = workloads.config(name)
+    N = c["N"]
+    m = workloads.mapping(N, G, kind)
+    buckets = [(n, es.ES_F32 if d == "f32" else es.ES_BF16) for n, d in c["buckets"]]
+    out = []
+    for g in range(G):
+        cfg = es.Config(N, G, g, m, buckets, sched=sched)
+        phases = {}
+        for b, (L, dt) in enumerate(buckets):
+            esz = 2 if dt == es.ES_BF16 else 4
+            ops, _ = es.es_plan_ops(cfg, b)
+            ph = 0
+            for f in ops:
+                op = int(f[0])
+                if op in (es.ES_OP_BARRIER, es.ES_OP_GROUP_END):
+                    ph += 1
+                    continue
+                hb, nv = phases.get(ph, (0, 0))
+                lo, hi = int(f[1]), int(f[2])
+                n = hi - lo
+                if op == es.ES_OP_FOLD:
+                    srcs = N if int(f[3]) < 0 else int(f[4])
+                    remote = 0
+                    if int(f[3]) < 0 and sched == es.ES_SCHED_PEER:
+                        remote = sum(1 for e in range(N) if m[e] != g)
+                    hb += n * esz * (srcs - remote)                        # local contributions
+                    nv += n * esz * remote                                  # peer slots over NVLink
+                    if int(f[5]) == es.ES_BUF_PART:
+                        hb += n * 4
+                    elif int(f[5]) == es.ES_BUF_PEER_PART:
+                        nv += n * 4
+                    hb += n * (4 if int(f[7]) == es.ES_BUF_PART else esz)   # write
+                elif op == es.ES_OP_RECV:
+                    w = 4 if int(f[4]) == es.ES_BUF_PART else esz
+                    nv += n * w
+                    hb += n * w
+                elif op == es.ES_OP_GATHER:
+                    if int(f[3]) != g:
+                        nv += n * esz
+                    hb += n * esz * (2 if int(f[3]) == g else 1)
+                phases[ph] = (hb, nv)
+        out.append([phases[k] for k in sorted(phases)])
+    return out
+
+
+def bound_ms(costs):
+    nph = max(len(r) for r in costs)
+    t = 0.0
+    for k in range(nph):
+        t += max(max(r[k][0] / HBM, r[k][1] / NVL) if k < len(r) else 0.0 for r in costs)
+    return t * 1e3
+
+
+def main(path):
+    rows = ["# Multi-GPU roofline of the exported plans (allreduce only; HBM 6.54 TB/s, NVLink 0.77 TB/s)\n",
+            "Per phase (between groups / barriers), the slowest rank's max(HBM, NVLink) time, summed.\n",
+            "| config | G | mapping | direct ms | chain ms | peer ms | peer_chain ms | AUTO picks | max NVLink in / rank MB (direct, chain) |",
+            "|---|---|---|---|---|---|---|---|---|"]
+    cases = [("resnet50", G, "contiguous") for G in (2, 4, 8)] + [("vgg19", G, "contiguous") for G in (2, 4, 8)] + \
+        [("bert_base", 8, "contiguous"), ("bert_base", 8, "round_robin")] + \
+        [("swin_b", G, "contiguous") for G in (2, 4, 8)]
+    for name, G, kind in cases:
+        res = {k: rank_costs(name, G, kind, v) for k, v in SCHEDS.items()}
+        c = workloads.config(name)
+        cfg = es.Config(c["N"], G, 0, workloads.mapping(c["N"], G, kind),
+                        [(n, es.ES_F32 if d == "f32" else es.ES_BF16) for n, d in c["buckets"]])
+        picks = sorted({es.es_plan_ops(cfg, b)[1] for b in range(len(c["buckets"]))})
+        pick = "/".join({1: "direct", 2: "chain"}[p] for p in picks)
+        nvd = max(sum(ph[1] for ph in r) for r in res["direct"]) / 1e6
+        nvc = max(sum(ph[1] for ph in r) for r in res["chain"]) / 1e6
+        rows.append(f"| {name} | {G} | {kind} | {bound_ms(res['direct']):.3f} | {bound_ms(res['chain']):.3f} | "
+                    f"{bound_ms(res['peer']):.3f} | {bound_ms(res['peer_chain']):.3f} | {pick} | "
+                    f"{nvd:.0f}, {nvc:.0f} |")
+    text = "\n".join(rows) + "\n"
+    with open(path, "w") as f:
+        f.write(text)
+    print(text)
+
+
+if __name__ == "__main__":
+    main(sys.argv[1] if len(sys.argv) > 1 else os.path.join(ROOT, "profiles", "r01_plan_roofline.md"))
