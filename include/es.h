@@ -292,9 +292,12 @@ es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void
  * to es_peer_open, which maps every peer's workspace (cudaIpcOpenMemHandle
  * with lazy peer access; the raw address when the peer lives in the same
  * process, as with the loopback transport).  Required before the first
- * es_allreduce of a handle whose schedule is PEER; ES_EUNSUPPORTED if the
- * workspace cannot be IPC-exported (e.g. a VMM / expandable-segments
- * allocation). */
+ * es_allreduce of a handle whose schedule is a peer one; ES_EUNSUPPORTED if
+ * the workspace cannot be IPC-exported (e.g. a VMM / expandable-segments
+ * allocation) or if more ranks share this process (loopback) than
+ * CUDA_DEVICE_MAX_CONNECTIONS (default 8): their spinning barrier kernels
+ * need a hardware queue each.  A peer that never arrives at a barrier makes
+ * the kernel trap after 60 s (sticky ES_ECUDA), never hang the GPU. */
 #define ES_PEER_BLOB_BYTES 128
 es_status es_peer_blob(es_handle h, void *blob, size_t bytes);
 es_status es_peer_open(es_handle h, const void *blobs, size_t bytes);

@@ -2,6 +2,8 @@
 // slots, EST context export / import (elastic resume), per-EST dropout.
 #include <unistd.h>
 
+#include <cstdlib>
+
 #include "handle.h"
 
 extern "C" {
@@ -76,6 +78,20 @@ es_status es_peer_open(es_handle h, const void *blobs, size_t bytes) {
   std::vector<unsigned char *> ws(p.G, nullptr);
   std::vector<void *> mapped;
   const int32_t me = (int32_t)getpid();
+  // Ranks sharing this process (loopback) share one device: their barrier
+  // kernels spin concurrently on different streams, which needs one hardware
+  // queue per rank -- more ranks than CUDA_DEVICE_MAX_CONNECTIONS (default 8)
+  // would serialise a spinning barrier in front of a peer's work.
+  int32_t same_process = 0;
+  for (int32_t g = 0; g < p.G; ++g) {
+    PeerBlob b;
+    std::memcpy(&b, reinterpret_cast<const unsigned char *>(blobs) + (size_t)g * ES_PEER_BLOB_BYTES, sizeof b);
+    same_process += b.pid == me;
+  }
+  const char *mc = std::getenv("CUDA_DEVICE_MAX_CONNECTIONS");
+  const int32_t max_conn = mc ? std::atoi(mc) : 8;
+  if (same_process > 1 && same_process > max_conn)
+    return set_err(ES_EUNSUPPORTED, "more same-process peer ranks than CUDA_DEVICE_MAX_CONNECTIONS hardware queues");
   for (int32_t g = 0; g < p.G; ++g) {
     PeerBlob b;
     std::memcpy(&b, reinterpret_cast<const unsigned char *>(blobs) + (size_t)g * ES_PEER_BLOB_BYTES, sizeof b);

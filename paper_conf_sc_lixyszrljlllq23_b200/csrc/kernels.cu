@@ -930,7 +930,11 @@ struct BarrierParams {
 };
 
 __global__ void __launch_bounds__(64) k_peer_barrier(const __grid_constant__ BarrierParams p) {
-  pdl_enter();
+  // Wait for the predecessor, but let the successor's CTAs become resident
+  // only after the barrier has passed: waiting CTAs must never occupy SM
+  // slots other ranks need to reach this barrier (they share a GPU under the
+  // loopback transport).
+  asm volatile("griddepcontrol.wait;" ::: "memory");
   const int t = threadIdx.x;
   __threadfence_system();                       // this GPU's completed writes before the arrival
   if (t < p.G) {
@@ -951,6 +955,7 @@ __global__ void __launch_bounds__(64) k_peer_barrier(const __grid_constant__ Bar
   }
   __syncthreads();
   __threadfence_system();
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
 
 }  // namespace

@@ -513,3 +513,50 @@ def test_incremental_fold_protocol_and_graph():
         Aggregator(4, 2, 0, [0, 0, 1, 1], [(L, "f32")], options=es.ES_OPT_INCREMENTAL,
                    transport=es.ES_TRANSPORT_LOOPBACK, comm=es.es_loopback_create(2).value)
     assert e.value.status == es.ES_EINVAL
+
+
+# ---- maximum sizes ----------------------------------------------------------------------------
+
+def test_max_n_1024():
+    """N at its limit (1024 ESTs -> 1024 source pointers in one launch)."""
+    rng = np.random.default_rng(1024)
+    xs = [_gauss(rng, 1024, 20011)]
+    for batched in (False, True):
+        assert_bits_equal(reduce_g1(xs, batched=batched)[0], oracle.reduce(xs[0], "f32"), f"batched={batched}")
+
+
+def test_max_bucket_numel_2p31_minus_1():
+    """The largest legal bucket (2^31 - 1 elements, bf16, 4 GiB per EST): the
+    32-bit chunk arithmetic and 64-bit offsets hold to the last element."""
+    from gpu_util import Aggregator, from_dev
+    L, N = (1 << 31) - 1, 3
+    g = torch.Generator(device="cuda").manual_seed(31)
+    xs = [(torch.randn(L, generator=g, device="cuda") * 1e-3).to(torch.bfloat16) for _ in range(N)]
+    agg = Aggregator(N, 1, 0, [0] * N, [(L, "bf16")])
+    for k in range(N):
+        agg.stash(k, 0, xs[k], es.ES_STASH_BORROW if k == N - 1 else es.ES_STASH_COPY)
+    out = agg.new_out(0)
+    agg.allreduce(0, out)
+    torch.cuda.synchronize()
+    C = oracle.chunk_elems(L, N)
+    for s in [0, C - 9, 2 * C - 5, L - 4099, (1 << 30) + 7]:
+        n = min(4099, L - s)
+        want = oracle.reduce([from_dev(x[s:s + n]) for x in xs], "bf16", L=L, first=s)
+        assert_bits_equal(from_dev(out[s:s + n]), want, f"s={s}")
+    agg.close()
+    with pytest.raises(es.EsError):                     # 2^31 is refused
+        es.es_workspace_bytes(es.Config(2, 1, 0, [0, 0], [(1 << 31, es.ES_BF16)]))
+
+
+def test_sixteen_loopback_ranks():
+    rng = np.random.default_rng(16)
+    xs = [_gauss(rng, 40, 50021), _gauss(rng, 40, 999, "bf16")]
+    want = [oracle.reduce(xs[0], "f32"), oracle.reduce(xs[1], "bf16")]
+    res = reduce_loopback(xs, 16, workloads.mapping(40, 16, "random", seed=5), es.ES_SCHED_AUTO)
+    for g in range(16):
+        for b in range(2):
+            assert_bits_equal(res[g][b], want[b], f"rank={g} b={b}")
+    # peer schedules need a hardware queue per same-process rank: refused, never hung
+    with pytest.raises(es.EsError) as e:
+        reduce_loopback(xs, 16, workloads.mapping(40, 16, "random", seed=5), es.ES_SCHED_PEER_AUTO)
+    assert e.value.status == es.ES_EUNSUPPORTED
