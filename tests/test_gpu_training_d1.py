@@ -1,0 +1,184 @@
+"""GPU: D1 elastic determinism at the training level -- a synthetic Fig. 9.
+
+PAPER.md:1032-1080 (Fig. 9) trains the same job on 4 V100 -> 2 V100 -> mixed
+GPUs and shows the loss is bitwise identical to fixed-DoP DDP.  Here a small
+MLP is trained by N = 4 ESTs for 4 global steps on G = 1, 2 and 4 "GPUs"
+(ranks over the loopback transport on this one device), and once with an
+elastic change G = 4 -> 2 after step 2 (on-demand checkpoint of the EST
+contexts).  Each EST draws its dropout masks from its own
+device Philox record (NEXT-4, swapped by es_switch_context) and its
+gradients are aggregated by es_allreduce in the canonical order.  Every run
+must end with bitwise identical parameters -- and G = 4 with one EST per
+rank is plain data-parallel training, the paper's DDP baseline.
+"""
+import os
+import threading
+
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_sc_lixyszrljlllq23_b200 import es
+from paper_conf_sc_lixyszrljlllq23_b200.aggregator import Aggregator
+
+pytestmark = pytest.mark.gpu
+os.environ.setdefault("CUBLAS_WORKSPACE_CONFIG", ":4096:8")
+
+N, D_IN, D_H, D_OUT, BATCH, P_DROP, LR = 4, 32, 64, 8, 16, 0.25, 0.05
+SEEDS = [7000 + 13 * k for k in range(N)]
+
+
+class EsDropout(torch.autograd.Function):
+    """Dropout whose mask comes from the running EST's device Philox record."""
+
+    @staticmethod
+    def forward(ctx, x, agg):
+        y, mask = agg.dropout(x.contiguous(), P_DROP, with_mask=True)
+        scale = np.float32(1) / (np.float32(1) - np.float32(P_DROP))
+        ctx.save_for_backward(mask.view(x.shape).to(x.dtype) * torch.tensor(float(scale), device=x.device))
+        return y.view(x.shape)
+
+    @staticmethod
+    def backward(ctx, g):
+        (m,) = ctx.saved_tensors
+        return g * m, None
+
+
+def make_model():
+    torch.manual_seed(1234)
+    w1 = (torch.randn(D_H, D_IN) * 0.2).cuda().requires_grad_()
+    w2 = (torch.randn(D_OUT, D_H) * 0.2).cuda().requires_grad_()
+    return [w1, w2]
+
+
+def batch(step, k):
+    g = torch.Generator().manual_seed(100000 * step + k)
+    x = torch.randn(BATCH, D_IN, generator=g)
+    y = torch.randn(BATCH, D_OUT, generator=g)
+    return x.cuda(), y.cuda()
+
+
+def flat_grad(params):
+    return torch.cat([p.grad.reshape(-1) for p in params])
+
+
+class Rank:
+    """One rank (GPU) of the job: a parameter replica and an aggregator."""
+
+    def __init__(self, G, r, mapping, world, chunk_align=16):
+        self.params = make_model()
+        self.n = sum(p.numel() for p in self.params)
+        self.agg = Aggregator(N, G, r, mapping, [(self.n, "f32")], state_nbytes=[16], chunk_align=chunk_align,
+                              transport=es.ES_TRANSPORT_LOOPBACK if G > 1 else es.ES_TRANSPORT_NONE,
+                              comm=world.value if G > 1 else None)
+        self.live = [torch.zeros(16, dtype=torch.uint8, device="cuda")]
+        self.agg.register_state(self.live)
+        self.stream = torch.cuda.Stream()
+
+    def init_contexts(self):
+        for k in self.agg.local_ests:
+            self.agg.init_state(k, 0, int(SEEDS[k]).to_bytes(8, "little") + bytes(8))
+
+    def step(self, step):
+        """Local steps of every local EST, then the aggregation."""
+        w1, w2 = self.params
+        bufs = []
+        loc = self.agg.local_ests
+        for i, k in enumerate(loc):
+            self.agg.switch(k)                                   # RNG context of EST k
+            x, y = batch(step, k)
+            h = torch.relu(x @ w1.t())
+            h = EsDropout.apply(h, self.agg)
+            loss = ((h @ w2.t() - y) ** 2).mean()
+            for p in self.params:
+                p.grad = None
+            loss.backward()
+            g = flat_grad(self.params).contiguous()
+            bufs.append(g)
+            self.agg.stash(k, 0, g, es.ES_STASH_BORROW if i == len(loc) - 1 else es.ES_STASH_COPY)
+        avg = torch.empty(self.n, device="cuda")
+        self.agg.allreduce(0, avg)
+        with torch.no_grad():                                    # replicated SGD update
+            off = 0
+            for p in self.params:
+                p -= LR * avg[off:off + p.numel()].view_as(p)
+                off += p.numel()
+
+    def close(self):
+        self.agg.close()
+
+
+def run_stage(ranks, steps):
+    errs = []
+
+    def work(r):
+        try:
+            with torch.cuda.stream(ranks[r].stream):
+                for s in steps:
+                    ranks[r].step(s)
+        except Exception as e:
+            errs.append(e)
+    ts = [threading.Thread(target=work, args=(r,)) for r in range(len(ranks))]
+    [t.start() for t in ts]
+    [t.join(timeout=300) for t in ts]
+    torch.cuda.synchronize()
+    if errs:
+        raise errs[0]
+
+
+def new_stage(G, mapping, chunk_align=16):
+    world = es.es_loopback_create(G) if G > 1 else None
+    ranks = [Rank(G, r, mapping, world, chunk_align) for r in range(G)]
+    return world, ranks
+
+
+def train(G, mapping, steps, chunk_align=16):
+    world, ranks = new_stage(G, mapping, chunk_align)
+    for r in ranks:
+        r.init_contexts()
+    run_stage(ranks, steps)
+    final = [[p.detach().clone() for p in r.params] for r in ranks]
+    for r in ranks:
+        r.close()
+    if world is not None:
+        es.es_loopback_destroy(world)
+    return final
+
+
+def bits(ts):
+    return [t.view(torch.int32).cpu() for t in ts]
+
+
+def test_training_is_bitwise_identical_across_g_and_elastic_change():
+    torch.backends.cuda.matmul.allow_tf32 = False
+    steps = [0, 1, 2, 3]
+    ref = bits(train(1, [0, 0, 0, 0], steps)[0])                       # 4 ESTs time-sliced on 1 GPU
+    for G, mapping in [(2, [0, 0, 1, 1]), (2, [1, 0, 1, 0]), (4, [0, 1, 2, 3])]:  # G = 4: plain DDP
+        for rank_params in train(G, mapping, steps):
+            assert all(torch.equal(a, b) for a, b in zip(bits(rank_params), ref)), (G, mapping)
+    # elastic: G = 4 for steps 0-1, on-demand checkpoint, G = 2 (other mapping) for steps 2-3
+    world, ranks = new_stage(4, [0, 1, 2, 3])
+    for r in ranks:
+        r.init_contexts()
+    run_stage(ranks, [0, 1])
+    params = [p.detach().clone() for p in ranks[0].params]             # one replica
+    blobs = {k: ranks[k].agg.export_context(k) for k in range(N)}      # EST contexts: Philox records
+    for r in ranks:
+        r.close()
+    es.es_loopback_destroy(world)
+    world, ranks = new_stage(2, [1, 1, 0, 0])
+    for r in ranks:
+        with torch.no_grad():
+            for p, q in zip(r.params, params):
+                p.copy_(q)
+        for k in r.agg.local_ests:
+            r.agg.import_context(k, blobs[k])
+    run_stage(ranks, [2, 3])
+    for r in ranks:
+        assert all(torch.equal(a, b) for a, b in zip(bits(r.params), ref)), "elastic run diverged"
+        r.close()
+    es.es_loopback_destroy(world)
+    # negative control (R8): another persisted layout -- here the chunk
+    # alignment -- changes the aggregation order and therefore the trained bits
+    other = bits(train(1, [0, 0, 0, 0], steps, chunk_align=1024)[0])
+    assert not all(torch.equal(a, b) for a, b in zip(other, ref))
