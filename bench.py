@@ -376,14 +376,29 @@ def main():
     payload = workloads.payload_bytes(name)
     value = payload / (ms / 1e3) / 1e9
     peak, peak_src = peaks()
-    achieved = fl_bytes / (fl_ms / 1e3) / 1e9 if fl_ms > 0 else None
-    per_launch = fl_bytes / max(fl_n, 1)
-    traffic = None
+    # Roofline of every HBM kernel of the step; `roofline` is the dominant one
+    # (largest share of the profiled step's device time).
+    traffic_all = {}
     tfile = os.path.join(ROOT, "profiles", f"traffic_{name}_g{G}.json")
     if os.path.exists(tfile) and not (args.incremental or args.per_bucket or args.no_fuse or args.no_graph
                                       or args.inplace):
         with open(tfile) as f:
-            traffic = json.load(f).get("fold_dram_bytes_per_launch")
+            traffic_all = json.load(f)
+
+    def roof(kind, kname):
+        n_, ms_, bytes_ = prof[kind]
+        if n_ == 0 or ms_ <= 0:
+            return None
+        a = bytes_ / (ms_ / 1e3) / 1e9
+        return {"bound": "hbm", "kernel": kname, "achieved": round(a, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(a / peak, 4), "traffic": traffic_all.get(f"{kname}_dram_bytes_per_launch"),
+                "algorithmic_bytes_per_launch": int(bytes_ / n_), "launches_per_step": int(n_ / steps_profiled),
+                "avg_launch_us": round(ms_ / n_ * 1e3, 2), "share_of_step": round(ms_ / steps_profiled / ms, 3),
+                "peak_source": peak_src}
+
+    roofs = {k: r for k, r in (("k_fold", roof("fold", "k_fold")), ("k_stash", roof("stash", "k_stash")),
+                               ("k_gather", roof("gather", "k_gather"))) if r is not None}
+    dominant = max(roofs.values(), key=lambda r: r["share_of_step"]) if roofs else None
 
     line = {
         "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
@@ -395,11 +410,8 @@ def main():
                                                                 ("batched" if args.no_fuse else "batched+fused-switch"))),
                    "l2": ("inputs larger than L2 (%.1f MB of EST gradients per GPU per step)" % (in_bytes / 1e6))
                    if flush is None else "L2 flushed between timed steps (512 MB write)"},
-        "roofline": {"bound": "hbm", "kernel": "k_fold", "achieved": round(achieved, 1) if achieved else None,
-                     "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4) if achieved else None,
-                     "traffic": traffic, "algorithmic_bytes_per_launch": int(per_launch),
-                     "launches_per_step": int(fl_n / steps_profiled),
-                     "avg_launch_us": round(fl_ms / max(fl_n, 1) * 1e3, 2), "peak_source": peak_src},
+        "roofline": dominant,
+        "roofline_by_kernel": roofs,
         "breakdown_ms_per_step": {k: round(v[1] / steps_profiled, 4) for k, v in prof.items()},
         "per_kernel": {k: {"launches_per_step": int(v[0] / steps_profiled),
                            "algorithmic_GBps": round(v[2] / (v[1] / 1e3) / 1e9, 1) if v[1] > 0 else None,

@@ -77,6 +77,14 @@ __device__ __forceinline__ void st_stream(uint2 *p, const uint2 &v) {
   asm volatile("st.global.L1::no_allocate.v2.u32 [%0], {%1, %2};" ::"l"(p), "r"(v.x), "r"(v.y) : "memory");
 }
 __device__ __forceinline__ void st_stream(int4 *p, const int4 &v) { st_stream(static_cast<void *>(p), v); }
+// Cache-streaming (evict-first) stores: experiment for the stash (ES_STASH_VARIANT=3).
+__device__ __forceinline__ void st_cs(int4 *p, const int4 &v) {
+  asm volatile("st.global.cs.v4.s32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+               : "memory");
+}
+__device__ __forceinline__ void st_cs(uint2 *p, const uint2 &v) {
+  asm volatile("st.global.cs.v2.u32 [%0], {%1, %2};" ::"l"(p), "r"(v.x), "r"(v.y) : "memory");
+}
 
 __device__ __forceinline__ uint32_t smem_addr(const void *p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -613,7 +621,7 @@ int swap_blocks_per_entry(uint64_t max_nbytes) {
   return (int)std::max<uint64_t>(1, std::min<uint64_t>((words + 255) / 256, 64));
 }
 
-template <typename S, typename D, int E, int kU, int MAXSEG>
+template <typename S, typename D, int E, int kU, int MAXSEG, int ST>
 __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashParams<MAXSEG> p) {
   using In = typename VecT<S::kSize * E>::T;
   using Out = typename VecT<D::kSize * E>::T;
@@ -643,7 +651,10 @@ __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashPara
 #pragma unroll
     for (int u = 0; u < kU; ++u) {
       const int64_t i = u0 + u * stride;
-      if (i < nunits) st_stream(d + i, Cast<S, D, E>::apply(in[u]));
+      if (i < nunits) {
+        if (ST == 1) st_cs(d + i, Cast<S, D, E>::apply(in[u]));
+        else st_stream(d + i, Cast<S, D, E>::apply(in[u]));
+      }
     }
   }
   const int64_t tail0 = nunits * E;
@@ -658,10 +669,10 @@ __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashPara
   }
 }
 
-template <typename S, typename D, int E>
-cudaError_t launch_stash_t(const StashSegDesc *segs, int nseg, cudaStream_t s, int bo, int to, int *launches,
+template <typename S, typename D, int E, int kU, int ST>
+cudaError_t launch_stash_v(const StashSegDesc *segs, int nseg, cudaStream_t s, int bo, int to, int *launches,
                            const SwapArgs *swap) {
-  constexpr int kU = 4, kMaxSeg = 32;
+  constexpr int kMaxSeg = 32;
   const int threads = to > 0 ? to : 256;
   for (int i = 0; i < nseg; i += kMaxSeg) {
     const int k = std::min(kMaxSeg, nseg - i);
@@ -690,11 +701,30 @@ cudaError_t launch_stash_t(const StashSegDesc *segs, int nseg, cudaStream_t s, i
     split_blocks(work, total, &block0, &p.nblocks);
     for (int j = 0; j < k; ++j) p.seg[j].block0 = block0[j];
     const int grid = p.nblocks + p.swap_bx * p.swap_n;
-    cudaError_t e = launch(k_stash<S, D, E, kU, kMaxSeg>, dim3(grid), dim3(threads), s, p);
+    cudaError_t e = launch(k_stash<S, D, E, kU, kMaxSeg, ST>, dim3(grid), dim3(threads), s, p);
     if (e != cudaSuccess) return e;
     ++*launches;
   }
   return cudaSuccess;
+}
+
+// ES_STASH_VARIANT (measured in profiles/): 0 = 4 units/thread (default),
+// 1 = 8, 2 = 2, 3 = 4 with cache-streaming stores, 4 = 1 unit/thread.
+int g_stash_variant = [] {
+  const char *e = std::getenv("ES_STASH_VARIANT");
+  return e ? std::atoi(e) : 0;
+}();
+
+template <typename S, typename D, int E>
+cudaError_t launch_stash_t(const StashSegDesc *segs, int nseg, cudaStream_t s, int bo, int to, int *launches,
+                           const SwapArgs *swap) {
+  switch (g_stash_variant) {
+    case 1: return launch_stash_v<S, D, E, 8, 0>(segs, nseg, s, bo, to, launches, swap);
+    case 2: return launch_stash_v<S, D, E, 2, 0>(segs, nseg, s, bo, to, launches, swap);
+    case 3: return launch_stash_v<S, D, E, 4, 1>(segs, nseg, s, bo, to, launches, swap);
+    case 4: return launch_stash_v<S, D, E, 1, 0>(segs, nseg, s, bo, to, launches, swap);
+    default: return launch_stash_v<S, D, E, 4, 0>(segs, nseg, s, bo, to, launches, swap);
+  }
 }
 
 // ---- k_copy_tma: TMA bulk-copy stash for same-dtype segments ------------------
