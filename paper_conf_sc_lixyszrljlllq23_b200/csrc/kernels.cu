@@ -621,7 +621,7 @@ int swap_blocks_per_entry(uint64_t max_nbytes) {
   return (int)std::max<uint64_t>(1, std::min<uint64_t>((words + 255) / 256, 64));
 }
 
-template <typename S, typename D, int E, int kU, int MAXSEG, int ST>
+template <typename S, typename D, int E, int kU, int MAXSEG, int ST, bool CR = false>
 __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashParams<MAXSEG> p) {
   using In = typename VecT<S::kSize * E>::T;
   using Out = typename VecT<D::kSize * E>::T;
@@ -639,27 +639,36 @@ __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashPara
   const In *s = reinterpret_cast<const In *>(g.src);
   Out *d = reinterpret_cast<Out *>(g.dst);
   const int64_t nunits = g.n / E;
-  const int64_t stride = (int64_t)nb * blockDim.x;
-  const int64_t gid = (int64_t)(bid - g.block0) * blockDim.x + threadIdx.x;
-  for (int64_t u0 = gid; u0 < nunits; u0 += stride * kU) {
+  int64_t stride = (int64_t)nb * blockDim.x;
+  int64_t gid = (int64_t)(bid - g.block0) * blockDim.x + threadIdx.x;
+  int64_t ubeg = 0, uend = nunits;
+  if (CR) {   // contiguous, equal range per block (balanced: every block finishes together)
+    const int64_t per = ((nunits + nb - 1) / nb + blockDim.x - 1) / blockDim.x * blockDim.x;
+    ubeg = min(nunits, (int64_t)(bid - g.block0) * per);
+    uend = min(nunits, ubeg + per);
+    stride = blockDim.x;
+    gid = ubeg + threadIdx.x;
+  }
+  for (int64_t u0 = gid; u0 < uend; u0 += stride * kU) {
     In in[kU];
 #pragma unroll
     for (int u = 0; u < kU; ++u) {
       const int64_t i = u0 + u * stride;
-      if (i < nunits) in[u] = ld_stream(s + i);
+      if (i < uend) in[u] = ld_stream(s + i);
     }
 #pragma unroll
     for (int u = 0; u < kU; ++u) {
       const int64_t i = u0 + u * stride;
-      if (i < nunits) {
+      if (i < uend) {
         if (ST == 1) st_cs(d + i, Cast<S, D, E>::apply(in[u]));
         else st_stream(d + i, Cast<S, D, E>::apply(in[u]));
       }
     }
   }
   const int64_t tail0 = nunits * E;
-  if (gid < g.n - tail0) {
-    const int64_t i = tail0 + gid;
+  const int64_t tid0 = (int64_t)(bid - g.block0) * blockDim.x + threadIdx.x;
+  if (tid0 < g.n - tail0) {
+    const int64_t i = tail0 + tid0;
     if (S::kSize == D::kSize) {
       if (S::kSize == 4) reinterpret_cast<uint32_t *>(g.dst)[i] = reinterpret_cast<const uint32_t *>(g.src)[i];
       else reinterpret_cast<uint16_t *>(g.dst)[i] = reinterpret_cast<const uint16_t *>(g.src)[i];
@@ -669,7 +678,7 @@ __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashPara
   }
 }
 
-template <typename S, typename D, int E, int kU, int ST>
+template <typename S, typename D, int E, int kU, int ST, bool CR = false>
 cudaError_t launch_stash_v(const StashSegDesc *segs, int nseg, cudaStream_t s, int bo, int to, int *launches,
                            const SwapArgs *swap) {
   constexpr int kMaxSeg = 32;
@@ -695,21 +704,34 @@ cudaError_t launch_stash_v(const StashSegDesc *segs, int nseg, cudaStream_t s, i
     }
     int total = (int)std::min<int64_t>((units + (int64_t)threads * kU - 1) / ((int64_t)threads * kU),
                                        (int64_t)kMaxBlocks);
+    if (CR) {   // whole waves of resident blocks
+      static int resident = 0;
+      if (!resident) {
+        int per_sm = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_stash<S, D, E, kU, kMaxSeg, ST, CR>, threads, 0);
+        resident = std::max(1, per_sm) * kSMs;
+      }
+      const int64_t waves = std::max<int64_t>(1, (total + resident / 2) / resident);
+      total = (int)std::min<int64_t>(waves * resident, (int64_t)kMaxBlocks);
+    }
     if (bo > 0) total = bo;
     total = std::max(total, k);
     std::vector<int32_t> block0;
     split_blocks(work, total, &block0, &p.nblocks);
     for (int j = 0; j < k; ++j) p.seg[j].block0 = block0[j];
     const int grid = p.nblocks + p.swap_bx * p.swap_n;
-    cudaError_t e = launch(k_stash<S, D, E, kU, kMaxSeg, ST>, dim3(grid), dim3(threads), s, p);
+    cudaError_t e = launch(k_stash<S, D, E, kU, kMaxSeg, ST, CR>, dim3(grid), dim3(threads), s, p);
     if (e != cudaSuccess) return e;
     ++*launches;
   }
   return cudaSuccess;
 }
 
-// ES_STASH_VARIANT (measured in profiles/): 0 = 4 units/thread (default),
-// 1 = 8, 2 = 2, 3 = 4 with cache-streaming stores, 4 = 1 unit/thread.
+// ES_STASH_VARIANT (measured in profiles/r01_stash_variants.md):
+// 0 (default) = one contiguous, equal range per block, whole waves of
+// resident blocks, 4 units per thread in flight; 5 = the one-shot grid
+// (~1 iteration per thread); 1 / 2 / 4 = one-shot with 8 / 2 / 1 units;
+// 3 = one-shot with cache-streaming stores; 6 = contiguous ranges, 8 units.
 int g_stash_variant = [] {
   const char *e = std::getenv("ES_STASH_VARIANT");
   return e ? std::atoi(e) : 0;
@@ -723,7 +745,9 @@ cudaError_t launch_stash_t(const StashSegDesc *segs, int nseg, cudaStream_t s, i
     case 2: return launch_stash_v<S, D, E, 2, 0>(segs, nseg, s, bo, to, launches, swap);
     case 3: return launch_stash_v<S, D, E, 4, 1>(segs, nseg, s, bo, to, launches, swap);
     case 4: return launch_stash_v<S, D, E, 1, 0>(segs, nseg, s, bo, to, launches, swap);
-    default: return launch_stash_v<S, D, E, 4, 0>(segs, nseg, s, bo, to, launches, swap);
+    case 5: return launch_stash_v<S, D, E, 4, 0>(segs, nseg, s, bo, to, launches, swap);   // one-shot grid
+    case 6: return launch_stash_v<S, D, E, 8, 0, true>(segs, nseg, s, bo, to, launches, swap);
+    default: return launch_stash_v<S, D, E, 4, 0, true>(segs, nseg, s, bo, to, launches, swap);
   }
 }
 
