@@ -200,6 +200,7 @@ struct FoldParams {
   int32_t nseg, N, nblocks;
   float r;
   uint32_t compat;        // NEXT-3 variant bits (COMPAT kernels only)
+  int32_t contiguous;     // 1: each block folds one contiguous, equal range of its segment
   FoldSeg seg[MAXSEG];
   const void *src[MAXSRC];
 };
@@ -326,9 +327,16 @@ __global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams
   const int nb = (si + 1 < p.nseg ? p.seg[si + 1].block0 : p.nblocks) - g.block0;
   const void *const *src = p.src + g.src0;
   const int64_t nvec = g.n / V;
-  const int64_t stride = (int64_t)nb * blockDim.x;
-  const int64_t gid = (int64_t)(blockIdx.x - g.block0) * blockDim.x + threadIdx.x;
-  for (int64_t v = gid; v < nvec; v += stride) {
+  const int64_t tid0 = (int64_t)(blockIdx.x - g.block0) * blockDim.x + threadIdx.x;
+  int64_t stride = (int64_t)nb * blockDim.x, gid = tid0, vend = nvec;
+  if (p.contiguous) {
+    const int64_t per = ((nvec + nb - 1) / nb + blockDim.x - 1) / blockDim.x * blockDim.x;
+    const int64_t vb = min(nvec, (int64_t)(blockIdx.x - g.block0) * per);
+    vend = min(nvec, vb + per);
+    stride = blockDim.x;
+    gid = vb + threadIdx.x;
+  }
+  for (int64_t v = gid; v < vend; v += stride) {
     const int64_t t = v * V;
     float acc[V];
     fold_vector<T, COMPAT>(g, src, p.N, t, acc, p.compat, p.r);
@@ -347,8 +355,8 @@ __global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams
     }
   }
   const int64_t tail0 = nvec * V;                                    // ragged tail (< V elements)
-  if (gid < g.n - tail0) {
-    const int64_t t = tail0 + gid;
+  if (tid0 < g.n - tail0) {
+    const int64_t t = tail0 + tid0;
     const float s = fold_scalar<T, COMPAT>(g, src, p.N, t, p.compat, p.r);
     if (g.out_partial) reinterpret_cast<float *>(g.out)[t] = s;
     else T::store1(g.out, t, post ? __fmul_rn(s, p.r) : s);
@@ -444,6 +452,13 @@ __global__ void __launch_bounds__(256) k_fold_tma(const __grid_constant__ FoldPa
   }
 }
 
+// ES_FOLD_CR=w (experiment): contiguous equal ranges per block in w whole
+// waves of resident blocks (0 = the one-shot grid, the default).
+int g_fold_cr = [] {
+  const char *e = std::getenv("ES_FOLD_CR");
+  return e ? std::atoi(e) : 0;
+}();
+
 int g_fold_tma = [] {
   const char *e = std::getenv("ES_FOLD_TMA");
   return e ? std::atoi(e) : 0;
@@ -457,6 +472,7 @@ cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSeg
   p.N = N;
   p.r = r;
   p.compat = compat;
+  p.contiguous = g_fold_cr ? 1 : 0;
   int nsrc = 0;
   std::vector<int64_t> work(nseg);
   for (int i = 0; i < nseg; ++i) {
@@ -479,6 +495,16 @@ cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSeg
   int64_t vecs = 0;
   for (int i = 0; i < nseg; ++i) vecs += (d[i].n + T::kVec - 1) / T::kVec;
   int total = (int)std::min<int64_t>((vecs + threads - 1) / threads, (int64_t)kMaxBlocks);
+  if (p.contiguous && bo == 0) {     // whole waves of resident blocks, `g_fold_cr` waves at least
+    static int resident = 0;
+    if (!resident) {
+      int per_sm = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fold<T, MAXSEG, MAXSRC, false>, threads, 0);
+      resident = std::max(1, per_sm) * kSMs;
+    }
+    const int64_t waves = std::max<int64_t>(1, std::min<int64_t>((total + resident - 1) / resident, g_fold_cr));
+    total = (int)(waves * resident);
+  }
   if (bo > 0) total = bo;
   total = std::max(total, nseg);
   std::vector<int32_t> block0;
