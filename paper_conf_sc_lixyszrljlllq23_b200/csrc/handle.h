@@ -75,6 +75,10 @@ struct es_ctx {
   es_status sticky = ES_OK;
   std::string sticky_msg;
 
+  // graph capture: node of our last stash launch (early-start proof)
+  cudaGraphNode_t last_stash_node = nullptr;
+  unsigned long long last_stash_cap = 0;
+
   // NEXT-1 incremental fold: next EST expected per bucket (0: none folded yet)
   std::vector<int32_t> inc_next;
 

@@ -49,6 +49,16 @@ bool g_pdl = [] {
   return !(e && e[0] == '1');
 }();
 
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
+// ES_STASH_EARLY=0 disables the early start of stash kernels (see
+// launch_stash_multi); it is on by default where the host proves it safe.
+bool g_stash_early_ok = [] {
+  const char *e = std::getenv("ES_STASH_EARLY");
+  return !(e && e[0] == '0');
+}();
+
 __device__ __forceinline__ void pdl_enter() {
   asm volatile("griddepcontrol.wait;" ::: "memory");             // predecessor complete + visible
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");  // successor may become resident
@@ -612,6 +622,7 @@ struct StashSeg {
 template <int MAXSEG>
 struct StashParams {
   int32_t nseg, nblocks;
+  int32_t early;              // 1: start before the predecessor completes (see launch_stash_multi)
   // fused context swap: blocks [0, swap_bx * swap_n) swap, the rest stash
   const SwapEntry *swap_tab;
   int32_t swap_n, swap_bx, swap_cur, swap_next;
@@ -651,9 +662,11 @@ template <typename S, typename D, int E, int kU, int MAXSEG, int ST, bool CR = f
 __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashParams<MAXSEG> p) {
   using In = typename VecT<S::kSize * E>::T;
   using Out = typename VecT<D::kSize * E>::T;
-  pdl_enter();
+  if (p.early) pdl_trigger();
+  else pdl_enter();
   const int nswap = p.swap_bx * p.swap_n;
   if ((int)blockIdx.x < nswap) {
+    if (p.early) pdl_wait();
     swap_entry(p.swap_tab, (int)blockIdx.x / p.swap_bx, (int)blockIdx.x % p.swap_bx, p.swap_bx, p.swap_cur,
                p.swap_next);
     return;
@@ -702,17 +715,19 @@ __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashPara
       D::store1(g.dst, i, S::load1(g.src, i));
     }
   }
+  if (p.early) pdl_wait();   // complete only after the predecessor: keeps completion order transitive
 }
 
 template <typename S, typename D, int E, int kU, int ST, bool CR = false>
 cudaError_t launch_stash_v(const StashSegDesc *segs, int nseg, cudaStream_t s, int bo, int to, int *launches,
-                           const SwapArgs *swap) {
+                           const SwapArgs *swap, bool early) {
   constexpr int kMaxSeg = 32;
   const int threads = to > 0 ? to : 256;
   for (int i = 0; i < nseg; i += kMaxSeg) {
     const int k = std::min(kMaxSeg, nseg - i);
     StashParams<kMaxSeg> p;
     p.nseg = k;
+    p.early = early && g_stash_early_ok && i == 0 ? 1 : 0;
     const bool fuse = i == 0 && swap && swap->n > 0;
     p.swap_tab = fuse ? swap->tab : nullptr;
     p.swap_n = fuse ? swap->n : 0;
@@ -765,15 +780,15 @@ int g_stash_variant = [] {
 
 template <typename S, typename D, int E>
 cudaError_t launch_stash_t(const StashSegDesc *segs, int nseg, cudaStream_t s, int bo, int to, int *launches,
-                           const SwapArgs *swap) {
+                           const SwapArgs *swap, bool early) {
   switch (g_stash_variant) {
-    case 1: return launch_stash_v<S, D, E, 8, 0>(segs, nseg, s, bo, to, launches, swap);
-    case 2: return launch_stash_v<S, D, E, 2, 0>(segs, nseg, s, bo, to, launches, swap);
-    case 3: return launch_stash_v<S, D, E, 4, 1>(segs, nseg, s, bo, to, launches, swap);
-    case 4: return launch_stash_v<S, D, E, 1, 0>(segs, nseg, s, bo, to, launches, swap);
-    case 5: return launch_stash_v<S, D, E, 4, 0>(segs, nseg, s, bo, to, launches, swap);   // one-shot grid
-    case 6: return launch_stash_v<S, D, E, 8, 0, true>(segs, nseg, s, bo, to, launches, swap);
-    default: return launch_stash_v<S, D, E, 4, 0, true>(segs, nseg, s, bo, to, launches, swap);
+    case 1: return launch_stash_v<S, D, E, 8, 0>(segs, nseg, s, bo, to, launches, swap, early);
+    case 2: return launch_stash_v<S, D, E, 2, 0>(segs, nseg, s, bo, to, launches, swap, early);
+    case 3: return launch_stash_v<S, D, E, 4, 1>(segs, nseg, s, bo, to, launches, swap, early);
+    case 4: return launch_stash_v<S, D, E, 1, 0>(segs, nseg, s, bo, to, launches, swap, early);
+    case 5: return launch_stash_v<S, D, E, 4, 0>(segs, nseg, s, bo, to, launches, swap, early);   // one-shot grid
+    case 6: return launch_stash_v<S, D, E, 8, 0, true>(segs, nseg, s, bo, to, launches, swap, early);
+    default: return launch_stash_v<S, D, E, 4, 0, true>(segs, nseg, s, bo, to, launches, swap, early);
   }
 }
 
@@ -1060,7 +1075,7 @@ cudaError_t launch_fold_multi(es_dtype dtype, int32_t N, float r, uint32_t compa
 }
 
 cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *segs, int nseg, cudaStream_t s,
-                               int bo, int to, int *launches, const SwapArgs *swap) {
+                               int bo, int to, int *launches, const SwapArgs *swap, bool early) {
   int dummy = 0;
   if (!launches) launches = &dummy;
   std::vector<StashSegDesc> live;
@@ -1079,12 +1094,12 @@ cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *s
     return g_stash_tma == 1 ? launch_copy_tma<4, 32768>(live.data(), n, es_, s, 1, launches)
                             : launch_copy_tma<6, 16384>(live.data(), n, es_, s, 2, launches);
   }
-  if (sdt == ES_F32 && ddt == ES_F32) return launch_stash_t<F32T, F32T, 4>(live.data(), n, s, bo, to, launches, swap);
+  if (sdt == ES_F32 && ddt == ES_F32) return launch_stash_t<F32T, F32T, 4>(live.data(), n, s, bo, to, launches, swap, early);
   if (sdt == ES_BF16 && ddt == ES_BF16)
-    return launch_stash_t<BF16T, BF16T, 8>(live.data(), n, s, bo, to, launches, swap);
+    return launch_stash_t<BF16T, BF16T, 8>(live.data(), n, s, bo, to, launches, swap, early);
   if (sdt == ES_F32 && ddt == ES_BF16)
-    return launch_stash_t<F32T, BF16T, 4>(live.data(), n, s, bo, to, launches, swap);
-  return launch_stash_t<BF16T, F32T, 4>(live.data(), n, s, bo, to, launches, swap);
+    return launch_stash_t<F32T, BF16T, 4>(live.data(), n, s, bo, to, launches, swap, early);
+  return launch_stash_t<BF16T, F32T, 4>(live.data(), n, s, bo, to, launches, swap, early);
 }
 
 cudaError_t launch_dropout(es_dtype dtype, const void *x, void *y, uint8_t *mask, int64_t n, float p, float scale,

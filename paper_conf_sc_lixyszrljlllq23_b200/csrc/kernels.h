@@ -66,9 +66,13 @@ struct SwapArgs {
 // If `swap` has entries, its blocks ride in the first stash launch (the
 // outgoing EST's stash and the context switch are independent), saving one
 // launch per context switch.
+// early: the caller has proven that the kernel immediately preceding this
+// launch on `s` is one of our stash kernels (independent data), so the copy
+// blocks may start while it is still running -- they wait for it only before
+// exiting (completion order stays transitive); swap blocks always wait first.
 cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *segs, int nseg, cudaStream_t s,
                                int blocks_override, int threads_override, int *launches,
-                               const SwapArgs *swap = nullptr);
+                               const SwapArgs *swap = nullptr, bool early = false);
 
 // One launch: for every entry, slot[cur] <- live, live <- slot[next]
 // (cur < 0: load only).  max_nbytes sizes the grid.
