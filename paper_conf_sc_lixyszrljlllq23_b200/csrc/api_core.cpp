@@ -204,6 +204,7 @@ es_status es_switch_context(es_handle h, int32_t est, es_stream stream) {
                    return es::launch_swap(tab, n, h->max_state, cur, li, cs);
                  });
     if (s != ES_OK) return s;
+    remember_stash_node(h, cs);      // a following stash may start early (independent data)
   }
   h->cur_local = li;
   return ES_OK;

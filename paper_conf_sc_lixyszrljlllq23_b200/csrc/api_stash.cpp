@@ -10,43 +10,6 @@ extern "C" {
 
 namespace {
 
-// Early start of a stash kernel is safe only when the kernel immediately
-// before it on the stream is one of our own stash kernels (independent
-// data).  That is provable only inside a CUDA-graph capture: the stream's
-// capture dependencies must be exactly the node of our previous stash launch
-// (no foreign kernel, event wait or timing node in between).  Eager launches
-// never start early.
-bool follows_own_stash(es_handle h, cudaStream_t cs) {
-  cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
-  unsigned long long id = 0;
-  cudaGraph_t g = nullptr;
-  const cudaGraphNode_t *deps = nullptr;
-  size_t nd = 0;
-  if (cudaStreamGetCaptureInfo(cs, &st, &id, &g, &deps, &nd) != cudaSuccess) {
-    cudaGetLastError();
-    return false;
-  }
-  return st == cudaStreamCaptureStatusActive && nd == 1 && h->last_stash_node && deps[0] == h->last_stash_node &&
-         id == h->last_stash_cap;
-}
-
-void remember_stash_node(es_handle h, cudaStream_t cs) {
-  cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
-  unsigned long long id = 0;
-  cudaGraph_t g = nullptr;
-  const cudaGraphNode_t *deps = nullptr;
-  size_t nd = 0;
-  h->last_stash_node = nullptr;
-  if (cudaStreamGetCaptureInfo(cs, &st, &id, &g, &deps, &nd) != cudaSuccess) {
-    cudaGetLastError();
-    return;
-  }
-  if (st == cudaStreamCaptureStatusActive && nd == 1 && !h->prof) {
-    h->last_stash_node = deps[0];
-    h->last_stash_cap = id;
-  }
-}
-
 // Stash of `n` buckets of local EST `est`, optionally fused with a context
 // switch to local EST `next_est` (-1: no switch) in the same launch.
 es_status stash_impl(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,

@@ -161,3 +161,40 @@ inline es_status check_handle(es_handle h) {
   if (!h) return set_err(ES_EINVAL, "handle is NULL");
   return h->check_sticky();
 }
+
+// Early start of a stash kernel is safe only when the kernel immediately
+// before it on the stream is one of our own stash or switch kernels
+// (independent data; the fused swap blocks still wait).  That is provable only inside a CUDA-graph capture: the stream's
+// capture dependencies must be exactly the node of our previous stash launch
+// (no foreign kernel, event wait or timing node in between).  Eager launches
+// never start early.
+inline bool follows_own_stash(es_handle h, cudaStream_t cs) {
+  cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+  unsigned long long id = 0;
+  cudaGraph_t g = nullptr;
+  const cudaGraphNode_t *deps = nullptr;
+  size_t nd = 0;
+  if (cudaStreamGetCaptureInfo(cs, &st, &id, &g, &deps, &nd) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return st == cudaStreamCaptureStatusActive && nd == 1 && h->last_stash_node && deps[0] == h->last_stash_node &&
+         id == h->last_stash_cap;
+}
+
+inline void remember_stash_node(es_handle h, cudaStream_t cs) {
+  cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+  unsigned long long id = 0;
+  cudaGraph_t g = nullptr;
+  const cudaGraphNode_t *deps = nullptr;
+  size_t nd = 0;
+  h->last_stash_node = nullptr;
+  if (cudaStreamGetCaptureInfo(cs, &st, &id, &g, &deps, &nd) != cudaSuccess) {
+    cudaGetLastError();
+    return;
+  }
+  if (st == cudaStreamCaptureStatusActive && nd == 1 && !h->prof) {
+    h->last_stash_node = deps[0];
+    h->last_stash_cap = id;
+  }
+}
