@@ -210,7 +210,6 @@ struct FoldParams {
   int32_t nseg, N, nblocks;
   float r;
   uint32_t compat;        // NEXT-3 variant bits (COMPAT kernels only)
-  int32_t contiguous;     // 1: each block folds one contiguous, equal range of its segment
   FoldSeg seg[MAXSEG];
   const void *src[MAXSRC];
 };
@@ -338,15 +337,8 @@ __global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams
   const void *const *src = p.src + g.src0;
   const int64_t nvec = g.n / V;
   const int64_t tid0 = (int64_t)(blockIdx.x - g.block0) * blockDim.x + threadIdx.x;
-  int64_t stride = (int64_t)nb * blockDim.x, gid = tid0, vend = nvec;
-  if (p.contiguous) {
-    const int64_t per = ((nvec + nb - 1) / nb + blockDim.x - 1) / blockDim.x * blockDim.x;
-    const int64_t vb = min(nvec, (int64_t)(blockIdx.x - g.block0) * per);
-    vend = min(nvec, vb + per);
-    stride = blockDim.x;
-    gid = vb + threadIdx.x;
-  }
-  for (int64_t v = gid; v < vend; v += stride) {
+  const int64_t stride = (int64_t)nb * blockDim.x;
+  for (int64_t v = tid0; v < nvec; v += stride) {
     const int64_t t = v * V;
     float acc[V];
     fold_vector<T, COMPAT>(g, src, p.N, t, acc, p.compat, p.r);
@@ -462,13 +454,6 @@ __global__ void __launch_bounds__(256) k_fold_tma(const __grid_constant__ FoldPa
   }
 }
 
-// ES_FOLD_CR=w (experiment): contiguous equal ranges per block in w whole
-// waves of resident blocks (0 = the one-shot grid, the default).
-int g_fold_cr = [] {
-  const char *e = std::getenv("ES_FOLD_CR");
-  return e ? std::atoi(e) : 0;
-}();
-
 int g_fold_tma = [] {
   const char *e = std::getenv("ES_FOLD_TMA");
   return e ? std::atoi(e) : 0;
@@ -482,7 +467,6 @@ cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSeg
   p.N = N;
   p.r = r;
   p.compat = compat;
-  p.contiguous = g_fold_cr ? 1 : 0;
   int nsrc = 0;
   std::vector<int64_t> work(nseg);
   for (int i = 0; i < nseg; ++i) {
@@ -505,16 +489,6 @@ cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSeg
   int64_t vecs = 0;
   for (int i = 0; i < nseg; ++i) vecs += (d[i].n + T::kVec - 1) / T::kVec;
   int total = (int)std::min<int64_t>((vecs + threads - 1) / threads, (int64_t)kMaxBlocks);
-  if (p.contiguous && bo == 0) {     // whole waves of resident blocks, `g_fold_cr` waves at least
-    static int resident = 0;
-    if (!resident) {
-      int per_sm = 0;
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fold<T, MAXSEG, MAXSRC, false>, threads, 0);
-      resident = std::max(1, per_sm) * kSMs;
-    }
-    const int64_t waves = std::max<int64_t>(1, std::min<int64_t>((total + resident - 1) / resident, g_fold_cr));
-    total = (int)(waves * resident);
-  }
   if (bo > 0) total = bo;
   total = std::max(total, nseg);
   std::vector<int32_t> block0;
@@ -769,10 +743,11 @@ cudaError_t launch_stash_v(const StashSegDesc *segs, int nseg, cudaStream_t s, i
 }
 
 // ES_STASH_VARIANT (measured in profiles/r01_stash_variants.md):
-// 0 (default) = one contiguous, equal range per block, whole waves of
-// resident blocks, 4 units per thread in flight; 5 = the one-shot grid
-// (~1 iteration per thread); 1 / 2 / 4 = one-shot with 8 / 2 / 1 units;
-// 3 = one-shot with cache-streaming stores; 6 = contiguous ranges, 8 units.
+// 0 (default) = one-shot grid, ~1 iteration of 4 units per thread (40 regs);
+// 5 = one contiguous, equal range per block in whole waves of resident
+// blocks (59 regs; +2.4 % alone, but -0.8 % once consecutive stashes
+// overlap through the early start); 1 / 2 / 4 = one-shot with 8 / 2 / 1
+// units; 3 = one-shot with cache-streaming stores; 6 = contiguous, 8 units.
 int g_stash_variant = [] {
   const char *e = std::getenv("ES_STASH_VARIANT");
   return e ? std::atoi(e) : 0;
@@ -786,9 +761,9 @@ cudaError_t launch_stash_t(const StashSegDesc *segs, int nseg, cudaStream_t s, i
     case 2: return launch_stash_v<S, D, E, 2, 0>(segs, nseg, s, bo, to, launches, swap, early);
     case 3: return launch_stash_v<S, D, E, 4, 1>(segs, nseg, s, bo, to, launches, swap, early);
     case 4: return launch_stash_v<S, D, E, 1, 0>(segs, nseg, s, bo, to, launches, swap, early);
-    case 5: return launch_stash_v<S, D, E, 4, 0>(segs, nseg, s, bo, to, launches, swap, early);   // one-shot grid
+    case 5: return launch_stash_v<S, D, E, 4, 0, true>(segs, nseg, s, bo, to, launches, swap, early);
     case 6: return launch_stash_v<S, D, E, 8, 0, true>(segs, nseg, s, bo, to, launches, swap, early);
-    default: return launch_stash_v<S, D, E, 4, 0, true>(segs, nseg, s, bo, to, launches, swap, early);
+    default: return launch_stash_v<S, D, E, 4, 0>(segs, nseg, s, bo, to, launches, swap, early);
   }
 }
 
