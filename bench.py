@@ -463,15 +463,27 @@ def main():
         h2d = len(local) * sum(n for n, _ in buckets) * esz
         d2h = sum(n for n, _ in buckets) * esz
 
+        # The result's D2H runs on its own stream (PCIe is full duplex), overlapping the next step's H2D;
+        # the next aggregation waits for it before overwriting `outs`.
+        d2h_stream = torch.cuda.Stream(device=dev)
+        d2h_done = torch.cuda.Event()
+        d2h_done.record(d2h_stream)
+
         def e2e_step():
             for i, k in enumerate(local):
                 for b in range(B):
                     live_grad[b].copy_(host[k][b], non_blocking=True)     # "backward" lands in the live buffer
                 agg.switch(k)
                 agg.stash_many(k, range(B), live_grad, es.ES_STASH_BORROW if i == len(local) - 1 else es.ES_STASH_COPY)
+            stream.wait_event(d2h_done)
             agg.allreduce_many(range(B), outs)
-            for b in range(B):
-                host_out[b].copy_(outs[b], non_blocking=True)
+            ready = torch.cuda.Event()
+            ready.record(stream)
+            d2h_stream.wait_event(ready)
+            with torch.cuda.stream(d2h_stream):
+                for b in range(B):
+                    host_out[b].copy_(outs[b], non_blocking=True)
+            d2h_done.record(d2h_stream)
 
         k_e2e = max(3, min(args.steps, 10))
         with torch.cuda.stream(stream):
@@ -484,6 +496,7 @@ def main():
             e0.record(stream)
             for _ in range(k_e2e):
                 e2e_step()
+            stream.wait_event(d2h_done)                   # the last result is on the host
             e1.record(stream)
         torch.cuda.synchronize()
         ems = e0.elapsed_time(e1) / k_e2e
