@@ -412,6 +412,12 @@ def main():
                    if flush is None else "L2 flushed between timed steps (512 MB write)"},
         "roofline": dominant,
         "roofline_by_kernel": roofs,
+        # the whole step against the same peak: every kernel's algorithmic bytes of one step divided by
+        # the UNPROFILED step time (per-kernel event pairs above add ~1-5 us per launch; this has none)
+        "step_roofline": {"achieved": round(sum(v[2] for v in prof.values()) / steps_profiled / (ms / 1e3) / 1e9, 1),
+                          "peak": peak, "unit": "GB/s",
+                          "frac": round(sum(v[2] for v in prof.values()) / steps_profiled / (ms / 1e3) / 1e9 / peak, 4),
+                          "bytes_per_step": int(sum(v[2] for v in prof.values()) / steps_profiled)},
         "breakdown_ms_per_step": {k: round(v[1] / steps_profiled, 4) for k, v in prof.items()},
         "per_kernel": {k: {"launches_per_step": int(v[0] / steps_profiled),
                            "algorithmic_GBps": round(v[2] / (v[1] / 1e3) / 1e9, 1) if v[1] > 0 else None,

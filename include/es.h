@@ -117,6 +117,8 @@ typedef enum {
  *             NCCL reduction, whose order is not the canonical one.  libnccl is
  *             resolved at es_init from the copy already loaded in the process
  *             (dlopen RTLD_NOLOAD "libnccl.so.2"), else dlopen'ed by name.
+ *             With G == 1 a non-NULL comm is only validated (size 1, rank 0;
+ *             ES_ENCCL otherwise) and never used.
  *   LOOPBACK: `comm` is an es_loopback world (es_loopback_create); all G ranks
  *             live in ONE process, each driven by its own host thread, all
  *             on the same device; bytes move with cudaMemcpyAsync.  Test

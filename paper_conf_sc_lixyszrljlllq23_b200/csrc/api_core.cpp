@@ -102,6 +102,11 @@ es_status es_init(const es_config *cfg, void *workspace, size_t workspace_bytes,
                            : es::make_loopback_transport(h->plan.comm, h->plan.G, h->plan.rank, &err);
     if (!t) return set_err(h->plan.transport == ES_TRANSPORT_NCCL ? ES_ENCCL : ES_EINVAL, err);
     h->tp.reset(t);
+  } else if (h->plan.transport == ES_TRANSPORT_NCCL && h->plan.comm) {
+    // G == 1 needs no exchange, but a communicator that was passed must still
+    // be a size-1 NCCL comm of this rank (catches a wrong pointer early).
+    std::unique_ptr<es::Transport> t(es::make_nccl_transport(h->plan.comm, 1, h->plan.rank, &err));
+    if (!t) return set_err(ES_ENCCL, err);
   }
   *out = h.release();
   return ES_OK;
