@@ -16,11 +16,9 @@ es_status peer_barrier(es_handle h, cudaStream_t cs) {
   const es::Plan &p = h->plan;
   std::vector<uint64_t *> pf(p.G);
   for (int32_t g = 0; g < p.G; ++g) pf[g] = reinterpret_cast<uint64_t *>(h->peer_ws[g] + p.flags_off);
-  const uint64_t epoch = ++h->barrier_epoch;
   return h->timed(ES_KERNEL_BARRIER, 0, cs, [&](int *nl) {
     *nl = 1;
-    return es::launch_peer_barrier(pf.data(), reinterpret_cast<uint64_t *>(h->ws + p.flags_off), p.G, p.rank, epoch,
-                                   cs);
+    return es::launch_peer_barrier(pf.data(), reinterpret_cast<uint64_t *>(h->ws + p.flags_off), p.G, p.rank, cs);
   });
 }
 

@@ -93,9 +93,20 @@ es_status es_init(const es_config *cfg, void *workspace, size_t workspace_bytes,
     if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
       return set_err(ES_ECUDA, "cudaEventCreate failed");
   for (uint64_t n : h->plan.state_nbytes) h->max_state = std::max<uint64_t>(h->max_state, n);
-  if (cudaMemset(h->ws + h->plan.scratch_off, 0, 256) != cudaSuccess) return set_err(ES_ECUDA, "cudaMemset failed");
-  if (h->plan.peer && cudaMemset(h->ws + h->plan.flags_off, 0, 64 * 8) != cudaSuccess)
-    return set_err(ES_ECUDA, "cudaMemset of the peer flags failed");
+  {
+    // Zero the scratch words and the peer flags + epoch counter on a private
+    // stream and wait for it: peers may write these flags as soon as they hold
+    // this rank's peer blob, and other ranks' work on shared streams must not
+    // be waited for (loopback ranks initialise concurrently).
+    cudaStream_t zs = nullptr;
+    if (cudaStreamCreateWithFlags(&zs, cudaStreamNonBlocking) != cudaSuccess)
+      return set_err(ES_ECUDA, "cudaStreamCreate failed");
+    bool ok = cudaMemsetAsync(h->ws + h->plan.scratch_off, 0, 256, zs) == cudaSuccess;
+    if (ok && h->plan.peer) ok = cudaMemsetAsync(h->ws + h->plan.flags_off, 0, es::kPeerFlagWords * 8, zs) == cudaSuccess;
+    ok = cudaStreamSynchronize(zs) == cudaSuccess && ok;
+    cudaStreamDestroy(zs);
+    if (!ok) return set_err(ES_ECUDA, "cudaMemsetAsync of the workspace scratch / peer flags failed");
+  }
   if (h->plan.G > 1 && h->plan.transport != ES_TRANSPORT_NONE) {
     es::Transport *t = h->plan.transport == ES_TRANSPORT_NCCL
                            ? es::make_nccl_transport(h->plan.comm, h->plan.G, h->plan.rank, &err)

@@ -75,6 +75,10 @@ es_status es_peer_open(es_handle h, const void *blobs, size_t bytes) {
   const es::Plan &p = h->plan;
   if (!blobs || bytes < (size_t)p.G * ES_PEER_BLOB_BYTES) return set_err(ES_EINVAL, "need G blobs");
   if (h->peer_open) return set_err(ES_ESTATE, "peers already open");
+  // Peer schedules spin in device barriers: load every kernel now, not on
+  // first use (a lazy load waits behind a spinning same-device barrier).
+  if (cudaError_t e = es::preload_kernels(); e != cudaSuccess)
+    return set_err(ES_ECUDA, std::string("loading the kernels failed: ") + cudaGetErrorString(e));
   std::vector<unsigned char *> ws(p.G, nullptr);
   std::vector<void *> mapped;
   const int32_t me = (int32_t)getpid();

@@ -86,7 +86,6 @@ struct es_ctx {
   std::vector<unsigned char *> peer_ws;   // [G] workspace base of every rank, mapped here
   std::vector<void *> ipc_mapped;         // cudaIpcOpenMemHandle results to close
   bool peer_open = false;
-  uint64_t barrier_epoch = 0;
 
   // instrumentation
   bool prof = false;

@@ -100,6 +100,20 @@ __device__ __forceinline__ uint32_t smem_addr(const void *p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
+// Every kernel instantiation a launch site can reach registers its host stub
+// when libes is loaded, so preload_kernels() can make CUDA's lazy loader
+// (CUDA_MODULE_LOADING=LAZY, the CUDA 12 default) load them all up front: a
+// first-use load cannot complete while another rank's barrier kernel spins on
+// the same device, which deadlocks same-device peer ranks.
+std::vector<const void *> &kernel_registry() {
+  static std::vector<const void *> r;
+  return r;
+}
+template <auto F>
+struct KernelReg {
+  static inline const bool token = (kernel_registry().push_back(reinterpret_cast<const void *>(F)), true);
+};
+
 template <typename K, typename P>
 cudaError_t launch(K kernel, dim3 grid, dim3 block, cudaStream_t s, const P &params) {
   cudaLaunchConfig_t cfg = {};
@@ -114,6 +128,12 @@ cudaError_t launch(K kernel, dim3 grid, dim3 block, cudaStream_t s, const P &par
   cfg.numAttrs = g_pdl ? 1 : 0;
   cudaError_t e = cudaLaunchKernelEx(&cfg, kernel, params);
   return e != cudaSuccess ? e : cudaGetLastError();
+}
+
+template <auto F, typename P>
+cudaError_t launch_k(dim3 grid, dim3 block, cudaStream_t s, const P &params) {
+  (void)KernelReg<F>::token;
+  return launch(F, grid, block, s, params);
 }
 
 // Block -> segment: the last segment whose first block is <= b.
@@ -521,11 +541,12 @@ cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSeg
     at[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = at;
     cfg.numAttrs = g_pdl ? 1 : 0;
+    (void)KernelReg<k_fold_tma<T, MAXSEG, MAXSRC, kS>>::token;
     cudaError_t e = cudaLaunchKernelEx(&cfg, k_fold_tma<T, MAXSEG, MAXSRC, kS>, p);
     return e != cudaSuccess ? e : cudaGetLastError();
   }
-  if (compat) return launch(k_fold<T, MAXSEG, MAXSRC, true>, dim3(p.nblocks), dim3(threads), s, p);
-  return launch(k_fold<T, MAXSEG, MAXSRC, false>, dim3(p.nblocks), dim3(threads), s, p);
+  if (compat) return launch_k<k_fold<T, MAXSEG, MAXSRC, true>>(dim3(p.nblocks), dim3(threads), s, p);
+  return launch_k<k_fold<T, MAXSEG, MAXSRC, false>>(dim3(p.nblocks), dim3(threads), s, p);
 }
 
 template <typename T>
@@ -735,7 +756,7 @@ cudaError_t launch_stash_v(const StashSegDesc *segs, int nseg, cudaStream_t s, i
     split_blocks(work, total, &block0, &p.nblocks);
     for (int j = 0; j < k; ++j) p.seg[j].block0 = block0[j];
     const int grid = p.nblocks + p.swap_bx * p.swap_n;
-    cudaError_t e = launch(k_stash<S, D, E, kU, kMaxSeg, ST, CR>, dim3(grid), dim3(threads), s, p);
+    cudaError_t e = launch_k<k_stash<S, D, E, kU, kMaxSeg, ST, CR>>(dim3(grid), dim3(threads), s, p);
     if (e != cudaSuccess) return e;
     ++*launches;
   }
@@ -902,6 +923,7 @@ cudaError_t launch_copy_tma(const StashSegDesc *segs, int nseg, int esize, cudaS
     at[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = at;
     cfg.numAttrs = g_pdl ? 1 : 0;
+    (void)KernelReg<k_copy_tma<S, T>>::token;
     cudaError_t e = cudaLaunchKernelEx(&cfg, k_copy_tma<S, T>, p);
     if (e == cudaSuccess) e = cudaGetLastError();
     if (e != cudaSuccess) return e;
@@ -996,7 +1018,7 @@ struct BarrierParams {
   uint64_t *peer_flags[64];
   uint64_t *my_flags;
   int32_t G, rank;
-  uint64_t epoch;
+  uint64_t timeout_ns;
 };
 
 __global__ void __launch_bounds__(64) k_peer_barrier(const __grid_constant__ BarrierParams p) {
@@ -1006,10 +1028,13 @@ __global__ void __launch_bounds__(64) k_peer_barrier(const __grid_constant__ Bar
   // loopback transport).
   asm volatile("griddepcontrol.wait;" ::: "memory");
   const int t = threadIdx.x;
+  // Every rank runs the same sequence of barriers, so the device-resident
+  // counters advance in lockstep, eager or replayed from a CUDA graph.
+  const uint64_t epoch = p.my_flags[kEpochSlot] + 1;
   __threadfence_system();                       // this GPU's completed writes before the arrival
   if (t < p.G) {
     uint64_t *dst = p.peer_flags[t] + p.rank;
-    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(dst), "l"(p.epoch) : "memory");
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(dst), "l"(epoch) : "memory");
   }
   if (t < p.G) {
     const uint64_t *src = p.my_flags + t;
@@ -1017,13 +1042,14 @@ __global__ void __launch_bounds__(64) k_peer_barrier(const __grid_constant__ Bar
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
     do {
       asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(src) : "memory");
-      if (v >= p.epoch) break;
+      if (v >= epoch) break;
       __nanosleep(256);
       asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now));
-      if (now - t0 > 60ull * 1000000000ull) __trap();   // a peer never arrived: fail loudly, never hang the GPU
+      if (now - t0 > p.timeout_ns) __trap();   // a peer never arrived: fail loudly, never hang the GPU
     } while (true);
   }
   __syncthreads();
+  if (t == 0) p.my_flags[kEpochSlot] = epoch;   // read back only by this rank's next barrier
   __threadfence_system();
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
@@ -1031,6 +1057,17 @@ __global__ void __launch_bounds__(64) k_peer_barrier(const __grid_constant__ Bar
 }  // namespace
 
 void set_pdl(bool on) { g_pdl = on; }
+
+cudaError_t preload_kernels() {
+  for (const void *f : kernel_registry()) {
+    cudaFuncAttributes a;
+    cudaError_t e = cudaFuncGetAttributes(&a, f);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
+size_t registered_kernels() { return kernel_registry().size(); }
 
 cudaError_t launch_fold_multi(es_dtype dtype, int32_t N, float r, uint32_t compat, const FoldSegDesc *segs, int nseg,
                               cudaStream_t s, int blocks_override, int threads_override, int *launches) {
@@ -1082,27 +1119,32 @@ cudaError_t launch_dropout(es_dtype dtype, const void *x, void *y, uint8_t *mask
   DropoutParams d{x, y, mask, n, p, scale, record, counter};
   const int64_t nq = std::max<int64_t>((n + 3) / 4, 1);
   const int blocks = (int)std::min<int64_t>((nq + 255) / 256, (int64_t)kSMs * 16);
-  if (dtype == ES_BF16) return launch(k_dropout<BF16T>, dim3(blocks), dim3(256), s, d);
-  return launch(k_dropout<F32T>, dim3(blocks), dim3(256), s, d);
+  if (dtype == ES_BF16) return launch_k<k_dropout<BF16T>>(dim3(blocks), dim3(256), s, d);
+  return launch_k<k_dropout<F32T>>(dim3(blocks), dim3(256), s, d);
 }
 
 cudaError_t launch_peer_barrier(uint64_t *const *peer_flags, uint64_t *my_flags, int32_t G, int32_t rank,
-                                uint64_t epoch, cudaStream_t s) {
+                                cudaStream_t s) {
   if (G < 1 || G > 64) return cudaErrorInvalidValue;
   BarrierParams b;
   for (int i = 0; i < 64; ++i) b.peer_flags[i] = i < G ? peer_flags[i] : nullptr;
   b.my_flags = my_flags;
   b.G = G;
   b.rank = rank;
-  b.epoch = epoch;
-  return launch(k_peer_barrier, dim3(1), dim3(64), s, b);
+  static const uint64_t timeout_ns = [] {
+    const char *e = getenv("ES_BARRIER_TIMEOUT_S");   // default 60 s
+    const double sec = e ? atof(e) : 60.0;
+    return (uint64_t)((sec > 0 ? sec : 60.0) * 1e9);
+  }();
+  b.timeout_ns = timeout_ns;
+  return launch_k<k_peer_barrier>(dim3(1), dim3(64), s, b);
 }
 
 cudaError_t launch_swap(const SwapEntry *table_dev, int32_t n, uint64_t max_nbytes, int32_t cur, int32_t next,
                         cudaStream_t s) {
   if (n <= 0) return cudaSuccess;
   SwapParams p{table_dev, cur, next};
-  return launch(k_swap, dim3(swap_blocks_per_entry(max_nbytes), (unsigned)n), dim3(256), s, p);
+  return launch_k<k_swap>(dim3(swap_blocks_per_entry(max_nbytes), (unsigned)n), dim3(256), s, p);
 }
 
 }  // namespace es

@@ -87,11 +87,20 @@ cudaError_t launch_swap(const SwapEntry *table_dev, int32_t n, uint64_t max_nbyt
 cudaError_t launch_dropout(es_dtype dtype, const void *x, void *y, uint8_t *mask, int64_t n, float p, float scale,
                            uint64_t *record, unsigned int *counter, cudaStream_t s);
 
-// PEER barrier: thread t < G publishes `epoch` into slot `rank` of peer t's
-// flag array (system-scope release) and then waits until this rank's own flag
-// array holds >= epoch in every slot (system-scope acquire).  One block.
+// PEER barrier: the epoch e = my_flags[kEpochSlot] + 1 lives in device memory
+// (so a CUDA-graph replay advances it); thread t < G publishes e into slot
+// `rank` of peer t's flag array (system-scope release) and then waits until
+// this rank's own flag array holds >= e in every slot (system-scope acquire).
+// One block.  my_flags has kPeerFlagWords u64 words, zeroed at es_init.
+constexpr int kEpochSlot = 64;
+constexpr int kPeerFlagWords = 65;
 cudaError_t launch_peer_barrier(uint64_t *const *peer_flags, uint64_t *my_flags, int32_t G, int32_t rank,
-                                uint64_t epoch, cudaStream_t s);
+                                cudaStream_t s);
+
+// Force-load every kernel instantiation libes can launch (see kernel_registry
+// in kernels.cu); called before any device-side spin-wait can run.
+cudaError_t preload_kernels();
+size_t registered_kernels();
 
 // Programmatic dependent launch (on by default; ES_NO_PDL=1 disables).
 void set_pdl(bool on);

@@ -7,6 +7,7 @@
 // Both schedules below realise exactly that order; they differ only in where
 // the partial sums live and how many bytes cross NVLink.
 #include "plan.h"
+#include "kernels.h"
 
 #include <algorithm>
 #include <cstring>
@@ -447,7 +448,7 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
   uint64_t head = 0;
   if (p->peer) {
     p->flags_off = 0;
-    p->result_off = align256(64 * 8);
+    p->result_off = align256(kPeerFlagWords * 8);   // G flags + the epoch counter
     head = p->result_off + p->slot_block;   // one bucket-layout block: shard results at bucket offsets
     p->peer_parts_off = head;               // PEER_CHAIN partials: per bucket, max over ranks
     head += align256(sum_peer_parts);

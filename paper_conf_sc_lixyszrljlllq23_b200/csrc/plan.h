@@ -72,7 +72,7 @@ struct Plan {
   uint64_t scratch_off = 0;             // 256 B of zeroed scratch (dropout grid counter)
   uint64_t stage_off = 0;               // exchange staging (max over buckets)
   uint64_t parts_off = 0;               // chain partials (max over buckets)
-  uint64_t flags_off = 0;               // PEER: G barrier flags (u64) written by peers
+  uint64_t flags_off = 0;               // PEER: G barrier flags (u64) written by peers + epoch counter
   uint64_t result_off = 0;              // PEER: per-bucket shard results (slot-block layout)
   uint64_t peer_parts_off = 0;          // PEER_CHAIN: partials read by the next GPU (uniform offset)
   bool peer = false;                    // some bucket uses ES_SCHED_PEER
