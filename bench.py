@@ -261,31 +261,45 @@ def main():
 
     fuse = not (args.per_bucket or args.no_fuse or args.incremental or args.inplace)
 
-    def step():
+    def step(marks=None):
+        # marks: three external CUDA events recorded at the phase boundaries
+        # (stashes start | stashes done | allreduce done) of one captured step
+        def mark(j):
+            if marks is not None:
+                marks[j].record(torch.cuda.current_stream())
         if args.inplace:
             agg.switch(local[0])
+            mark(0)
             for i, k in enumerate(local):
                 if i == len(local) - 1:
                     agg.stash_many(k, range(B), grads[k], es.ES_STASH_INPLACE)
                 else:
                     agg.stash_and_switch(k, range(B), grads[k], local[i + 1], es.ES_STASH_INPLACE)
+            mark(1)
             agg.allreduce_many(range(B), outs)
+            mark(2)
             return
         if args.incremental:
+            mark(0)
             for i, k in enumerate(local):
                 agg.switch(k)
                 agg.stash_fold(k, range(B), grads[k], es.ES_STASH_BORROW if i == len(local) - 1 else es.ES_STASH_COPY)
+            mark(1)
             agg.allreduce_many(range(B), outs)
+            mark(2)
             return
         if fuse:
             # switch-in of the first local EST, then per EST: stash its
             # buckets + switch to the next EST in one launch
             agg.switch(local[0])
+            mark(0)
             for i, k in enumerate(local):
                 if i == len(local) - 1:
                     agg.stash_many(k, range(B), grads[k], es.ES_STASH_BORROW)
                 else:
                     agg.stash_and_switch(k, range(B), grads[k], local[i + 1], es.ES_STASH_COPY)
+        if not fuse:
+            mark(0)
         for i, k in enumerate(local if not fuse else []):
             agg.switch(k)
             mode = es.ES_STASH_BORROW if i == len(local) - 1 else es.ES_STASH_COPY
@@ -294,11 +308,13 @@ def main():
                     agg.stash(k, b, grads[k][b], mode)
             else:
                 agg.stash_many(k, range(B), grads[k], mode)
+        mark(1)
         if args.per_bucket:
             for b in range(B):
                 agg.allreduce(b, outs[b])
         else:
             agg.allreduce_many(range(B), outs)
+        mark(2)
 
     use_graph = not args.no_graph
     stream = torch.cuda.Stream(device=dev)
@@ -306,14 +322,19 @@ def main():
         with torch.cuda.stream(stream):
             step()
     torch.cuda.synchronize()
-    graph = graph_prof = None
+    graph = graph_prof = graph_phase = None
+    marks = [torch.cuda.Event(enable_timing=True, external=use_graph) for _ in range(3)]
     if use_graph:
-        # Two captures of the same step: without timing events (the steps we
-        # time) and with per-kernel event nodes (the last timed step, which
-        # provides the kernel durations for the roofline).
+        # Three captures of the same step: without timing events (the steps we
+        # time), with phase-boundary events only (second-to-last timed step:
+        # stash and allreduce phases with every overlap intact), and with
+        # per-kernel event nodes (the last timed step: per-kind durations).
         graph = torch.cuda.CUDAGraph()
         with torch.cuda.graph(graph, stream=stream):
             step()
+        graph_phase = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph_phase, stream=stream):
+            step(marks)
         agg.profile(True)
         agg.profile_reset()
         graph_prof = torch.cuda.CUDAGraph()
@@ -350,9 +371,10 @@ def main():
                 flush.zero_()                     # L2 flush between timed steps (untimed)
             starts[i].record(stream)
             if graph is not None:
-                (graph_prof if i == args.steps - 1 else graph).replay()
+                g_ = graph_prof if i == args.steps - 1 else (graph_phase if i == args.steps - 2 else graph)
+                g_.replay()
             else:
-                step()
+                step(marks if i == args.steps - 2 else None)
             ends[i].record(stream)
     torch.cuda.synchronize()
     t_end = time.time()
@@ -385,16 +407,29 @@ def main():
         with open(tfile) as f:
             traffic_all = json.load(f)
 
+    # Phase timing (fused G=1 step only, where the stash phase holds nothing but stash kernels with
+    # their fused switches and the allreduce phase nothing but the fold): events at the phase
+    # boundaries of one timed step, no event between kernels, so early start and PDL overlap stay
+    # intact.  The per-kernel event pairs of the profiled step add ~1-5 us per launch.
+    phase_ms = None
+    if fuse and G == 1 and args.steps >= 2:
+        phase_ms = {"stash": marks[0].elapsed_time(marks[1]), "fold": marks[1].elapsed_time(marks[2])}
+
     def roof(kind, kname):
         n_, ms_, bytes_ = prof[kind]
         if n_ == 0 or ms_ <= 0:
             return None
-        a = bytes_ / (ms_ / 1e3) / 1e9
+        ev_us = ms_ / n_ * 1e3                                       # per-kernel event pairs
+        if phase_ms is not None and kind in phase_ms:
+            us, how = phase_ms[kind] * 1e3 / (n_ / steps_profiled), "phase events (no event between launches)"
+        else:
+            us, how = ev_us, "per-launch event pairs"
+        a = bytes_ / n_ / (us / 1e6) / 1e9
         return {"bound": "hbm", "kernel": kname, "achieved": round(a, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(a / peak, 4), "traffic": traffic_all.get(f"{kname}_dram_bytes_per_launch"),
                 "algorithmic_bytes_per_launch": int(bytes_ / n_), "launches_per_step": int(n_ / steps_profiled),
-                "avg_launch_us": round(ms_ / n_ * 1e3, 2), "share_of_step": round(ms_ / steps_profiled / ms, 3),
-                "peak_source": peak_src}
+                "avg_launch_us": round(us, 2), "timing": how, "avg_launch_us_event_pairs": round(ev_us, 2),
+                "share_of_step": round(us * n_ / steps_profiled / 1e3 / ms, 3), "peak_source": peak_src}
 
     roofs = {k: r for k, r in (("k_fold", roof("fold", "k_fold")), ("k_stash", roof("stash", "k_stash")),
                                ("k_gather", roof("gather", "k_gather"))) if r is not None}
