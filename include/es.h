@@ -99,9 +99,14 @@ typedef enum { ES_STASH_COPY = 0, ES_STASH_BORROW = 1, ES_STASH_INPLACE = 2 } es
 /*   PEER_CHAIN: the CHAIN schedule without a transport: the GPU of segment r
  *           of chunk c reads the incoming unrounded fp32 partial directly from
  *           the producer's workspace over NVLink inside its fold kernel (the
- *           partial's transfer and the local fold are one kernel); a device
- *           barrier separates rounds; chunk c is gathered from the RESULT area
- *           of the GPU of EST c.
+ *           partial's transfer and the local fold are one kernel).  By
+ *           default all rounds run as ONE tile-pipelined kernel per dtype:
+ *           the consumer of a partial starts on tile t as soon as the
+ *           producer has published tile t (per-tile flags in peer memory), so
+ *           the only device barriers are at the start and the end of the
+ *           step; ES_OPT_PEER_ROUNDS runs one fold launch per round with a
+ *           barrier between rounds instead (same bits).  Chunk c is gathered
+ *           from the RESULT area of the GPU of EST c.
  *   PEER_AUTO: per bucket PEER_CHAIN where CHAIN would move fewer bytes,
  *           else PEER (the AUTO rule over the peer-memory schedules). */
 typedef enum {
@@ -156,6 +161,9 @@ typedef struct {
 /* ES_OPT_INCREMENTAL: reserve fp32 partials so that es_stash_fold_grads can
  * fold each EST into the running partials at its switch (NEXT-1, G == 1). */
 #define ES_OPT_INCREMENTAL 1u
+/* ES_OPT_PEER_ROUNDS: PEER_CHAIN without tile pipelining (a device barrier
+ * between rounds).  Same bits; kept for comparison and as a fallback. */
+#define ES_OPT_PEER_ROUNDS 2u
 
 /* NEXT-3 compatibility variants -- same canonical order, different step
  * arithmetic:

@@ -30,6 +30,7 @@ es_status peer_barrier(es_handle h, cudaStream_t cs) {
 es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *const *outs, cudaStream_t cs, float r) {
   const es::Plan &p = h->plan;
   if (!h->peer_open) return set_err(ES_ESTATE, "peer-memory schedules need es_peer_open before es_allreduce");
+  const bool pipe = !(p.options & ES_OPT_PEER_ROUNDS) && p.compat == 0;
   es_status s;
   auto slot_of = [&](int32_t rank, int32_t e, int32_t b) {
     return h->peer_ws[rank] + p.grad_off + (uint64_t)p.owner_index[e] * p.slot_block + p.slot_off[b];
@@ -61,19 +62,29 @@ es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *c
     });
     if (s != ES_OK) return s;
   }
-  // 2. phases
+  // 2. phases.  Tile-pipelined (default): every bucket runs as three
+  //    phases -- [barrier] all folds (PEER: one shard fold; PEER_CHAIN: every
+  //    round in k_fold_pipe, ordered by per-tile flags) [barrier] gathers --
+  //    so a phase index is mapped: PEER_CHAIN folds of any round -> phase 1,
+  //    gathers -> phase 2.  Otherwise phase k = the ops after the k-th barrier.
   int32_t phases = 0;
   for (int32_t i = 0; i < n; ++i) {
     int32_t k = 0;
     for (const es::Op &op : p.bp[buckets[i]].ops) k += op.f[0] == ES_OP_BARRIER;
     phases = std::max(phases, k + 1);
   }
+  if (pipe) phases = std::min(phases, 3);
+  auto phase_of = [&](const es::BucketPlan &b, int32_t k, int64_t op) -> int32_t {
+    if (!pipe || b.sched != ES_SCHED_PEER_CHAIN) return k;
+    return op == ES_OP_GATHER ? 2 : 1;
+  };
   for (int32_t ph = 0; ph < phases; ++ph) {
     for (int dd = 0; dd < 2; ++dd) {
       std::vector<es::FoldSegDesc> folds;
       std::vector<std::vector<const void *>> srcs;
       std::vector<es::StashSegDesc> gathers;
-      uint64_t fbytes = 0, gbytes = 0;
+      std::vector<std::pair<int32_t, es::PipeSegDesc>> pipes;   // (round, segment)
+      uint64_t fbytes = 0, pbytes = 0, gbytes = 0;
       for (int32_t i = 0; i < n; ++i) {
         const int32_t bk = buckets[i];
         const es::BucketPlan &b = p.bp[bk];
@@ -86,7 +97,7 @@ es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *c
             ++k;
             continue;
           }
-          if (k != ph) continue;
+          if (phase_of(b, k, f[0]) != ph) continue;
           const int64_t lo = f[1], hi = f[2];
           if (f[0] == ES_OP_GATHER) {
             gathers.push_back({h->peer_ws[f[3]] + p.result_off + p.slot_off[bk] + (uint64_t)lo * esz,
@@ -121,16 +132,47 @@ es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *c
           d.out_partial = f[7] == ES_BUF_PART;
           d.out = d.out_partial ? (void *)(h->ws + p.peer_parts_off + b.peer_part_base + (uint64_t)f[8])
                                 : (void *)(h->ws + p.result_off + p.slot_off[bk] + (uint64_t)lo * esz);
-          fbytes += (uint64_t)d.n * ((uint64_t)src.size() * esz + (d.part_in ? 4 : 0) + (d.out_partial ? 4 : esz));
-          folds.push_back(d);
+          const uint64_t nbytes =
+              (uint64_t)d.n * ((uint64_t)src.size() * esz + (d.part_in ? 4 : 0) + (d.out_partial ? 4 : esz));
+          d.src = src.data();                     // the buffer survives the move below
           srcs.push_back(std::move(src));
+          if (pipe && b.sched == ES_SCHED_PEER_CHAIN) {
+            const int32_t rd = k - 1;                     // round of this segment
+            const uint64_t c = (uint64_t)lo / b.C;        // its chunk (segments span whole chunks)
+            auto flag = [&](unsigned char *base, int32_t round) {
+              return reinterpret_cast<uint64_t *>(base + p.pipe_flags_off) + b.pipe_flag_base +
+                     (c * (uint64_t)b.chain_rounds + (uint64_t)round) * b.tiles_per_chunk;
+            };
+            es::PipeSegDesc q;
+            q.f = d;
+            q.wait = d.part_in ? flag(h->peer_ws[f[6]], rd - 1) : nullptr;
+            q.pub = d.out_partial ? flag(h->ws, rd) : nullptr;
+            pipes.push_back({rd, q});
+            pbytes += nbytes;
+          } else {
+            folds.push_back(d);
+            fbytes += nbytes;
+          }
         }
       }
       if (!folds.empty()) {
-        for (size_t j = 0; j < folds.size(); ++j) folds[j].src = srcs[j].data();
         s = h->timed(ES_KERNEL_FOLD, fbytes, cs, [&](int *nl) {
           return es::launch_fold_multi((es_dtype)dd, p.N, r, p.compat, folds.data(), (int)folds.size(), cs,
                                        h->blocks_ov, h->threads_ov, nl);
+        });
+        if (s != ES_OK) return s;
+      }
+      if (!pipes.empty()) {
+        // round-major order across buckets: k_fold_pipe's forward-progress rule
+        std::stable_sort(pipes.begin(), pipes.end(), [](const auto &x, const auto &y) { return x.first < y.first; });
+        std::vector<es::PipeSegDesc> segs;
+        for (auto &q : pipes) segs.push_back(q.second);
+        s = h->timed(ES_KERNEL_FOLD, pbytes, cs, [&](int *nl) {
+          return es::launch_fold_pipe((es_dtype)dd, p.N, r, segs.data(), (int)segs.size(),
+                                      reinterpret_cast<const uint64_t *>(h->ws + p.flags_off) + es::kEpochSlot,
+                                      reinterpret_cast<unsigned int *>(
+                                          reinterpret_cast<uint64_t *>(h->ws + p.flags_off) + es::kTicketSlot),
+                                      h->peer_share, cs, nl);
         });
         if (s != ES_OK) return s;
       }

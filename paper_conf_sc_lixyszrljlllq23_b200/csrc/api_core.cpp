@@ -103,6 +103,8 @@ es_status es_init(const es_config *cfg, void *workspace, size_t workspace_bytes,
       return set_err(ES_ECUDA, "cudaStreamCreate failed");
     bool ok = cudaMemsetAsync(h->ws + h->plan.scratch_off, 0, 256, zs) == cudaSuccess;
     if (ok && h->plan.peer) ok = cudaMemsetAsync(h->ws + h->plan.flags_off, 0, es::kPeerFlagWords * 8, zs) == cudaSuccess;
+    if (ok && h->plan.pipe_flag_words > 0)
+      ok = cudaMemsetAsync(h->ws + h->plan.pipe_flags_off, 0, h->plan.pipe_flag_words * 8, zs) == cudaSuccess;
     ok = cudaStreamSynchronize(zs) == cudaSuccess && ok;
     cudaStreamDestroy(zs);
     if (!ok) return set_err(ES_ECUDA, "cudaMemsetAsync of the workspace scratch / peer flags failed");

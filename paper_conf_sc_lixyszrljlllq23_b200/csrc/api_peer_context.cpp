@@ -131,6 +131,7 @@ es_status es_peer_open(es_handle h, const void *blobs, size_t bytes) {
   h->peer_ws = ws;
   h->ipc_mapped = mapped;
   h->peer_open = true;
+  h->peer_share = std::max<int32_t>(1, same_process);
   return ES_OK;
 }
 

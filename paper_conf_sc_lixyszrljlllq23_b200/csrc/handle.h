@@ -86,6 +86,7 @@ struct es_ctx {
   std::vector<unsigned char *> peer_ws;   // [G] workspace base of every rank, mapped here
   std::vector<void *> ipc_mapped;         // cudaIpcOpenMemHandle results to close
   bool peer_open = false;
+  int32_t peer_share = 1;                 // ranks of this process sharing the device (loopback)
 
   // instrumentation
   bool prof = false;

@@ -30,6 +30,7 @@
 #include <cuda_bf16.h>
 
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 #include <vector>
 
@@ -43,6 +44,17 @@ constexpr int kBatch = 8;        // sources loaded per batch in k_fold
 // persistent grid-stride ones; 148 x 64 blocks covers every bucket this build
 // plans for, larger ones loop.
 constexpr int kMaxBlocks = kSMs * 64;
+
+// Device spin-waits (peer barrier, pipelined chain) trap after this long
+// instead of hanging the GPU; ES_BARRIER_TIMEOUT_S overrides the 60 s default.
+uint64_t barrier_timeout_ns() {
+  static const uint64_t ns = [] {
+    const char *e = std::getenv("ES_BARRIER_TIMEOUT_S");
+    const double sec = e ? std::atof(e) : 60.0;
+    return (uint64_t)((sec > 0 ? sec : 60.0) * 1e9);
+  }();
+  return ns;
+}
 
 bool g_pdl = [] {
   const char *e = std::getenv("ES_NO_PDL");
@@ -77,6 +89,20 @@ __device__ __forceinline__ uint2 ld_stream(const uint2 *p) {
   return r;
 }
 __device__ __forceinline__ int4 ld_stream(const int4 *p) { return ld_stream(static_cast<const void *>(p)); }
+
+// L2-coherent loads (bypass L1) of data another GPU publishes during this
+// kernel behind a flag (k_fold_pipe's incoming partials).
+__device__ __forceinline__ int4 ld_cg(const void *p) {
+  int4 r;
+  asm volatile("ld.global.cg.v4.s32 {%0, %1, %2, %3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p)
+               : "memory");
+  return r;
+}
+__device__ __forceinline__ float ld_cg1(const float *p) {
+  float r;
+  asm volatile("ld.global.cg.f32 %0, [%1];" : "=f"(r) : "l"(p) : "memory");
+  return r;
+}
 
 __device__ __forceinline__ void st_stream(void *p, const int4 &v) {
   asm volatile("st.global.L1::no_allocate.v4.s32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x), "r"(v.y),
@@ -259,7 +285,7 @@ __device__ __forceinline__ float add_step(float s, float v, uint32_t compat) {
 }
 
 // Fold of one 16-byte vector at segment offset t (elements), into acc[V].
-template <typename T, bool COMPAT>
+template <typename T, bool COMPAT, bool CG = false>
 __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const *src, int32_t N, int64_t t,
                                             float *acc, uint32_t compat, float r) {
   const float fN = (float)N;
@@ -279,7 +305,7 @@ __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const 
     const float *pp = g.part_in + t;
 #pragma unroll
     for (int q = 0; q < V / 4; ++q) {
-      int4 w = ld_stream(pp + 4 * q);
+      int4 w = CG ? ld_cg(pp + 4 * q) : ld_stream(pp + 4 * q);
       acc[4 * q + 0] = __int_as_float(w.x); acc[4 * q + 1] = __int_as_float(w.y);
       acc[4 * q + 2] = __int_as_float(w.z); acc[4 * q + 3] = __int_as_float(w.w);
     }
@@ -316,7 +342,7 @@ __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const 
   }
 }
 
-template <typename T, bool COMPAT>
+template <typename T, bool COMPAT, bool CG = false>
 __device__ __forceinline__ float fold_scalar(const FoldSeg &g, const void *const *src, int32_t N, int64_t t,
                                              uint32_t compat, float r) {
   const float fN = (float)N;
@@ -332,7 +358,7 @@ __device__ __forceinline__ float fold_scalar(const FoldSeg &g, const void *const
   float s;
   int done = 0;
   if (g.part_in) {
-    s = g.part_in[t];
+    s = CG ? ld_cg1(g.part_in + t) : g.part_in[t];
   } else {
     s = prep<COMPAT>(T::load1(src[idx], t), compat, r, fN);
     idx = (idx + 1 == cnt) ? 0 : idx + 1;
@@ -382,6 +408,125 @@ __global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams
     const float s = fold_scalar<T, COMPAT>(g, src, p.N, t, p.compat, p.r);
     if (g.out_partial) reinterpret_cast<float *>(g.out)[t] = s;
     else T::store1(g.out, t, post ? __fmul_rn(s, p.r) : s);
+  }
+}
+
+// ---- k_fold_pipe: the PEER_CHAIN rounds as one tile-pipelined kernel ----------------
+// Every chain segment on this GPU (all rounds, all buckets of one dtype) is cut
+// into tiles of kPipeTile elements; CTAs take tiles from an atomic ticket in
+// (round, bucket, chunk, tile) order.  A tile of a segment that continues a
+// partial first waits until the producer GPU has published that tile
+// (system-scope acquire on the producer's flag, read over NVLink), folds its
+// local contributions onto it and, if the chunk continues on another GPU,
+// publishes its own tile (system-scope release).  Round r+1 of a chunk thus
+// starts on tile 0 while round r is still folding later tiles: the partial's
+// transfer overlaps the folds tile by tile, with no device-wide barrier between
+// rounds.  Forward progress: on every GPU the tickets of round r are all taken
+// before any of round r+1 and round 0 waits for nothing (induction on r).
+// Flag value v = the epoch the step's closing barrier will publish, read from
+// this rank's device epoch counter: identical on every rank and larger than
+// any value of an earlier step.
+
+struct PipeSeg {
+  FoldSeg f;              // f.block0 unused
+  const uint64_t *wait;   // producer's flags for this chunk's previous round (tile t: wait[t]), or null
+  uint64_t *pub;          // own flags for this round (tile t: pub[t]), or null (the chunk ends here)
+  int32_t tile0;          // first ticket of this segment
+};
+
+template <int MAXSEG, int MAXSRC>
+struct PipeParams {
+  int32_t nseg, N, ntiles;
+  float r;
+  const uint64_t *epoch;  // this rank's barrier epoch counter
+  unsigned int *ticket;   // zeroed before the launch
+  uint64_t timeout_ns;
+  int32_t debug;          // ES_PIPE_DEBUG=1: on timeout print the stuck wait and skip it (wrong bits) instead of trapping
+  PipeSeg seg[MAXSEG];
+  const void *src[MAXSRC];
+};
+
+__device__ __forceinline__ int find_tile_seg(const PipeSeg *seg, int nseg, int tk) {
+  int lo = 0, hi = nseg - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (seg[mid].tile0 <= tk) lo = mid;
+    else hi = mid - 1;
+  }
+  return lo;
+}
+
+template <typename T, int MAXSEG, int MAXSRC>
+__global__ void __launch_bounds__(256) k_fold_pipe(const __grid_constant__ PipeParams<MAXSEG, MAXSRC> p) {
+  constexpr int V = T::kVec;
+  static_assert(kPipeTile % (4 * V) == 0, "tiles hold whole vectors");
+  __shared__ int s_tk;
+  // Wait for the predecessor but never let the successor (the closing
+  // barrier) become resident early: a dependent grid parked on the SMs while
+  // these CTAs spin on peers was measured to stall same-device peers
+  // (loopback) until the timeout; the successor launches at completion.
+  pdl_wait();
+  const uint64_t v = *reinterpret_cast<const volatile uint64_t *>(p.epoch) + 1;
+  for (;;) {
+    if (threadIdx.x == 0) s_tk = (int)atomicAdd(p.ticket, 1u);
+    __syncthreads();
+    const int tk = s_tk;
+    __syncthreads();                                   // s_tk is rewritten next iteration
+    if (tk >= p.ntiles) break;
+    const PipeSeg &ps = p.seg[find_tile_seg(p.seg, p.nseg, tk)];
+    const FoldSeg &g = ps.f;
+    const int64_t tile = tk - ps.tile0;
+    const int64_t e0 = tile * kPipeTile, e1 = min(g.n, e0 + (int64_t)kPipeTile);
+    if (ps.wait && threadIdx.x == 0) {                 // the producer's tile, published over NVLink
+      const uint64_t *fl = ps.wait + tile;
+      uint64_t f = 0, t0 = 0, now = 0;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+      for (;;) {
+        asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(f) : "l"(fl) : "memory");
+        if (f >= v) break;
+        __nanosleep(64);
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now));
+        if (now - t0 > p.timeout_ns) {                // the producer never published: fail loudly
+          if (!p.debug) __trap();
+          printf("k_fold_pipe stuck: block %d ticket %d seg lo %lld n %lld tile %lld flag %llu want %llu wait %p\n",
+                 (int)blockIdx.x, tk, (long long)g.lo, (long long)g.n, (long long)tile, (unsigned long long)f,
+                 (unsigned long long)v, (const void *)fl);
+          break;
+        }
+      }
+    }
+    __syncthreads();
+    const void *const *src = p.src + g.src0;
+    const int64_t tail0 = (g.n / V) * V;
+    const int64_t vend = min(e1, tail0);
+    for (int64_t t = e0 + (int64_t)threadIdx.x * V; t < vend; t += (int64_t)blockDim.x * V) {
+      float acc[V];
+      fold_vector<T, false, true>(g, src, p.N, t, acc, 0u, p.r);
+      if (g.out_partial) {
+        float *o = reinterpret_cast<float *>(g.out) + t;
+#pragma unroll
+        for (int q = 0; q < V / 4; ++q)
+          st_stream(o + 4 * q, make_int4(__float_as_int(acc[4 * q]), __float_as_int(acc[4 * q + 1]),
+                                         __float_as_int(acc[4 * q + 2]), __float_as_int(acc[4 * q + 3])));
+      } else {
+#pragma unroll
+        for (int e = 0; e < V; ++e) acc[e] = __fmul_rn(acc[e], p.r);   // R5: one rounding
+        st_stream(reinterpret_cast<char *>(g.out) + t * T::kSize, T::narrow(acc));  // R13
+      }
+    }
+    if (e1 == g.n && tail0 < g.n && (int64_t)threadIdx.x < g.n - tail0) {   // ragged tail, last tile
+      const int64_t t = tail0 + threadIdx.x;
+      const float sc = fold_scalar<T, false, true>(g, src, p.N, t, 0u, p.r);
+      if (g.out_partial) reinterpret_cast<float *>(g.out)[t] = sc;
+      else T::store1(g.out, t, __fmul_rn(sc, p.r));
+    }
+    if (ps.pub) {                                      // publish this tile to the next GPU
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        __threadfence_system();
+        asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(ps.pub + tile), "l"(v) : "memory");
+      }
+    }
   }
 }
 
@@ -566,6 +711,80 @@ cudaError_t launch_fold_t(int32_t N, float r, uint32_t compat, const FoldSegDesc
     cudaError_t e = (j - i <= kSmallSeg && nsrc <= kSmallSrc)
                         ? launch_fold_group<T, kSmallSeg, kSmallSrc>(N, r, compat, segs + i, j - i, s, bo, to)
                         : launch_fold_group<T, kBigSeg, kBigSrc>(N, r, compat, segs + i, j - i, s, bo, to);
+    if (e != cudaSuccess) return e;
+    ++*launches;
+    i = j;
+  }
+  return cudaSuccess;
+}
+
+
+template <typename T, int MAXSEG, int MAXSRC>
+cudaError_t launch_pipe_group(int32_t N, float r, const PipeSegDesc *d, int nseg, const uint64_t *epoch,
+                              unsigned int *ticket, int share, cudaStream_t s) {
+  PipeParams<MAXSEG, MAXSRC> p;
+  p.nseg = nseg;
+  p.N = N;
+  p.r = r;
+  p.epoch = epoch;
+  p.ticket = ticket;
+  p.timeout_ns = barrier_timeout_ns();
+  static const int dbg = [] {
+    const char *e = std::getenv("ES_PIPE_DEBUG");
+    return e && e[0] == '1' ? 1 : 0;
+  }();
+  p.debug = dbg;
+  int nsrc = 0, tiles = 0;
+  for (int i = 0; i < nseg; ++i) {
+    PipeSeg &g = p.seg[i];
+    const FoldSegDesc &f = d[i].f;
+    g.f.part_in = f.part_in;
+    g.f.out = f.out;
+    g.f.lo = f.lo;
+    g.f.n = f.n;
+    g.f.C = f.C;
+    g.f.rot = 0;
+    g.f.m = f.m;
+    g.f.src0 = nsrc;
+    g.f.out_partial = f.out_partial ? 1 : 0;
+    g.f.block0 = 0;
+    for (int j = 0; j < f.m; ++j) p.src[nsrc + j] = f.src[j];
+    nsrc += f.m;
+    g.wait = d[i].wait;
+    g.pub = d[i].pub;
+    g.tile0 = tiles;
+    tiles += (int)((f.n + kPipeTile - 1) / kPipeTile);
+  }
+  p.ntiles = tiles;
+  static const int occ = [] {
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_fold_pipe<T, MAXSEG, MAXSRC>, 256, 0) != cudaSuccess) {
+      cudaGetLastError();
+      b = 1;
+    }
+    return std::max(b, 1);
+  }();
+  static const int share_env = [] {   // ES_PIPE_SHARE: diagnostic override of the device share
+    const char *e = std::getenv("ES_PIPE_SHARE");
+    return e ? std::atoi(e) : 0;
+  }();
+  if (share_env > 0) share = share_env;
+  const int grid = std::max(1, std::min(tiles, kSMs * occ / std::max(share, 1)));
+  cudaError_t e = cudaMemsetAsync(ticket, 0, sizeof(unsigned int), s);
+  if (e != cudaSuccess) return e;
+  return launch_k<k_fold_pipe<T, MAXSEG, MAXSRC>>(dim3(grid), dim3(256), s, p);
+}
+
+template <typename T>
+cudaError_t launch_pipe_t(int32_t N, float r, const PipeSegDesc *segs, int nseg, const uint64_t *epoch,
+                          unsigned int *ticket, int share, cudaStream_t s, int *launches) {
+  constexpr int kSeg = 64, kSrc = 1024;
+  int i = 0;
+  while (i < nseg) {                                   // groups keep the (round-major) order
+    int j = i, nsrc = 0;
+    while (j < nseg && j - i < kSeg && nsrc + segs[j].f.m <= kSrc) nsrc += segs[j++].f.m;
+    if (j == i) return cudaErrorInvalidValue;
+    cudaError_t e = launch_pipe_group<T, kSeg, kSrc>(N, r, segs + i, j - i, epoch, ticket, share, s);
     if (e != cudaSuccess) return e;
     ++*launches;
     i = j;
@@ -1114,6 +1333,19 @@ cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *s
   return launch_stash_t<BF16T, F32T, 4>(live.data(), n, s, bo, to, launches, swap, early);
 }
 
+cudaError_t launch_fold_pipe(es_dtype dtype, int32_t N, float r, const PipeSegDesc *segs, int nseg,
+                             const uint64_t *epoch, unsigned int *ticket, int share, cudaStream_t s, int *launches) {
+  int dummy = 0;
+  if (!launches) launches = &dummy;
+  std::vector<PipeSegDesc> live;
+  for (int i = 0; i < nseg; ++i)
+    if (segs[i].f.n > 0) live.push_back(segs[i]);
+  if (live.empty()) return cudaSuccess;
+  if (dtype == ES_BF16)
+    return launch_pipe_t<BF16T>(N, r, live.data(), (int)live.size(), epoch, ticket, share, s, launches);
+  return launch_pipe_t<F32T>(N, r, live.data(), (int)live.size(), epoch, ticket, share, s, launches);
+}
+
 cudaError_t launch_dropout(es_dtype dtype, const void *x, void *y, uint8_t *mask, int64_t n, float p, float scale,
                            uint64_t *record, unsigned int *counter, cudaStream_t s) {
   DropoutParams d{x, y, mask, n, p, scale, record, counter};
@@ -1131,12 +1363,7 @@ cudaError_t launch_peer_barrier(uint64_t *const *peer_flags, uint64_t *my_flags,
   b.my_flags = my_flags;
   b.G = G;
   b.rank = rank;
-  static const uint64_t timeout_ns = [] {
-    const char *e = getenv("ES_BARRIER_TIMEOUT_S");   // default 60 s
-    const double sec = e ? atof(e) : 60.0;
-    return (uint64_t)((sec > 0 ? sec : 60.0) * 1e9);
-  }();
-  b.timeout_ns = timeout_ns;
+  b.timeout_ns = barrier_timeout_ns();
   return launch_k<k_peer_barrier>(dim3(1), dim3(64), s, b);
 }
 

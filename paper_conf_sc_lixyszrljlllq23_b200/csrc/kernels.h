@@ -40,6 +40,22 @@ struct FoldSegDesc {
 cudaError_t launch_fold_multi(es_dtype dtype, int32_t N, float r, uint32_t compat, const FoldSegDesc *segs, int nseg,
                               cudaStream_t s, int blocks_override, int threads_override, int *launches);
 
+// PEER_CHAIN, tile-pipelined (k_fold_pipe): chain segments (rot == false)
+// cut into tiles of kPipeTile elements.  wait: the producer GPU's flags of
+// this chunk's previous round (tile t at wait[t]; null in round 0); pub: this
+// GPU's flags of the round (null when the chunk ends here).  Segments must be
+// passed in round-major order.  epoch: this rank's barrier epoch word (the
+// flag value is *epoch + 1); ticket: a zeroable device word; share: number of
+// ranks sharing this device (the grid is cut so that all of them fit).
+constexpr int kPipeTile = 8192;
+struct PipeSegDesc {
+  FoldSegDesc f;
+  const uint64_t *wait = nullptr;
+  uint64_t *pub = nullptr;
+};
+cudaError_t launch_fold_pipe(es_dtype dtype, int32_t N, float r, const PipeSegDesc *segs, int nseg,
+                             const uint64_t *epoch, unsigned int *ticket, int share, cudaStream_t s, int *launches);
+
 // Stash segments: dst[i] = cast(src[i]) for i < n, all with
 // the same (source dtype, destination dtype).
 struct StashSegDesc {
@@ -93,7 +109,8 @@ cudaError_t launch_dropout(es_dtype dtype, const void *x, void *y, uint8_t *mask
 // this rank's own flag array holds >= e in every slot (system-scope acquire).
 // One block.  my_flags has kPeerFlagWords u64 words, zeroed at es_init.
 constexpr int kEpochSlot = 64;
-constexpr int kPeerFlagWords = 65;
+constexpr int kTicketSlot = 65;     // k_fold_pipe's work counter (local)
+constexpr int kPeerFlagWords = 66;
 cudaError_t launch_peer_barrier(uint64_t *const *peer_flags, uint64_t *my_flags, int32_t G, int32_t rank,
                                 cudaStream_t s);
 

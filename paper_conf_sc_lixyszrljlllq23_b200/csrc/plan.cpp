@@ -295,6 +295,8 @@ void plan_peer_chain(const Plan &p, BucketPlan *b) {
   std::vector<std::vector<std::vector<int64_t>>> offs(p.G);
   for (int32_t h = 0; h < p.G; ++h) b->peer_part_bytes = std::max(b->peer_part_bytes, chain_out_parts(sh, h, &offs[h]));
   b->part_bytes = 0;
+  b->chain_rounds = sh.R;
+  b->tiles_per_chunk = (b->C + kPipeTile - 1) / kPipeTile;
   b->ops.push_back(make_op(ES_OP_BARRIER, 0));
   for (int32_t r = 0; r < sh.R; ++r) {
     for (int32_t c = 0; c < p.N; ++c) {
@@ -360,7 +362,7 @@ bool validate(const es_config *cfg, std::string *err, bool need_comm) {
     return fail(err, "unknown compat bits");
   if ((cfg->compat & ES_COMPAT_PREDIV) && (cfg->compat & ES_COMPAT_PREMUL))
     return fail(err, "compat PREDIV and PREMUL are exclusive");
-  if (cfg->options & ~(uint32_t)ES_OPT_INCREMENTAL) return fail(err, "unknown option bits");
+  if (cfg->options & ~(uint32_t)(ES_OPT_INCREMENTAL | ES_OPT_PEER_ROUNDS)) return fail(err, "unknown option bits");
   if ((cfg->options & ES_OPT_INCREMENTAL) && cfg->G != 1) return fail(err, "ES_OPT_INCREMENTAL needs G == 1");
   const bool peer_sched = cfg->sched == ES_SCHED_PEER || cfg->sched == ES_SCHED_PEER_CHAIN ||
                           cfg->sched == ES_SCHED_PEER_AUTO;
@@ -400,7 +402,7 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
   p->options = cfg->options;
 
   p->bp.resize(cfg->n_buckets);
-  uint64_t max_stage = 0, max_parts = 0, sum_peer_parts = 0;
+  uint64_t max_stage = 0, max_parts = 0, sum_peer_parts = 0, sum_pipe_flags = 0;
   for (int32_t bi = 0; bi < cfg->n_buckets; ++bi) {
     BucketPlan &b = p->bp[bi];
     b.L = p->buckets[bi].numel;
@@ -430,6 +432,10 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
     max_parts = std::max(max_parts, b.part_bytes);
     b.peer_part_base = sum_peer_parts;   // buckets of one batched call run their rounds together
     sum_peer_parts += align256(b.peer_part_bytes);
+    if (b.sched == ES_SCHED_PEER_CHAIN) {
+      b.pipe_flag_base = sum_pipe_flags;
+      sum_pipe_flags += (uint64_t)p->N * (uint64_t)b.chain_rounds * b.tiles_per_chunk;
+    }
   }
 
   // Workspace layout.
@@ -452,6 +458,9 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
     head = p->result_off + p->slot_block;   // one bucket-layout block: shard results at bucket offsets
     p->peer_parts_off = head;               // PEER_CHAIN partials: per bucket, max over ranks
     head += align256(sum_peer_parts);
+    p->pipe_flags_off = head;               // PEER_CHAIN tile flags (k_fold_pipe)
+    p->pipe_flag_words = sum_pipe_flags;
+    head += align256(sum_pipe_flags * 8);
   }
   p->grad_off = head;
   uint64_t total = head + p->slot_block * p->local_ests.size();

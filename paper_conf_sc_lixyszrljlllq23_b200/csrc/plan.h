@@ -41,6 +41,10 @@ struct BucketPlan {
   uint64_t part_bytes = 0;
   uint64_t peer_part_bytes = 0;         // PEER_CHAIN: max over ranks of their outgoing partials
   uint64_t peer_part_base = 0;          // PEER_CHAIN: this bucket's base in the peer partials area
+  int32_t chain_rounds = 0;             // PEER_CHAIN: R, the most segments of any chunk (all ranks)
+  uint64_t tiles_per_chunk = 0;         // PEER_CHAIN: ceil(C / kPipeTile)
+  uint64_t pipe_flag_base = 0;          // PEER_CHAIN: first tile flag (u64 words) of this bucket;
+                                        //   chunk c, round r, tile t at base + (c*R + r)*tiles_per_chunk + t
   std::vector<Op> ops;
 };
 
@@ -75,6 +79,8 @@ struct Plan {
   uint64_t flags_off = 0;               // PEER: G barrier flags (u64) written by peers + epoch counter
   uint64_t result_off = 0;              // PEER: per-bucket shard results (slot-block layout)
   uint64_t peer_parts_off = 0;          // PEER_CHAIN: partials read by the next GPU (uniform offset)
+  uint64_t pipe_flags_off = 0;          // PEER_CHAIN: per-tile publish flags (uniform offset)
+  uint64_t pipe_flag_words = 0;
   bool peer = false;                    // some bucket uses ES_SCHED_PEER
   std::vector<int32_t> owner_index;     // [N]: EST's index among its owner's local ESTs
   uint64_t total = 0;

@@ -26,6 +26,7 @@ ES_BUF_NONE, ES_BUF_SRC, ES_BUF_STAGE, ES_BUF_PART, ES_BUF_OUT, ES_BUF_RESULT, E
 ES_PEER_BLOB_BYTES = 128
 ES_COMPAT_PREDIV, ES_COMPAT_PREMUL, ES_COMPAT_BF16_HOP = 1, 2, 4
 ES_OPT_INCREMENTAL = 1
+ES_OPT_PEER_ROUNDS = 2
 
 EXPORTED = [
     "es_workspace_bytes", "es_init", "es_destroy", "es_sync", "es_register_state", "es_init_state",

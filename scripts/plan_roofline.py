@@ -68,23 +68,39 @@ def rank_costs(name, G, kind, sched):
                         nv += n * esz
                     hb += n * esz * (2 if int(f[3]) == g else 1)
                 phases[ph] = (hb, nv)
-        out.append([phases[k] for k in sorted(phases)])
+        out.append(phases)
     return out
 
 
 def bound_ms(costs):
-    nph = max(len(r) for r in costs)
+    keys = sorted({k for r in costs for k in r})
     t = 0.0
-    for k in range(nph):
-        t += max(max(r[k][0] / HBM, r[k][1] / NVL) if k < len(r) else 0.0 for r in costs)
+    for k in keys:
+        t += max(max(r[k][0] / HBM, r[k][1] / NVL) if k in r else 0.0 for r in costs)
     return t * 1e3
+
+
+def bound_ms_pipelined(costs):
+    """PEER_CHAIN as k_fold_pipe runs it: every fold round of a rank overlaps
+    (per-tile flags, no barrier between rounds), so the folds are one phase;
+    the gathers (the last phase) follow the closing barrier."""
+    last = max(k for r in costs for k in r)
+    merged = []
+    for r in costs:
+        hb = sum(v[0] for k, v in r.items() if k < last)
+        nv = sum(v[1] for k, v in r.items() if k < last)
+        merged.append({0: (hb, nv), 1: r.get(last, (0, 0))})
+    return bound_ms(merged)
 
 
 def main(path):
     rows = ["# Multi-GPU roofline of the exported plans (allreduce only; HBM 6.54 TB/s, NVLink 0.77 TB/s)\n",
             "Per phase (between groups / barriers), the slowest rank's max(HBM, NVLink) time, summed.\n",
-            "| config | G | mapping | direct ms | chain ms | peer ms | peer_chain ms | AUTO picks | max NVLink in / rank MB (direct, chain) |",
-            "|---|---|---|---|---|---|---|---|---|"]
+            "peer_chain = rounds separated by barriers (ES_OPT_PEER_ROUNDS); pipelined = the default k_fold_pipe step "
+            "(all rounds overlapped through per-tile flags, then the gather).\n",
+            "| config | G | mapping | direct ms | chain ms | peer ms | peer_chain ms | peer_chain pipelined ms | AUTO picks | "
+            "max NVLink in / rank MB (direct, chain) |",
+            "|---|---|---|---|---|---|---|---|---|---|"]
     cases = [("resnet50", G, "contiguous") for G in (2, 4, 8)] + [("vgg19", G, "contiguous") for G in (2, 4, 8)] + \
         [("bert_base", 8, "contiguous"), ("bert_base", 8, "round_robin")] + \
         [("swin_b", G, "contiguous") for G in (2, 4, 8)]
@@ -95,11 +111,11 @@ def main(path):
                         [(n, es.ES_F32 if d == "f32" else es.ES_BF16) for n, d in c["buckets"]])
         picks = sorted({es.es_plan_ops(cfg, b)[1] for b in range(len(c["buckets"]))})
         pick = "/".join({1: "direct", 2: "chain"}[p] for p in picks)
-        nvd = max(sum(ph[1] for ph in r) for r in res["direct"]) / 1e6
-        nvc = max(sum(ph[1] for ph in r) for r in res["chain"]) / 1e6
+        nvd = max(sum(ph[1] for ph in r.values()) for r in res["direct"]) / 1e6
+        nvc = max(sum(ph[1] for ph in r.values()) for r in res["chain"]) / 1e6
         rows.append(f"| {name} | {G} | {kind} | {bound_ms(res['direct']):.3f} | {bound_ms(res['chain']):.3f} | "
-                    f"{bound_ms(res['peer']):.3f} | {bound_ms(res['peer_chain']):.3f} | {pick} | "
-                    f"{nvd:.0f}, {nvc:.0f} |")
+                    f"{bound_ms(res['peer']):.3f} | {bound_ms(res['peer_chain']):.3f} | "
+                    f"{bound_ms_pipelined(res['peer_chain']):.3f} | {pick} | {nvd:.0f}, {nvc:.0f} |")
     text = "\n".join(rows) + "\n"
     with open(path, "w") as f:
         f.write(text)

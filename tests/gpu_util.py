@@ -96,7 +96,7 @@ def reduce_g1(xs_per_bucket, A=16, borrow_last=True, override=None, stash_dtypes
 
 
 def reduce_loopback(xs_per_bucket, G, mapping, sched=es.ES_SCHED_AUTO, A=16, borrow_last=True, steps=1,
-                    batched=False):
+                    batched=False, options=0):
     """G ranks in one process over the LOOPBACK transport, one host thread and
     one CUDA stream per rank, all on the current GPU.  Returns per-rank lists
     of outputs (each rank must hold the full averaged buckets)."""
@@ -104,7 +104,7 @@ def reduce_loopback(xs_per_bucket, G, mapping, sched=es.ES_SCHED_AUTO, A=16, bor
     buckets = [(x[0].size, code(x[0])) for x in xs_per_bucket]
     world = es.es_loopback_create(G)
     aggs = [Aggregator(N, G, g, mapping, buckets, chunk_align=A, transport=es.ES_TRANSPORT_LOOPBACK,
-                       comm=world.value, sched=sched) for g in range(G)]
+                       comm=world.value, sched=sched, options=options) for g in range(G)]
     if sched in es.PEER_SCHEDS:                   # same process: peers map by raw address
         blobs = [a.peer_blob() for a in aggs]
         for a in aggs:

@@ -560,3 +560,37 @@ def test_sixteen_loopback_ranks():
     with pytest.raises(es.EsError) as e:
         reduce_loopback(xs, 16, workloads.mapping(40, 16, "random", seed=5), es.ES_SCHED_PEER_AUTO)
     assert e.value.status == es.ES_EUNSUPPORTED
+
+
+# ---- PEER_CHAIN tile pipelining (k_fold_pipe) --------------------------------------------------
+
+@pytest.mark.parametrize("options", [0, es.ES_OPT_PEER_ROUNDS])
+@pytest.mark.parametrize("G,N,kind", [(2, 8, "contiguous"), (4, 8, "contiguous"), (3, 12, "random"),
+                                      (8, 12, "contiguous"), (4, 16, "round_robin")])
+def test_peer_chain_pipelined_many_tiles(options, G, N, kind):
+    """Chunks of tens of k_fold_pipe tiles (8192 elements) plus ragged tails,
+    mixed dtypes, three steps on the same handles: the tile-pipelined chain
+    (per-tile flags instead of round barriers) and the round-barrier chain
+    both give the oracle's bits on every rank."""
+    rng = np.random.default_rng(1000 + G * N)
+    xs = [_gauss(rng, N, 1_000_003), _gauss(rng, N, 262_147, "bf16"), _gauss(rng, N, 8195)]
+    want = [oracle.reduce(xs[0], "f32"), oracle.reduce(xs[1], "bf16"), oracle.reduce(xs[2], "f32")]
+    m = workloads.mapping(N, G, kind, seed=11)
+    res = reduce_loopback(xs, G, m, es.ES_SCHED_PEER_CHAIN, steps=3, batched=True, options=options)
+    for g in range(G):
+        for b in range(3):
+            assert_bits_equal(res[g][b], want[b], f"G={G} N={N} {kind} opt={options} rank={g} b={b}")
+
+
+def test_peer_auto_mixed_pipelined():
+    """PEER_AUTO mixes PEER and PEER_CHAIN buckets in one batched call; both
+    share the pipelined step's two barriers."""
+    rng = np.random.default_rng(77)
+    N, G = 8, 4
+    xs = [_gauss(rng, N, 400_001), _gauss(rng, N, 70_001, "bf16"), _gauss(rng, N, 5)]
+    want = [oracle.reduce(xs[0], "f32"), oracle.reduce(xs[1], "bf16"), oracle.reduce(xs[2], "f32")]
+    for kind in ("contiguous", "round_robin"):
+        res = reduce_loopback(xs, G, workloads.mapping(N, G, kind), es.ES_SCHED_PEER_AUTO, steps=2, batched=True)
+        for g in range(G):
+            for b in range(3):
+                assert_bits_equal(res[g][b], want[b], f"{kind} rank={g} b={b}")
