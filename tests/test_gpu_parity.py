@@ -594,3 +594,37 @@ def test_peer_auto_mixed_pipelined():
         for g in range(G):
             for b in range(3):
                 assert_bits_equal(res[g][b], want[b], f"{kind} rank={g} b={b}")
+
+
+# ---- randomized schedules ------------------------------------------------------------------------
+
+SCHED_NAMES = {es.ES_SCHED_DIRECT: "direct", es.ES_SCHED_CHAIN: "chain", es.ES_SCHED_AUTO: "auto",
+               es.ES_SCHED_PEER: "peer", es.ES_SCHED_PEER_CHAIN: "peer_chain",
+               es.ES_SCHED_PEER_AUTO: "peer_auto"}
+
+
+@pytest.mark.parametrize("seed", range(int(os.environ.get("ES_FUZZ_SEEDS", "40"))))
+def test_random_schedules_mappings_layouts(seed):
+    """Seeded random N, G, EST->GPU map (any surjection), bucket layout (empty,
+    tiny, ragged, multi-tile; f32/bf16), chunk alignment, schedule and
+    PEER_CHAIN executor, one to three steps: every rank holds the oracle's bits."""
+    rng = np.random.default_rng(5000 + seed)
+    N = int(rng.integers(2, 17))
+    G = int(rng.integers(2, min(N, 6) + 1))
+    m = list(range(G)) + [int(v) for v in rng.integers(0, G, N - G)]
+    rng.shuffle(m)
+    nb = int(rng.integers(1, 5))
+    sizes = [int(rng.choice([0, 1, 7, 15, 16, 17, 1000, 8191, 8193, 65537, 300_001])) for _ in range(nb)]
+    sizes[0] = max(sizes[0], 1)                                   # at least one non-empty bucket
+    dts = [str(rng.choice(["f32", "bf16"])) for _ in range(nb)]
+    A = int(rng.choice([8, 16, 64, 1024]))
+    sched = int(rng.choice(list(SCHED_NAMES)))
+    options = int(rng.choice([0, es.ES_OPT_PEER_ROUNDS]))
+    steps = int(rng.integers(1, 4))
+    xs = [_gauss(rng, N, L, d) for L, d in zip(sizes, dts)]
+    want = [oracle.reduce(x, d, A=A) for x, d in zip(xs, dts)]
+    what = f"seed={seed} N={N} G={G} map={m} sizes={sizes} dts={dts} A={A} {SCHED_NAMES[sched]} opt={options}"
+    res = reduce_loopback(xs, G, m, sched, A=A, steps=steps, batched=bool(seed % 2), options=options)
+    for g in range(G):
+        for b in range(nb):
+            assert_bits_equal(res[g][b], want[b], f"{what} rank={g} b={b}")
