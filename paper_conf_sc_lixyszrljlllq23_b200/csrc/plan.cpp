@@ -246,9 +246,11 @@ void plan_chain(const Plan &p, BucketPlan *b) {
 // The CHAIN schedule without a transport: the GPU of segment r of chunk c
 // reads the incoming unrounded fp32 partial directly out of the producer's
 // workspace over NVLink (part_in = a peer pointer) inside its fold kernel, so
-// the partial's transfer and the local fold are one kernel.  A device barrier
-// separates rounds; chunk c ends in the RESULT area of the GPU of EST c and
-// is gathered from there.
+// the partial's transfer and the local fold are one kernel.  The op list keeps
+// a BARRIER between rounds; the default executor replaces those inner barriers
+// by per-tile flags (k_fold_pipe, tile flags at pipe_flag_base) and keeps only
+// the first and the last; ES_OPT_PEER_ROUNDS executes them as written.  Chunk
+// c ends in the RESULT area of the GPU of EST c and is gathered from there.
 
 struct ChainShape {
   std::vector<std::vector<Seg>> segs;
