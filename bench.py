@@ -49,6 +49,8 @@ def parse():
     p.add_argument("--inplace", action="store_true",
                    help="NEXT-2 zero-copy stash: each EST's gradients are produced in its slot (es_slot_ptr) and "
                         "stashed with ES_STASH_INPLACE")
+    p.add_argument("--stash-background", action="store_true",
+                   help="ES_OPT_STASH_BACKGROUND: one-wave stash grids (for overlap with compute; scripts/overlap_probe.py)")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     p.add_argument("--cpu-seconds", type=float, default=10.0)
@@ -274,7 +276,8 @@ def main():
     snb = workloads.state_nbytes()
     agg = Aggregator(N, G, rank, mapping, buckets, state_nbytes=snb,
                      transport=es.ES_TRANSPORT_NONE if G == 1 else es.ES_TRANSPORT_NCCL, comm=comm, sched=sched,
-                     device=dev, options=es.ES_OPT_INCREMENTAL if args.incremental else 0)
+                     device=dev, options=(es.ES_OPT_INCREMENTAL if args.incremental else 0) |
+                     (es.ES_OPT_STASH_BACKGROUND if args.stash_background else 0))
     if G > 1 and sched in es.PEER_SCHEDS:
         agg.peer_connect()                       # CUDA IPC map of every peer's workspace (NVLink)
     live = [torch.zeros(n, dtype=torch.uint8, device=dev) for n in snb]
@@ -476,7 +479,8 @@ def main():
         "config": {**workload_config(args, cfg, G), "graph": graph is not None,
                    "api": "per-bucket" if args.per_bucket else ("incremental" if args.incremental else
                                                                ("zero-copy-inplace" if args.inplace else
-                                                                ("batched" if args.no_fuse else "batched+fused-switch"))),
+                                                                ("batched" if args.no_fuse else "batched+fused-switch")))
+                   + (" +stash-background" if args.stash_background else ""),
                    "l2": ("inputs larger than L2 (%.1f MB of EST gradients per GPU per step)" % (in_bytes / 1e6))
                    if flush is None else "L2 flushed between timed steps (512 MB write)"},
         "roofline": dominant,

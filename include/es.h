@@ -164,6 +164,14 @@ typedef struct {
 /* ES_OPT_PEER_ROUNDS: PEER_CHAIN without tile pipelining (a device barrier
  * between rounds).  Same bits; kept for comparison and as a fallback. */
 #define ES_OPT_PEER_ROUNDS 2u
+/* ES_OPT_STASH_BACKGROUND: the kernels that run at an EST's switch (stash,
+ * incremental fold) use at most two 256-thread CTAs per SM instead of a
+ * one-shot grid.  A one-shot grid of thousands of CTAs is dispatched ahead of
+ * any kernel queued after it on another stream, so the model's next forward
+ * waits for the whole stash; a one-wave grid leaves the SMs' other slots to
+ * it, and the stash streams in the background.  Slightly
+ * slower when nothing else runs.  Same bits. */
+#define ES_OPT_STASH_BACKGROUND 4u
 
 /* NEXT-3 compatibility variants -- same canonical order, different step
  * arithmetic:
@@ -263,10 +271,13 @@ es_status es_stash_and_switch(es_handle h, int32_t est, int32_t n, const int32_t
  * fold its contribution straight into the running unrounded fp32 partials of
  * the chunks c < est -- for them `est` comes after c+1..est-1 in canonical
  * order (R2), and ESTs run in index order -- and stash only chunks >= est,
- * which wait for the wrap.  es_allreduce of the bucket then folds the
- * partials with the stashed 0..c of each chunk: the end-of-step critical
- * path reads ~(N+3)/2 contributions per element instead of N+1, with the
- * same bits (segmentability, R14) and about the same total bytes.
+ * which wait for the wrap.  The last EST (N-1) folds nothing at its call
+ * (COPY stashes the whole bucket, BORROW keeps the buffer): es_allreduce of
+ * the bucket folds, per chunk c, the partial (ESTs c+1..N-2), EST N-1 and
+ * the stashed 0..c, so the end-of-step critical path reads the partial plus
+ * c+2 contributions per element -- ~(N+3)/2 on average -- instead of N,
+ * with the same bits (segmentability, R14).  Total bytes grow by the
+ * partials' round trips, which the paper's overlap hides.
  * Requirements: G == 1, cfg.options has ES_OPT_INCREMENTAL, every EST of the
  * step calls this for the bucket in order 0, 1, ..., N-1 (ES_ESTATE
  * otherwise; mixing with es_stash_grad for the same bucket and step is an

@@ -274,8 +274,10 @@ es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void
     };
     unsigned char *outp = reinterpret_cast<unsigned char *>(outs[i]);
     if (h->inc_next[bucket] == p.N && b.L > 0) {
-      // NEXT-1 end of step: chunk c < N-1 continues from its partial (ESTs
-      // c+1..N-1) over the stashed ESTs 0..c; chunk N-1 folds 0..N-1.
+      // NEXT-1 end of step (the last EST's fold was deferred to here): chunk
+      // c < N-2 continues from its partial (ESTs c+1..N-2) over EST N-1 and
+      // the stashed ESTs 0..c; chunk N-2 folds N-1, 0..N-2 (EST N-1 is its
+      // first); chunk N-1 folds 0..N-1.
       if (!pend.empty() && pend_dt != b.dtype && (s = flush()) != ES_OK) return s;
       pend_dt = b.dtype;
       const float *part = reinterpret_cast<const float *>(h->ws + p.inc_off + p.inc_bucket_off[bucket]);
@@ -288,12 +290,13 @@ es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void
         d.n = hi - lo;
         d.C = (uint32_t)b.C;
         d.rot = false;
-        const bool cont = c < p.N - 1;
-        d.m = cont ? c + 1 : p.N;
+        const bool cont = c < p.N - 2;
+        std::vector<const void *> src;
+        if (c < p.N - 1) src.push_back(src_base(p.N - 1) + (uint64_t)lo * esz);
+        for (int32_t e = 0; e <= (c < p.N - 1 ? c : p.N - 1); ++e) src.push_back(src_base(e) + (uint64_t)lo * esz);
+        d.m = (int32_t)src.size();
         d.part_in = cont ? part + lo : nullptr;
         d.out = outp + (uint64_t)lo * esz;
-        std::vector<const void *> src;
-        for (int32_t e = 0; e < d.m; ++e) src.push_back(src_base(e) + (uint64_t)lo * esz);
         pend_bytes += (uint64_t)d.n * ((uint64_t)d.m * esz + (cont ? 4 : 0) + esz);
         pend.push_back(d);
         pend_src.push_back(std::move(src));

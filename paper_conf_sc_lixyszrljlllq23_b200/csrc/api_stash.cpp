@@ -87,8 +87,8 @@ es_status stash_impl(es_handle h, int32_t est, int32_t n, const int32_t *buckets
         const es::SwapArgs *sw = swapped ? nullptr : &swap;
         const bool early = follows_own_stash(h, cs);
         s = h->timed(ES_KERNEL_STASH, nbytes + (sw ? swap_bytes : 0), cs, [&](int *nl) {
-          return es::launch_stash_multi((es_dtype)sd, (es_dtype)dd, segs.data(), (int)segs.size(), cs, h->blocks_ov,
-                                        h->threads_ov, nl, sw, early);
+          return es::launch_stash_multi((es_dtype)sd, (es_dtype)dd, segs.data(), (int)segs.size(), cs, h->switch_blocks(),
+                                        h->switch_threads(), nl, sw, early);
         });
         if (s != ES_OK) return s;
         remember_stash_node(h, cs);
@@ -170,8 +170,12 @@ es_status es_stash_fold_grads(es_handle h, int32_t est, int32_t n, const int32_t
       const unsigned char *x = reinterpret_cast<const unsigned char *>(grads[i]);
       float *part = reinterpret_cast<float *>(h->ws + p.inc_off + p.inc_bucket_off[bk]);
       const int64_t L = (int64_t)b.L, C = (int64_t)b.C;
-      const int64_t cont_hi = std::min<int64_t>(L, (int64_t)std::max(est - 1, 0) * C);   // chunks < est-1
-      const int64_t inc_hi = std::min<int64_t>(L, (int64_t)est * C);                     // chunks < est
+      // The last EST's fold is deferred into the end-of-step fold (which reads
+      // its gradient right after the partials), so the partials make no extra
+      // round trip through HBM on the critical path: nothing is folded here.
+      const bool last = est == p.N - 1;
+      const int64_t cont_hi = last ? 0 : std::min<int64_t>(L, (int64_t)std::max(est - 1, 0) * C);   // chunks < est-1
+      const int64_t inc_hi = last ? 0 : std::min<int64_t>(L, (int64_t)est * C);                     // chunks < est
       auto add = [&](int64_t lo, int64_t hi, bool cont) {
         if (hi <= lo) return;
         es::FoldSegDesc d;
@@ -198,15 +202,15 @@ es_status es_stash_fold_grads(es_handle h, int32_t est, int32_t n, const int32_t
     if (!segs.empty()) {
       for (size_t j = 0; j < segs.size(); ++j) segs[j].src = srcs[j].data();
       s = h->timed(ES_KERNEL_FOLD, fbytes, cs, [&](int *nl) {
-        return es::launch_fold_multi((es_dtype)dd, p.N, r, p.compat, segs.data(), (int)segs.size(), cs, h->blocks_ov,
-                                     h->threads_ov, nl);
+        return es::launch_fold_multi((es_dtype)dd, p.N, r, p.compat, segs.data(), (int)segs.size(), cs,
+                                     h->switch_blocks(), h->switch_threads(), nl);
       });
       if (s != ES_OK) return s;
     }
     if (!st.empty()) {
       s = h->timed(ES_KERNEL_STASH, sbytes, cs, [&](int *nl) {
-        return es::launch_stash_multi((es_dtype)dd, (es_dtype)dd, st.data(), (int)st.size(), cs, h->blocks_ov,
-                                      h->threads_ov, nl);
+        return es::launch_stash_multi((es_dtype)dd, (es_dtype)dd, st.data(), (int)st.size(), cs,
+                                      h->switch_blocks(), h->switch_threads(), nl);
       });
       if (s != ES_OK) return s;
     }

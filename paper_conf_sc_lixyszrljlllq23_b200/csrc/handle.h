@@ -102,6 +102,14 @@ struct es_ctx {
   uint64_t bytes[ES_KERNEL_KINDS] = {};
   double ms[ES_KERNEL_KINDS] = {};
   int blocks_ov = 0, threads_ov = 0;
+  // Grid of the kernels that run at an EST's switch (stash, incremental
+  // fold): ES_OPT_STASH_BACKGROUND caps it (negative = a cap for the
+  // launchers) at two 256-thread CTAs per SM, so the model's kernels queued
+  // behind it are dispatched at once ("Overlap with compute").
+  int switch_blocks() const {
+    return blocks_ov ? blocks_ov : ((plan.options & ES_OPT_STASH_BACKGROUND) ? -2 * 148 : 0);
+  }
+  int switch_threads() const { return threads_ov ? threads_ov : ((plan.options & ES_OPT_STASH_BACKGROUND) ? 256 : 0); }
 
   ~es_ctx() {
     for (auto e : stash_ev) if (e) cudaEventDestroy(e);

@@ -655,6 +655,7 @@ cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSeg
   for (int i = 0; i < nseg; ++i) vecs += (d[i].n + T::kVec - 1) / T::kVec;
   int total = (int)std::min<int64_t>((vecs + threads - 1) / threads, (int64_t)kMaxBlocks);
   if (bo > 0) total = bo;
+  else if (bo < 0) total = std::min(total, -bo);   // a cap (ES_OPT_STASH_BACKGROUND)
   total = std::max(total, nseg);
   std::vector<int32_t> block0;
   split_blocks(work, total, &block0, &p.nblocks);
@@ -970,6 +971,8 @@ cudaError_t launch_stash_v(const StashSegDesc *segs, int nseg, cudaStream_t s, i
       total = (int)std::min<int64_t>(waves * resident, (int64_t)kMaxBlocks);
     }
     if (bo > 0) total = bo;
+    else if (bo < 0) total = std::min(total, -bo);   // a cap (ES_OPT_STASH_BACKGROUND)
+  else if (bo < 0) total = std::min(total, -bo);   // a cap (ES_OPT_STASH_BACKGROUND)
     total = std::max(total, k);
     std::vector<int32_t> block0;
     split_blocks(work, total, &block0, &p.nblocks);

@@ -628,3 +628,30 @@ def test_random_schedules_mappings_layouts(seed):
     for g in range(G):
         for b in range(nb):
             assert_bits_equal(res[g][b], want[b], f"{what} rank={g} b={b}")
+
+
+# ---- ES_OPT_STASH_BACKGROUND (one-wave stash / incremental-fold grids) ------------------------
+
+@pytest.mark.parametrize("incremental", [False, True])
+def test_stash_background_grid_bit_exact(incremental):
+    """The capped switch-time grid changes only which CTA does which element."""
+    from gpu_util import Aggregator, from_dev, to_dev
+    N = 8
+    rng = np.random.default_rng(1300 + incremental)
+    Ls, dts = [3_000_017, 40, 77_777], ["f32", "bf16", "f32"]
+    opts = es.ES_OPT_STASH_BACKGROUND | (es.ES_OPT_INCREMENTAL if incremental else 0)
+    agg = Aggregator(N, 1, 0, [0] * N, list(zip(Ls, dts)), options=opts)
+    outs = [agg.new_out(b) for b in range(len(Ls))]
+    xs = [_gauss(rng, N, L, d) for L, d in zip(Ls, dts)]
+    devs = [[to_dev(xs[b][k]) for b in range(len(Ls))] for k in range(N)]
+    for k in range(N):
+        mode = es.ES_STASH_BORROW if k == N - 1 else es.ES_STASH_COPY
+        if incremental:
+            agg.stash_fold(k, range(len(Ls)), devs[k], mode)
+        else:
+            agg.stash_many(k, range(len(Ls)), devs[k], mode)
+    agg.allreduce_many(range(len(Ls)), outs)
+    torch.cuda.synchronize()
+    for b, d in enumerate(dts):
+        assert_bits_equal(from_dev(outs[b]), oracle.reduce(xs[b], d), f"b={b}")
+    agg.close()
