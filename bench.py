@@ -14,6 +14,7 @@ value = N * sum_b L_b * bytes / step time (whole job; inputs resident in HBM).
 Prints ONE JSON line on rank 0.  See DESIGN.md "Measurement".
 """
 import argparse
+import hashlib
 import json
 import os
 import statistics
@@ -530,6 +531,24 @@ def main():
             mism += int((w != g_).sum())
             checked += n
         line["parity"] = {"checked_elements": checked, "mismatched_words": mism, "vs": "CPU oracle, bit-exact"}
+        # SURVEY 8(d) bit-exact flag: SHA-256 of the whole reduced bucket set (bucket order, raw
+        # words).  Equal across G and mappings (D1); the scaling run's lines can be compared.
+        h = hashlib.sha256()
+        for o in outs:
+            h.update(o.view(torch.uint8).cpu().numpy().tobytes())
+        line["output_sha256"] = h.hexdigest()
+        if payload <= 3e9 and not args.no_cpu:
+            # the whole output against the oracle (seconds of single-thread C for these sizes)
+            ho, mism_all = hashlib.sha256(), 0
+            for b, (L_b, d_b) in enumerate(buckets):
+                want = oracle.reduce([fetch(k, b, 0, L_b) for k in range(N)], d_b)
+                ho.update(want.tobytes())
+                got = outs[b].view(torch.uint8).cpu().numpy()
+                mism_all += int((got.view(want.dtype) != want).sum()) if want.dtype != np.float32 else \
+                    int((got.view(np.uint32) != want.view(np.uint32)).sum())
+            line["parity"].update({"full_output_checked": True, "full_output_mismatched_words": mism_all,
+                                   "oracle_sha256": ho.hexdigest(),
+                                   "sha256_equal": ho.hexdigest() == line["output_sha256"]})
         if world == 1 and not args.no_cpu:
             line["cpu_baseline"] = {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
                                     "sample": sample, "host_cores_available": cores_used()}
