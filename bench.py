@@ -52,6 +52,9 @@ def parse():
                         "stashed with ES_STASH_INPLACE")
     p.add_argument("--stash-background", action="store_true",
                    help="ES_OPT_STASH_BACKGROUND: one-wave stash grids (for overlap with compute; scripts/overlap_probe.py)")
+    p.add_argument("--rehearse-same-gpu", action="store_true",
+                   help="functional rehearsal of the N>1 path on ONE GPU: every rank on cuda:0, gloo process "
+                        "group, a peer schedule (CUDA IPC, no NCCL); times are not GPU-scaling numbers")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     p.add_argument("--cpu-seconds", type=float, default=10.0)
@@ -256,10 +259,24 @@ def main():
     from paper_conf_sc_lixyszrljlllq23_b200 import es, workloads
     from paper_conf_sc_lixyszrljlllq23_b200.aggregator import Aggregator, nccl_comm_ptr
 
+    rehearse = args.rehearse_same_gpu and world > 1
+    if rehearse and args.sched not in ("peer", "peer_chain", "peer_auto"):
+        raise SystemExit("--rehearse-same-gpu needs --sched peer|peer_chain|peer_auto (NCCL refuses two ranks per GPU)")
+    if rehearse:
+        local_rank = 0
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
     comm = None
-    if world > 1:
+
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cpu" if rehearse else dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+    if rehearse:
+        dist.init_process_group("gloo")
+    elif world > 1:
         dist.init_process_group("nccl", device_id=dev)
         t = torch.ones(1, device=dev)
         dist.all_reduce(t)                       # create the NCCL communicator
@@ -276,7 +293,8 @@ def main():
              "peer": es.ES_SCHED_PEER, "peer_chain": es.ES_SCHED_PEER_CHAIN, "peer_auto": es.ES_SCHED_PEER_AUTO}[args.sched]
     snb = workloads.state_nbytes()
     agg = Aggregator(N, G, rank, mapping, buckets, state_nbytes=snb,
-                     transport=es.ES_TRANSPORT_NONE if G == 1 else es.ES_TRANSPORT_NCCL, comm=comm, sched=sched,
+                     transport=es.ES_TRANSPORT_NONE if G == 1 or rehearse else es.ES_TRANSPORT_NCCL, comm=comm,
+                     sched=sched,
                      device=dev, options=(es.ES_OPT_INCREMENTAL if args.incremental else 0) |
                      (es.ES_OPT_STASH_BACKGROUND if args.stash_background else 0))
     if G > 1 and sched in es.PEER_SCHEDS:
@@ -421,10 +439,7 @@ def main():
     clk = clocks.stop(t_start, t_end)
     step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
     ms = sum(step_ms) / len(step_ms)
-    if world > 1:
-        t = torch.tensor([ms], device=dev, dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+    ms = max_over_ranks(ms)
 
     kinds = {"stash": es.ES_KERNEL_STASH, "fold": es.ES_KERNEL_FOLD, "swap": es.ES_KERNEL_SWAP,
              "gather": es.ES_KERNEL_GATHER, "barrier": es.ES_KERNEL_BARRIER}
@@ -478,6 +493,8 @@ def main():
         "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": cfg["dtype"], "data": "synthetic",
         "config": {**workload_config(args, cfg, G), "graph": graph is not None,
+                   **({"rehearsal": "all ranks on cuda:0 (functional check of the N>1 path, not a scaling number)"}
+                      if rehearse else {}),
                    "api": "per-bucket" if args.per_bucket else ("incremental" if args.incremental else
                                                                ("zero-copy-inplace" if args.inplace else
                                                                 ("batched" if args.no_fuse else "batched+fused-switch")))
@@ -537,7 +554,7 @@ def main():
         for o in outs:
             h.update(o.view(torch.uint8).cpu().numpy().tobytes())
         line["output_sha256"] = h.hexdigest()
-        if payload <= 3e9 and not args.no_cpu:
+        if payload <= 3e9:
             # the whole output against the oracle (seconds of single-thread C for these sizes)
             ho, mism_all = hashlib.sha256(), 0
             for b, (L_b, d_b) in enumerate(buckets):
@@ -602,10 +619,7 @@ def main():
             e1.record(stream)
         torch.cuda.synchronize()
         ems = e0.elapsed_time(e1) / k_e2e
-        if world > 1:
-            t = torch.tensor([ems], device=dev, dtype=torch.float64)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            ems = float(t.item())
+        ems = max_over_ranks(ems)
         line["e2e"] = {"value": round(payload / (ems / 1e3) / 1e9, 3), "unit": "GB/s", "h2d_bytes_per_step": h2d,
                        "d2h_bytes_per_step": d2h, "ms_per_step": round(ems, 3), "steps": k_e2e}
     agg.sync()
