@@ -521,6 +521,33 @@ def main():
         "clocks": clk,
     }
 
+    # ---- context-switch latency (reported separately) ----
+    if len(local) > 1:
+        n_sw = len(local) * max(1, 64 // len(local))      # a cycle: the graph ends on the EST it starts from
+        seq = [local[(i + 1) % len(local)] for i in range(n_sw)]
+        with torch.cuda.stream(stream):
+            agg.switch(local[0])
+        torch.cuda.synchronize()
+        gsw = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(gsw, stream=stream):
+            for k in seq:
+                agg.switch(k)
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with torch.cuda.stream(stream):
+            for _ in range(3):
+                gsw.replay()
+            s0.record(stream)
+            for _ in range(10):
+                gsw.replay()
+            s1.record(stream)
+        torch.cuda.synchronize()
+        us = s0.elapsed_time(s1) * 1e3 / (10 * n_sw)
+        ctx_bytes = sum(snb)
+        line["switch"] = {"us_per_switch": round(us, 3), "context_bytes": ctx_bytes,
+                          "algorithmic_GBps": round(4 * ctx_bytes / (us / 1e6) / 1e9, 1),
+                          "timed": f"{10 * n_sw} back-to-back es_switch_context in a CUDA graph",
+                          "share_of_step": round(us * len(local) / 1e3 / ms, 4)}
+
     # ---- parity of the timed outputs against the oracle on sampled windows (+ cpu_baseline) ----
     if rank == 0:
         import oracle  # test infrastructure: the cpu_baseline leg and parity check only
