@@ -39,7 +39,8 @@ def parse():
     p.add_argument("--config", default="resnet50",
                    choices=["tiny", "resnet50", "vgg19", "bert_base", "swin_b"])
     p.add_argument("--mapping", default="contiguous", choices=["contiguous", "round_robin", "random"])
-    p.add_argument("--sched", default="auto", choices=["auto", "direct", "chain", "peer", "peer_chain", "peer_auto"])
+    p.add_argument("--sched", default=None, choices=["auto", "direct", "chain", "peer", "peer_chain", "peer_auto"],
+                   help="default: auto at G=1; peer_auto at G>1 (fused folds over NVLink peer memory, CUDA IPC)")
     p.add_argument("--no-graph", action="store_true", help="eager launches instead of one CUDA graph per step")
     p.add_argument("--per-bucket", action="store_true",
                    help="one es_stash_grad / es_allreduce call per bucket (DDP-style) instead of the batched calls")
@@ -248,6 +249,8 @@ def main():
     args = parse()
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
+    if args.sched is None:
+        args.sched = "peer_auto" if world > 1 else "auto"
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     if args.impl == "reference":
         return run_reference(args, rank, world)
