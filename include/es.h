@@ -164,13 +164,15 @@ typedef struct {
 /* ES_OPT_PEER_ROUNDS: PEER_CHAIN without tile pipelining (a device barrier
  * between rounds).  Same bits; kept for comparison and as a fallback. */
 #define ES_OPT_PEER_ROUNDS 2u
-/* ES_OPT_STASH_BACKGROUND: the kernels that run at an EST's switch (stash,
- * incremental fold) use at most two 256-thread CTAs per SM instead of a
- * one-shot grid.  A one-shot grid of thousands of CTAs is dispatched ahead of
- * any kernel queued after it on another stream, so the model's next forward
- * waits for the whole stash; a one-wave grid leaves the SMs' other slots to
- * it, and the stash streams in the background.  Slightly
- * slower when nothing else runs.  Same bits. */
+/* ES_OPT_STASH_BACKGROUND: stash for overlap with the model's compute
+ * (PAPER.md:599-606).  A one-shot stash grid of thousands of CTAs is
+ * dispatched ahead of any kernel queued after it on another stream, so the
+ * next forward waits for the whole stash, and its CTAs take SM slots a GEMM
+ * needs.  With this option same-dtype stashes run as one warp per SM driving
+ * a 4 x 4 KB TMA bulk-copy ring (16 KB of shared memory: it fits beside a
+ * tensor-core GEMM's CTA); casts, the fused context swap's launch and the
+ * incremental folds use at most two 256-thread CTAs per SM.  About half the
+ * copy bandwidth when nothing else runs.  Same bits. */
 #define ES_OPT_STASH_BACKGROUND 4u
 
 /* NEXT-3 compatibility variants -- same canonical order, different step

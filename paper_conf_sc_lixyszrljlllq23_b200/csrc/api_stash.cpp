@@ -88,7 +88,7 @@ es_status stash_impl(es_handle h, int32_t est, int32_t n, const int32_t *buckets
         const bool early = follows_own_stash(h, cs);
         s = h->timed(ES_KERNEL_STASH, nbytes + (sw ? swap_bytes : 0), cs, [&](int *nl) {
           return es::launch_stash_multi((es_dtype)sd, (es_dtype)dd, segs.data(), (int)segs.size(), cs, h->switch_blocks(),
-                                        h->switch_threads(), nl, sw, early);
+                                        h->switch_threads(), nl, sw, early, h->background());
         });
         if (s != ES_OK) return s;
         remember_stash_node(h, cs);
@@ -210,7 +210,8 @@ es_status es_stash_fold_grads(es_handle h, int32_t est, int32_t n, const int32_t
     if (!st.empty()) {
       s = h->timed(ES_KERNEL_STASH, sbytes, cs, [&](int *nl) {
         return es::launch_stash_multi((es_dtype)dd, (es_dtype)dd, st.data(), (int)st.size(), cs,
-                                      h->switch_blocks(), h->switch_threads(), nl);
+                                      h->switch_blocks(), h->switch_threads(), nl, nullptr, false,
+                                      h->background());
       });
       if (s != ES_OK) return s;
     }

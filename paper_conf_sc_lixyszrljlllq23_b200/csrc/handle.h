@@ -102,10 +102,12 @@ struct es_ctx {
   uint64_t bytes[ES_KERNEL_KINDS] = {};
   double ms[ES_KERNEL_KINDS] = {};
   int blocks_ov = 0, threads_ov = 0;
-  // Grid of the kernels that run at an EST's switch (stash, incremental
-  // fold): ES_OPT_STASH_BACKGROUND caps it (negative = a cap for the
-  // launchers) at two 256-thread CTAs per SM, so the model's kernels queued
-  // behind it are dispatched at once ("Overlap with compute").
+  // ES_OPT_STASH_BACKGROUND: same-dtype stashes run as the small TMA ring
+  // (launch_stash_multi); the other switch-time kernels (casts, incremental
+  // folds) get a grid capped (negative = a cap for the launchers) at two
+  // 256-thread CTAs per SM, so the model's kernels queued behind them are
+  // dispatched at once ("Overlap with compute").
+  bool background() const { return (plan.options & ES_OPT_STASH_BACKGROUND) != 0; }
   int switch_blocks() const {
     return blocks_ov ? blocks_ov : ((plan.options & ES_OPT_STASH_BACKGROUND) ? -2 * 148 : 0);
   }

@@ -122,6 +122,39 @@ __device__ __forceinline__ void st_cs(uint2 *p, const uint2 &v) {
   asm volatile("st.global.cs.v2.u32 [%0], {%1, %2};" ::"l"(p), "r"(v.x), "r"(v.y) : "memory");
 }
 
+// L2 evict-first loads/stores (experiment for the stash, ES_STASH_VARIANT=7:
+// a stream copied once should not push a concurrent kernel's working set out
+// of L2).
+__device__ __forceinline__ uint64_t l2_evict_first_policy() {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+__device__ __forceinline__ int4 ld_ef(const int4 *p, uint64_t pol) {
+  int4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ uint2 ld_ef(const uint2 *p, uint64_t pol) {
+  uint2 r;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0, %1}, [%2], %3;"
+               : "=r"(r.x), "=r"(r.y)
+               : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ void st_ef(int4 *p, const int4 &v, uint64_t pol) {
+  asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.s32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p), "r"(v.x),
+               "r"(v.y), "r"(v.z), "r"(v.w), "l"(pol)
+               : "memory");
+}
+__device__ __forceinline__ void st_ef(uint2 *p, const uint2 &v, uint64_t pol) {
+  asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u32 [%0], {%1, %2}, %3;" ::"l"(p), "r"(v.x), "r"(v.y),
+               "l"(pol)
+               : "memory");
+}
+
 __device__ __forceinline__ uint32_t smem_addr(const void *p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
@@ -903,18 +936,20 @@ __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashPara
     stride = blockDim.x;
     gid = ubeg + threadIdx.x;
   }
+  const uint64_t pol = ST == 2 ? l2_evict_first_policy() : 0;
   for (int64_t u0 = gid; u0 < uend; u0 += stride * kU) {
     In in[kU];
 #pragma unroll
     for (int u = 0; u < kU; ++u) {
       const int64_t i = u0 + u * stride;
-      if (i < uend) in[u] = ld_stream(s + i);
+      if (i < uend) in[u] = ST == 2 ? ld_ef(s + i, pol) : ld_stream(s + i);
     }
 #pragma unroll
     for (int u = 0; u < kU; ++u) {
       const int64_t i = u0 + u * stride;
       if (i < uend) {
         if (ST == 1) st_cs(d + i, Cast<S, D, E>::apply(in[u]));
+        else if (ST == 2) st_ef(d + i, Cast<S, D, E>::apply(in[u]), pol);
         else st_stream(d + i, Cast<S, D, E>::apply(in[u]));
       }
     }
@@ -1006,6 +1041,7 @@ cudaError_t launch_stash_t(const StashSegDesc *segs, int nseg, cudaStream_t s, i
     case 4: return launch_stash_v<S, D, E, 1, 0>(segs, nseg, s, bo, to, launches, swap, early);
     case 5: return launch_stash_v<S, D, E, 4, 0, true>(segs, nseg, s, bo, to, launches, swap, early);
     case 6: return launch_stash_v<S, D, E, 8, 0, true>(segs, nseg, s, bo, to, launches, swap, early);
+    case 7: return launch_stash_v<S, D, E, 4, 2>(segs, nseg, s, bo, to, launches, swap, early);
     default: return launch_stash_v<S, D, E, 4, 0>(segs, nseg, s, bo, to, launches, swap, early);
   }
 }
@@ -1093,16 +1129,22 @@ __global__ void __launch_bounds__(32) k_copy_tma(const __grid_constant__ CopyTma
                  "r"(smem_addr(ring + (size_t)st * T)), "r"(tn[st])
                  : "memory");
     asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-    const unsigned char *ns;
-    unsigned char *nd;
-    uint32_t nn;
-    if (next_tile(ns, nd, nn)) {
-      asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // stage st has been read out
-      tsrc[st] = ns;
-      tdst[st] = nd;
-      tn[st] = nn;
-      load(st);
-      ++loaded;
+    // Refill the stage of the PREVIOUS tile: its store group is the second
+    // most recent, so wait_group.read 1 returns once it has read the stage,
+    // while this tile's store still runs (no load <-> store serialisation).
+    if (i >= 1) {
+      const int ps = (i - 1) % S;
+      const unsigned char *ns;
+      unsigned char *nd;
+      uint32_t nn;
+      if (next_tile(ns, nd, nn)) {
+        asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+        tsrc[ps] = ns;
+        tdst[ps] = nd;
+        tn[ps] = nn;
+        load(ps);
+        ++loaded;
+      }
     }
   }
   asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
@@ -1308,8 +1350,14 @@ cudaError_t launch_fold_multi(es_dtype dtype, int32_t N, float r, uint32_t compa
                              launches);
 }
 
+// ES_BG_TMA=0: ES_OPT_STASH_BACKGROUND without the TMA ring (capped k_stash grid only; experiment)
+int g_bg_tma = [] {
+  const char *e = std::getenv("ES_BG_TMA");
+  return !(e && e[0] == '0');
+}();
+
 cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *segs, int nseg, cudaStream_t s,
-                               int bo, int to, int *launches, const SwapArgs *swap, bool early) {
+                               int bo, int to, int *launches, const SwapArgs *swap, bool early, bool background) {
   int dummy = 0;
   if (!launches) launches = &dummy;
   std::vector<StashSegDesc> live;
@@ -1323,10 +1371,28 @@ cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *s
     return cudaSuccess;
   }
   const int n = (int)live.size();
-  if (sdt == ddt && g_stash_tma > 0 && !(swap && swap->n > 0)) {
+  bool aligned = true;
+  for (const StashSegDesc &g : live)
+    aligned = aligned && !(reinterpret_cast<uintptr_t>(g.src) & 15) && !(reinterpret_cast<uintptr_t>(g.dst) & 15);
+  if (background && g_bg_tma && sdt == ddt && aligned && bo <= 0) {   // bo > 0: an explicit es_set_launch_override
+    // ES_OPT_STASH_BACKGROUND, same dtype: the copy runs as one warp per SM
+    // driving a 4 x 4 KB TMA bulk-copy ring (16 KB of shared memory, a
+    // few registers), a footprint that fits beside a tensor-core GEMM's CTA, so
+    // the stash streams while the model computes (profiles/r01_overlap.md).
+    // The context swap, if any, is its own small launch first.
+    if (swap && swap->n > 0) {
+      ++*launches;
+      cudaError_t e = launch_swap(swap->tab, swap->n, swap->max_nbytes, swap->cur, swap->next, s);
+      if (e != cudaSuccess) return e;
+    }
+    return launch_copy_tma<4, 4096>(live.data(), n, sdt == ES_BF16 ? 2 : 4, s, 1, launches);
+  }
+  if (sdt == ddt && g_stash_tma > 0 && aligned && !(swap && swap->n > 0)) {
     const int es_ = sdt == ES_BF16 ? 2 : 4;
-    return g_stash_tma == 1 ? launch_copy_tma<4, 32768>(live.data(), n, es_, s, 1, launches)
-                            : launch_copy_tma<6, 16384>(live.data(), n, es_, s, 2, launches);
+    // 3: the small-footprint ring of ES_OPT_STASH_BACKGROUND, for every stash
+    return g_stash_tma == 1   ? launch_copy_tma<4, 32768>(live.data(), n, es_, s, 1, launches)
+           : g_stash_tma == 3 ? launch_copy_tma<4, 4096>(live.data(), n, es_, s, 1, launches)
+                              : launch_copy_tma<6, 16384>(live.data(), n, es_, s, 2, launches);
   }
   if (sdt == ES_F32 && ddt == ES_F32) return launch_stash_t<F32T, F32T, 4>(live.data(), n, s, bo, to, launches, swap, early);
   if (sdt == ES_BF16 && ddt == ES_BF16)

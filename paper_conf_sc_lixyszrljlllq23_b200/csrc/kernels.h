@@ -88,7 +88,7 @@ struct SwapArgs {
 // exiting (completion order stays transitive); swap blocks always wait first.
 cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *segs, int nseg, cudaStream_t s,
                                int blocks_override, int threads_override, int *launches,
-                               const SwapArgs *swap = nullptr, bool early = false);
+                               const SwapArgs *swap = nullptr, bool early = false, bool background = false);
 
 // One launch: for every entry, slot[cur] <- live, live <- slot[next]
 // (cur < 0: load only).  max_nbytes sizes the grid.

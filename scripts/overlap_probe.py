@@ -135,6 +135,9 @@ def main():
         ev_grad = [torch.cuda.Event() for _ in range(N)]
         ev_stash = [torch.cuda.Event() for _ in range(N)]
         ev_done = torch.cuda.Event()
+        # per EST: aggregation-stream busy time (stash start -> stash done), last step only
+        ev_s0 = [torch.cuda.Event(enable_timing=True) for _ in range(N)]
+        ev_s1 = [torch.cuda.Event(enable_timing=True) for _ in range(N)]
 
         def step(t0, t_last, t1):
             with torch.cuda.stream(sc):
@@ -155,6 +158,7 @@ def main():
                         continue
                     with torch.cuda.stream(sa):
                         sa.wait_event(ev_grad[k])
+                        ev_s0[k].record(sa)
                         last = k == N - 1
                         if base_mode == "copy":
                             agg.stash_many(k, range(B), live, es.ES_STASH_BORROW if last else es.ES_STASH_COPY,
@@ -171,6 +175,7 @@ def main():
                         else:
                             agg.stash_many(k, range(B), dst, es.ES_STASH_INPLACE, stream=sa)
                         ev_stash[k].record(sa)
+                        ev_s1[k].record(sa)
                 t_last.record(sc)
                 if base_mode != "none":
                     sa.wait_event(ev_grad[N - 1])
@@ -179,10 +184,13 @@ def main():
                         ev_done.record(sa)
                     sc.wait_event(ev_done)
                 t1.record(sc)
-        return {"agg": agg, "outs": outs, "step": step}
+        def stash_ms():
+            return sum(a.elapsed_time(b) for a, b in zip(ev_s0, ev_s1)) if base_mode != "none" else 0.0
+        return {"agg": agg, "outs": outs, "step": step, "stash_ms": stash_ms}
 
     ctx = {m: make(m) for m in modes}
-    times = {m: [] for m in modes}                   # (step, tail) per timed step
+    times = {m: [] for m in modes}
+    stash_t = {}                   # (step, tail) per timed step
     for r in range(args.rounds):                     # modes interleaved: clock/power drift hits all alike
         for m in modes:
             ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.warmup + args.steps)]
@@ -190,6 +198,7 @@ def main():
                 ctx[m]["step"](*ev[i])
             torch.cuda.synchronize()
             times[m] += [(e[0].elapsed_time(e[2]), e[1].elapsed_time(e[2])) for e in ev[args.warmup:]]
+            stash_t.setdefault(m, []).append(ctx[m]["stash_ms"]())
     results, ref = [], None
 
     def block_medians(m):
@@ -203,7 +212,8 @@ def main():
         res = {"mode": m, "step_ms": round(statistics.median(t for t, _ in times[m]), 4),
                "exposed_ms": round(statistics.median(d), 4),
                "exposed_min_max_ms": [round(d[0], 4), round(d[-1], 4)],
-               "tail_ms": round(statistics.median(t for _, t in times[m]), 4)}
+               "tail_ms": round(statistics.median(t for _, t in times[m]), 4),
+               "stash_stream_busy_ms": round(statistics.median(stash_t[m]), 4)}
         if m != "none":
             got = ctx[m]["outs"]
             if ref is None:
