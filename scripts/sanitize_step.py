@@ -29,10 +29,10 @@ def data(rng, N, Ls, dts):
     return xs
 
 
-def g1(rng):
+def g1(rng, options=0):
     N, Ls, dts = 5, [1001, 17, 64, 3], ["f32", "bf16", "f32", "bf16"]
     sizes = [16, 4096, 37]
-    agg = Aggregator(N, 1, 0, [0] * N, list(zip(Ls, dts)), state_nbytes=sizes)
+    agg = Aggregator(N, 1, 0, [0] * N, list(zip(Ls, dts)), state_nbytes=sizes, options=options)
     live = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in sizes]
     agg.register_state(live)
     for k in range(N):
@@ -55,7 +55,7 @@ def g1(rng):
     blob = agg.export_context(2)
     agg.import_context(2, blob)
     agg.close()
-    inc = Aggregator(N, 1, 0, [0] * N, list(zip(Ls, dts)), options=es.ES_OPT_INCREMENTAL)
+    inc = Aggregator(N, 1, 0, [0] * N, list(zip(Ls, dts)), options=options | es.ES_OPT_INCREMENTAL)
     for k in range(N):
         inc.stash_fold(k, range(len(Ls)), devs[k])
     inc.allreduce_many(range(len(Ls)), outs)
@@ -65,13 +65,13 @@ def g1(rng):
     inc.close()
 
 
-def multi(rng, sched):
+def multi(rng, sched, options=0):
     N, G, m = 6, 3, [0, 1, 2, 2, 0, 1]
     Ls, dts = [1003, 40, 9], ["f32", "bf16", "f32"]
     xs = data(rng, N, Ls, dts)
     world = es.es_loopback_create(G)
     aggs = [Aggregator(N, G, g, m, list(zip(Ls, dts)), transport=es.ES_TRANSPORT_LOOPBACK, comm=world.value,
-                       sched=sched) for g in range(G)]
+                       sched=sched, options=options) for g in range(G)]
     if sched in es.PEER_SCHEDS:
         blobs = [a.peer_blob() for a in aggs]
         for a in aggs:
@@ -106,9 +106,20 @@ def multi(rng, sched):
     es.es_loopback_destroy(world)
 
 
+SCHEDS = {"direct": (es.ES_SCHED_DIRECT, 0), "chain": (es.ES_SCHED_CHAIN, 0), "peer": (es.ES_SCHED_PEER, 0),
+          "peer_chain": (es.ES_SCHED_PEER_CHAIN, 0),
+          "peer_chain_rounds": (es.ES_SCHED_PEER_CHAIN, es.ES_OPT_PEER_ROUNDS)}
+
 if __name__ == "__main__":
+    # argv: which parts to run (default: all): g1 g1_bg direct chain peer peer_chain peer_chain_rounds
+    parts = sys.argv[1:] or ["g1", "g1_bg"] + list(SCHEDS)
     rng = np.random.default_rng(0)
-    g1(rng)
-    for sched in (es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_PEER, es.ES_SCHED_PEER_CHAIN):
-        multi(rng, sched)
+    for part in parts:
+        if part == "g1":
+            g1(rng)
+        elif part == "g1_bg":
+            g1(rng, es.ES_OPT_STASH_BACKGROUND)    # TMA-ring stash (k_copy_tma<4, 4096>) and capped grids
+        else:
+            multi(rng, *SCHEDS[part])
+        print("part ok:", part, flush=True)
     print("sanitize_step ok")
