@@ -8,6 +8,10 @@
 the profiled time (cold-cache, serialised -- compare shares, not absolutes).
 `full`: the key `--set full` metrics per profiled launch (duration, DRAM
 bytes read/written, DRAM throughput, occupancy, registers, stall summary).
+`traffic`: python scripts/ncu_summary.py traffic <config> [G]  reads
+gpurun_out/full_{fold,stash}_<config>.ncu-rep and writes
+profiles/traffic_<config>_g<G>.json (dram read + write bytes per launch), which
+bench.py reports as roofline.traffic.
 """
 import collections
 import csv
@@ -75,5 +79,34 @@ def full(path):
         print("```json\n" + json.dumps(d, indent=1) + "\n```")
 
 
+def _raw(path):
+    out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(io.StringIO(out)))
+    return rows[0], rows[1], rows[2:]
+
+
+def _bytes(v, unit):
+    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}[unit]
+    return int(round(float(v.replace(",", "")) * scale))
+
+
+def traffic(config, G="1"):
+    d = {}
+    for kname, tag in (("k_fold", "fold"), ("k_stash", "stash")):
+        rep = f"gpurun_out/full_{tag}_{config}.ncu-rep"
+        hdr, units, rows = _raw(rep)
+        r = rows[0]
+        rd, wr = hdr.index("dram__bytes_read.sum"), hdr.index("dram__bytes_write.sum")
+        d[f"{kname}_dram_bytes_per_launch"] = _bytes(r[rd], units[rd]) + _bytes(r[wr], units[wr])
+    d["source"] = (f"ncu --set full (profiles/r01_k_fold_full_{config}.md, r01_k_stash_full_{config}.md): "
+                   "dram__bytes_read.sum + dram__bytes_write.sum per launch, cold cache; writes still dirty "
+                   "in L2 at kernel end are not counted")
+    path = f"profiles/traffic_{config}_g{G}.json"
+    with open(path, "w") as f:
+        json.dump(d, f, indent=1)
+        f.write("\n")
+    print(path, d)
+
+
 if __name__ == "__main__":
-    {"launches": launches, "full": full}[sys.argv[1]](sys.argv[2])
+    {"launches": launches, "full": full, "traffic": traffic}[sys.argv[1]](*sys.argv[2:])
