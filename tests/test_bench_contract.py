@@ -56,6 +56,7 @@ def test_main_arm_line_keys():
     assert {"value", "unit", "cores", "kind", "sample"} <= set(d["cpu_baseline"]) and d["cpu_baseline"]["kind"] == "oracle"
     e = d["e2e"]
     assert e["value"] > 0 and e["h2d_bytes_per_step"] == 4 * 1048576 * 4 and e["d2h_bytes_per_step"] == 4 * 1048576
+    assert e["roofline"]["bound"] == "pcie_h2d" and e["roofline"]["peak"] > 0 and 0 < e["roofline"]["frac"] < 1.5
     assert d["gpu_launches"] > 0 and {"sm_mhz", "sm_max_mhz", "reasons"} <= set(d["clocks"])
     assert d["parity"]["mismatched_words"] == 0 and d["parity"]["full_output_mismatched_words"] == 0
     assert d["parity"]["sha256_equal"] is True and d["switch"]["us_per_switch"] > 0
