@@ -191,6 +191,7 @@ es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *c
 }  // namespace
 
 es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void *const *outs, es_stream stream) {
+  ES_NVTX();
   es_status s = check_handle(h);
   if (s != ES_OK) return s;
   const es::Plan &p = h->plan;

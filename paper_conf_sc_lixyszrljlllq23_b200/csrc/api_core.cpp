@@ -57,6 +57,7 @@ es_status es_plan_ops(const es_config *cfg, int32_t bucket, int64_t *ops, size_t
 }
 
 es_status es_init(const es_config *cfg, void *workspace, size_t workspace_bytes, es_handle *out) {
+  ES_NVTX();
   if (!out) return set_err(ES_EINVAL, "out is NULL");
   *out = nullptr;
   std::unique_ptr<es_ctx> h(new es_ctx());
@@ -126,6 +127,7 @@ es_status es_init(const es_config *cfg, void *workspace, size_t workspace_bytes,
 }
 
 es_status es_destroy(es_handle h) {
+  ES_NVTX();
   if (!h) return set_err(ES_EINVAL, "handle is NULL");
   delete h;
   return ES_OK;
@@ -201,6 +203,7 @@ es_status es_read_state(es_handle h, int32_t est, int32_t idx, void *host_dst) {
 }
 
 es_status es_switch_context(es_handle h, int32_t est, es_stream stream) {
+  ES_NVTX();
   es_status s = check_handle(h);
   if (s != ES_OK) return s;
   const es::Plan &p = h->plan;

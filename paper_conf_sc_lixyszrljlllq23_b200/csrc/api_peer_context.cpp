@@ -70,6 +70,7 @@ es_status es_peer_blob(es_handle h, void *blob, size_t bytes) {
 }
 
 es_status es_peer_open(es_handle h, const void *blobs, size_t bytes) {
+  ES_NVTX();
   es_status s = check_handle(h);
   if (s != ES_OK) return s;
   const es::Plan &p = h->plan;
@@ -204,6 +205,7 @@ es_status es_context_bytes(es_handle h, size_t *bytes) {
 }
 
 es_status es_export_context(es_handle h, int32_t est, void *host_dst, size_t bytes, es_stream stream) {
+  ES_NVTX();
   es_status s = check_handle(h);
   if (s != ES_OK) return s;
   const es::Plan &p = h->plan;
@@ -262,6 +264,7 @@ es_status es_export_context(es_handle h, int32_t est, void *host_dst, size_t byt
 }
 
 es_status es_import_context(es_handle h, int32_t est, const void *host_src, size_t bytes, es_stream stream) {
+  ES_NVTX();
   es_status s = check_handle(h);
   if (s != ES_OK) return s;
   const es::Plan &p = h->plan;
@@ -318,6 +321,7 @@ es_status es_import_context(es_handle h, int32_t est, const void *host_src, size
 
 es_status es_dropout(es_handle h, const void *x, void *y, uint8_t *mask, uint64_t n, es_dtype dtype, float p,
                      int32_t state_idx, es_stream stream) {
+  ES_NVTX();
   es_status s = check_handle(h);
   if (s != ES_OK) return s;
   const es::Plan &pl = h->plan;

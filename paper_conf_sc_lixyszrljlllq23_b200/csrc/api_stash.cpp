@@ -117,11 +117,13 @@ es_status stash_impl(es_handle h, int32_t est, int32_t n, const int32_t *buckets
 
 es_status es_stash_grads(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
                          const es_dtype *gdts, es_stash_mode mode, es_stream stream) {
+  ES_NVTX();
   return stash_impl(h, est, n, buckets, grads, gdts, mode, -1, stream);
 }
 
 es_status es_stash_fold_grads(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
                               const es_dtype *gdts, es_stash_mode mode, es_stream stream) {
+  ES_NVTX();
   es_status s = check_handle(h);
   if (s != ES_OK) return s;
   const es::Plan &p = h->plan;
@@ -229,12 +231,14 @@ es_status es_stash_fold_grads(es_handle h, int32_t est, int32_t n, const int32_t
 
 es_status es_stash_and_switch(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
                               const es_dtype *gdts, es_stash_mode mode, int32_t next_est, es_stream stream) {
+  ES_NVTX();
   if (next_est < 0) return set_err(ES_EINVAL, "next_est must be a valid EST (use es_stash_grads to only stash)");
   return stash_impl(h, est, n, buckets, grads, gdts, mode, next_est, stream);
 }
 
 es_status es_stash_grad(es_handle h, int32_t est, int32_t bucket, const void *grad, es_dtype gdt, es_stash_mode mode,
                         es_stream stream) {
+  ES_NVTX();
   return stash_impl(h, est, 1, &bucket, &grad, &gdt, mode, -1, stream);
 }
 

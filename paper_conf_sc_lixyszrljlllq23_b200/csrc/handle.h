@@ -4,6 +4,7 @@
 #pragma once
 
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <algorithm>
 #include <cstring>
@@ -24,6 +25,17 @@ inline es_status set_err(es_status s, const std::string &msg) {
   g_err = msg;
   return s;
 }
+
+// Tracing: one NVTX range per C-ABI call that enqueues work, named after the call, so
+// nsys timelines and `ncu --nvtx` filters see the stash / switch / allreduce structure of a step.
+// NVTX v3 is header-only; without an attached tool a range costs one predictable branch.
+struct NvtxRange {
+  explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+  NvtxRange(const NvtxRange &) = delete;
+  NvtxRange &operator=(const NvtxRange &) = delete;
+};
+#define ES_NVTX() ::es_detail::NvtxRange es_nvtx_range_(__func__)
 
 inline bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
