@@ -23,3 +23,10 @@ for c in $CONFIGS; do
       -o gpurun_out/full_stash_$c $B --config $c > gpurun_out/full_stash_$c.log 2>&1
   echo "$c done: $(ls gpurun_out/*_$c* | tr '\n' ' ')"
 done
+# The default bench command itself (CUDA graph, PDL, early-start stashes) for the default workload:
+# the first 2 eager warm-up steps + the graph replays after them, 9 of our launches per ResNet-50 step.
+if [[ " $CONFIGS " == *" resnet50 "* ]]; then
+  timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k 'regex:k_(fold|stash|swap)' \
+      -c 90 --csv --log-file gpurun_out/launches_resnet50_default_cmd.csv python bench.py --steps 5 --warmup 3 \
+      > gpurun_out/launches_resnet50_default_cmd.log 2>&1
+fi
