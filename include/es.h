@@ -37,6 +37,9 @@
  *     for the most recent failing call on this thread.
  *   - A handle is not thread-safe; use one handle per thread (one per GPU
  *     rank).  Different handles may be used concurrently.
+ *   - Every call that enqueues device work is an NVTX range named after the
+ *     call ("es_stash_and_switch", "es_allreduce_many", ...) for nsys / ncu
+ *     filtering (NVTX v3; a no-op when no tool is attached).
  */
 #ifndef ES_H
 #define ES_H
