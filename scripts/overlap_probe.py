@@ -25,9 +25,16 @@ modes: base[+flag...]
   copy_ce      diagnostic: the slot copy by cudaMemcpyAsync (copy engines, no
                SMs) on the aggregation stream, then ES_STASH_INPLACE
 flags
+  +bk          DDP-style buckets (copy / inplace): the backward is split into one slice per bucket
+               and bucket b's gradient is written after its slice (buckets are in reverse layer
+               order, as DDP fills them); each bucket is stashed as soon as it is written, and for
+               the last EST es_allreduce(b) is launched as soon as its bucket b is written, so the
+               folds of all but the last bucket overlap the last EST's backward
   +bg          ES_OPT_STASH_BACKGROUND (stash / incremental-fold grids of one wave)
   +lp          compute stream at high priority (the aggregation fills the gaps)
   +hp          aggregation stream at high priority
+  +ovK         es_set_launch_override(148*K, 256): every libes launch (stash, fold) is a grid of
+               K CTAs per SM (grid-stride), leaving SM slots to the compute stream
 
 Reported per mode: step ms, exposed ms = median over rounds of (this mode's
 median step - the compute-only median of the same round), tail ms = last gradient
@@ -127,6 +134,9 @@ def main():
         agg = Aggregator(N, 1, 0, [0] * N, buckets, state_nbytes=snb, device=dev,
                          options=opts)
         agg.register_state(state)
+        for f in flags:                               # +ovK: every launch capped at K 256-thread CTAs per SM
+            if f.startswith("ov"):
+                agg.set_launch_override(148 * int(f[2:]), 256)
         for k in range(N):
             for i, blob in enumerate(workloads.est_state(args.config, k)):
                 agg.init_state(k, i, blob)
@@ -138,16 +148,64 @@ def main():
         # per EST: aggregation-stream busy time (stash start -> stash done), last step only
         ev_s0 = [torch.cuda.Event(enable_timing=True) for _ in range(N)]
         ev_s1 = [torch.cuda.Event(enable_timing=True) for _ in range(N)]
+        # compute-stream time per EST (switch .. last gradient written), last step only
+        ev_est = [torch.cuda.Event(enable_timing=True) for _ in range(N + 1)]
+
+        bucketed = "bk" in flags and base_mode in ("copy", "inplace")
+        n_bwd = 2 * n_fwd
+        bwd_slices = [n_bwd * (j + 1) // B - n_bwd * j // B for j in range(B)]
+        ev_gb = [[torch.cuda.Event() for _ in range(B)] for _ in range(N)]      # bucket written
+        ev_sb = [[torch.cuda.Event() for _ in range(B)] for _ in range(N)]      # bucket stashed
+
+        def step_bucketed(t0, t_last, t1):
+            # DDP-style: per-bucket gradient readiness inside each EST's backward
+            with torch.cuda.stream(sc):
+                t0.record(sc)
+                sc.wait_event(ev_done)
+                for k in range(N):
+                    last = k == N - 1
+                    ev_est[k].record(sc)
+                    agg.switch(k, stream=sc)
+                    compute(n_fwd)
+                    for b in range(B):
+                        compute(bwd_slices[b])
+                        if base_mode == "copy" and k > 0:
+                            sc.wait_event(ev_sb[k - 1][b])           # EST k-1's bucket b left the live buffer
+                        dst = slots[k][b] if base_mode == "inplace" else live[b]
+                        dst.copy_(src[k][b])
+                        ev_gb[k][b].record(sc)
+                        with torch.cuda.stream(sa):
+                            sa.wait_event(ev_gb[k][b])
+                            if b == 0:
+                                ev_s0[k].record(sa)
+                            mode_b = es.ES_STASH_INPLACE if base_mode == "inplace" else \
+                                (es.ES_STASH_BORROW if last else es.ES_STASH_COPY)
+                            agg.stash_many(k, [b], [dst], mode_b, stream=sa)
+                            ev_sb[k][b].record(sa)
+                            if last:
+                                agg.allreduce_many([b], [outs[b]], stream=sa)
+                            if b == B - 1:
+                                ev_s1[k].record(sa)
+                ev_est[N].record(sc)
+                t_last.record(sc)
+                with torch.cuda.stream(sa):
+                    ev_done.record(sa)
+                sc.wait_event(ev_done)
+                t1.record(sc)
 
         def step(t0, t_last, t1):
+            if bucketed:
+                return step_bucketed(t0, t_last, t1)
             with torch.cuda.stream(sc):
                 t0.record(sc)
                 sc.wait_event(ev_done)                # previous step's allreduce (BORROW / slots)
                 for k in range(N):
+                    ev_est[k].record(sc)
                     if base_mode != "none":
                         agg.switch(k, stream=sc)
                     compute(n_fwd)
-                    compute(2 * n_fwd)
+                    for b in range(B):                        # the backward in B slices in every mode,
+                        compute(bwd_slices[b])                # so +bk adds no kernel boundaries
                     if base_mode in ("copy", "incremental", "copy_ce") and k > 0:
                         sc.wait_event(ev_stash[k - 1])    # the live buffer is free again
                     dst = slots[k] if base_mode == "inplace" else live
@@ -176,6 +234,7 @@ def main():
                             agg.stash_many(k, range(B), dst, es.ES_STASH_INPLACE, stream=sa)
                         ev_stash[k].record(sa)
                         ev_s1[k].record(sa)
+                ev_est[N].record(sc)
                 t_last.record(sc)
                 if base_mode != "none":
                     sa.wait_event(ev_grad[N - 1])
@@ -186,11 +245,15 @@ def main():
                 t1.record(sc)
         def stash_ms():
             return sum(a.elapsed_time(b) for a, b in zip(ev_s0, ev_s1)) if base_mode != "none" else 0.0
-        return {"agg": agg, "outs": outs, "step": step, "stash_ms": stash_ms}
+        def est_ms():
+            d = [ev_est[k].elapsed_time(ev_est[k + 1]) for k in range(N)]
+            return [d[0], statistics.median(d[1:-1]) if N > 2 else 0.0, d[-1]]
+        return {"agg": agg, "outs": outs, "step": step, "stash_ms": stash_ms, "est_ms": est_ms}
 
     ctx = {m: make(m) for m in modes}
     times = {m: [] for m in modes}
     stash_t = {}                   # (step, tail) per timed step
+    est_t = {}                     # [first, median middle, last] EST compute-stream ms, last step per round
     for r in range(args.rounds):                     # modes interleaved: clock/power drift hits all alike
         for m in modes:
             ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.warmup + args.steps)]
@@ -199,6 +262,7 @@ def main():
             torch.cuda.synchronize()
             times[m] += [(e[0].elapsed_time(e[2]), e[1].elapsed_time(e[2])) for e in ev[args.warmup:]]
             stash_t.setdefault(m, []).append(ctx[m]["stash_ms"]())
+            est_t.setdefault(m, []).append(ctx[m]["est_ms"]())
     results, ref = [], None
 
     def block_medians(m):
@@ -213,7 +277,8 @@ def main():
                "exposed_ms": round(statistics.median(d), 4),
                "exposed_min_max_ms": [round(d[0], 4), round(d[-1], 4)],
                "tail_ms": round(statistics.median(t for _, t in times[m]), 4),
-               "stash_stream_busy_ms": round(statistics.median(stash_t[m]), 4)}
+               "stash_stream_busy_ms": round(statistics.median(stash_t[m]), 4),
+               "est_ms_first_mid_last": [round(statistics.median(e[i] for e in est_t[m]), 4) for i in range(3)]}
         if m != "none":
             got = ctx[m]["outs"]
             if ref is None:
