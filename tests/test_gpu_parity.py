@@ -191,6 +191,36 @@ def test_borrow_equals_copy_and_out_aliasing():
     agg.close()
 
 
+@pytest.mark.parametrize("options", [0, es.ES_OPT_STASH_BACKGROUND])
+def test_per_bucket_allreduce_interleaved_with_last_stashes(options):
+    """DDP-style bucket overlap (profiles/r01_overlap.md, +bk): the last EST stashes bucket b and
+    es_allreduce(b) runs at once, before its later buckets exist; earlier ESTs stash per bucket
+    on a side stream in the order their buckets become ready.  Every bucket equals the oracle."""
+    from gpu_util import Aggregator, to_dev, from_dev
+    rng = np.random.default_rng(21)
+    N = 5
+    sizes = [(40003, "f32"), (777, "bf16"), (123457, "f32"), (16, "bf16")]
+    xs = [_gauss(rng, N, L, d) for L, d in sizes]
+    agg = Aggregator(N, 1, 0, [0] * N, sizes, options=options)
+    side = torch.cuda.Stream()
+    outs = [agg.new_out(b) for b in range(len(sizes))]
+    devs = [[to_dev(xs[b][k]) for b in range(len(sizes))] for k in range(N)]
+    torch.cuda.synchronize()
+    with torch.cuda.stream(side):
+        for k in range(N):
+            for b in range(len(sizes)):
+                if k < N - 1:
+                    agg.stash(k, b, devs[k][b])
+                else:
+                    agg.stash(k, b, devs[k][b], es.ES_STASH_BORROW)
+                    agg.allreduce(b, outs[b])
+    torch.cuda.synchronize()
+    agg.sync()
+    for b, (L, d) in enumerate(sizes):
+        assert_bits_equal(from_dev(outs[b]), oracle.reduce(xs[b], d), f"bucket {b}")
+    agg.close()
+
+
 # ---- G > 1 over the loopback transport (one GPU, every mapping) ------------------------------
 
 def _surjections(N, G):
