@@ -28,6 +28,7 @@ sys.path.insert(0, ROOT)
 
 METRIC = "EST-gradient GB/s reduced (bit-exact across G) at 1/2/4/8 B200; % of roofline"
 L2_BYTES = 126 * 1024 * 1024
+HBM_NOMINAL_GBPS = 8000.0     # B200 HBM3e nominal (SURVEY 8(d) t_roof uses 8.0 TB/s); `frac` uses the measured peak
 
 
 def parse():
@@ -489,7 +490,8 @@ def main():
                 "frac": round(a / peak, 4), "traffic": traffic_all.get(f"{kname}_dram_bytes_per_launch"),
                 "algorithmic_bytes_per_launch": int(bytes_ / n_), "launches_per_step": int(n_ / steps_profiled),
                 "avg_launch_us": round(us, 2), "timing": how, "avg_launch_us_event_pairs": round(ev_us, 2),
-                "share_of_step": round(us * n_ / steps_profiled / 1e3 / ms, 3), "peak_source": peak_src}
+                "share_of_step": round(us * n_ / steps_profiled / 1e3 / ms, 3), "peak_source": peak_src,
+                "frac_of_nominal": round(a / HBM_NOMINAL_GBPS, 4)}
 
     roofs = {k: r for k, r in (("k_fold", roof("fold", "k_fold")), ("k_stash", roof("stash", "k_stash")),
                                ("k_gather", roof("gather", "k_gather"))) if r is not None}
@@ -516,7 +518,9 @@ def main():
         "step_roofline": {"achieved": round(sum(v[2] for v in prof.values()) / steps_profiled / (ms / 1e3) / 1e9, 1),
                           "peak": peak, "unit": "GB/s",
                           "frac": round(sum(v[2] for v in prof.values()) / steps_profiled / (ms / 1e3) / 1e9 / peak, 4),
-                          "bytes_per_step": int(sum(v[2] for v in prof.values()) / steps_profiled)},
+                          "bytes_per_step": int(sum(v[2] for v in prof.values()) / steps_profiled),
+                          "frac_of_nominal": round(sum(v[2] for v in prof.values()) / steps_profiled / (ms / 1e3) / 1e9
+                                                   / HBM_NOMINAL_GBPS, 4)},
         "breakdown_ms_per_step": {k: round(v[1] / steps_profiled, 4) for k, v in prof.items()},
         "per_kernel": {k: {"launches_per_step": int(v[0] / steps_profiled),
                            "algorithmic_GBps": round(v[2] / (v[1] / 1e3) / 1e9, 1) if v[1] > 0 else None,
