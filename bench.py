@@ -388,10 +388,11 @@ def main():
     graph = graph_prof = graph_phase = None
     marks = [torch.cuda.Event(enable_timing=True, external=use_graph) for _ in range(3)]
     if use_graph:
-        # Three captures of the same step: without timing events (the steps we
-        # time), with phase-boundary events only (second-to-last timed step:
-        # stash and allreduce phases with every overlap intact), and with
-        # per-kernel event nodes (the last timed step: per-kind durations).
+        # Three captures of the same step: without timing events (the K steps
+        # we time), with phase-boundary events only (replayed once after the
+        # timed region: stash and allreduce phases with every overlap intact),
+        # and with per-kernel event nodes (replayed once after that: per-kind
+        # durations).
         graph = torch.cuda.CUDAGraph()
         with torch.cuda.graph(graph, stream=stream):
             step()
@@ -435,13 +436,23 @@ def main():
                 flush_sink.copy_(flush_words.amax())   # drained here, not inside the next timed step
             starts[i].record(stream)
             if graph is not None:
-                g_ = graph_prof if i == args.steps - 1 else (graph_phase if i == args.steps - 2 else graph)
-                g_.replay()
+                graph.replay()                    # the K timed steps carry no instrumentation
             else:
                 step(marks if i == args.steps - 2 else None)
             ends[i].record(stream)
     torch.cuda.synchronize()
     t_end = time.time()
+    if graph is not None:
+        # after (outside) the timed region, in the same steady state (queued back to back behind
+        # plain replays, no host sync in between): one replay with phase-boundary events, one with
+        # per-kernel event pairs, each prepared like a timed step
+        with torch.cuda.stream(stream):
+            for g_ in (graph, graph, graph_phase, graph, graph_prof):
+                if flush is not None:
+                    flush.zero_()
+                    flush_sink.copy_(flush_words.amax())
+                g_.replay()
+        torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     clk = clocks.stop(t_start, t_end)
@@ -473,7 +484,7 @@ def main():
     # boundaries of one timed step, no event between kernels, so early start and PDL overlap stay
     # intact.  The per-kernel event pairs of the profiled step add ~1-5 us per launch.
     phase_ms = None
-    if fuse and G == 1 and args.steps >= 2:
+    if fuse and G == 1 and (graph is not None or args.steps >= 2):
         phase_ms = {"stash": marks[0].elapsed_time(marks[1]), "fold": marks[1].elapsed_time(marks[2])}
 
     def roof(kind, kname):
