@@ -114,6 +114,40 @@ __global__ void __launch_bounds__(256) k_foldpat(const __grid_constant__ Srcs s,
   }
 }
 
+// bf16 fold pattern (BERT: N = 12): 8 bf16 per 16-B vector widened to fp32, folded, rounded back;
+// sources loaded in batches of BATCH (k_fold uses 8: 8 + 4 for N = 12).
+template <int BATCH>
+__global__ void __launch_bounds__(256) k_foldpat_bf16(const __grid_constant__ Srcs s, int N, uint16_t *out,
+                                                     int64_t nvec) {
+  const int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (v >= nvec) return;
+  float acc[8];
+#pragma unroll
+  for (int e = 0; e < 8; ++e) acc[e] = 0.f;
+  for (int k0 = 0; k0 < N; k0 += BATCH) {
+    int4 buf[BATCH];
+#pragma unroll
+    for (int b = 0; b < BATCH; ++b)
+      buf[b] = k0 + b < N ? ldnc(reinterpret_cast<const int4 *>(s.p[k0 + b]) + v) : make_int4(0, 0, 0, 0);
+#pragma unroll
+    for (int b = 0; b < BATCH; ++b) {
+      if (k0 + b < N) {
+        const uint32_t w[4] = {(uint32_t)buf[b].x, (uint32_t)buf[b].y, (uint32_t)buf[b].z, (uint32_t)buf[b].w};
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          acc[2 * q] = __fadd_rn(acc[2 * q], __uint_as_float(w[q] << 16));
+          acc[2 * q + 1] = __fadd_rn(acc[2 * q + 1], __uint_as_float(w[q] & 0xffff0000u));
+        }
+      }
+    }
+  }
+  uint32_t o[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q)
+    o[q] = (__float_as_uint(acc[2 * q]) >> 16) | (__float_as_uint(acc[2 * q + 1]) & 0xffff0000u);
+  stna(reinterpret_cast<int4 *>(out) + v, make_int4(o[0], o[1], o[2], o[3]));
+}
+
 template <typename F>
 static float best_ms(F f, int reps = 10) {
   cudaEvent_t a, b;
@@ -174,6 +208,22 @@ int main() {
              "\"U1_nowrite_read_GBps\": %.1f}\n", N, g1, alg / (m1 * 1e-3) / 1e9, alg / (m2 * 1e-3) / 1e9,
              rd / (r1 * 1e-3) / 1e9);
     }
+  }
+  {  // bf16, N = 12 (BERT), one-shot grid
+    const int N = 12;
+    const int64_t L = (bytes / 2) / N / 8 * 8;     // bf16 elements per source
+    Srcs s;
+    for (int k = 0; k < N; ++k) s.p[k] = reinterpret_cast<const float *>(a + (size_t)k * L * 2);
+    const int64_t nv = L / 8;
+    const double alg = (double)(N + 1) * L * 2;
+    const int g = (int)((nv + 255) / 256);
+    float m8 = best_ms([&] { k_foldpat_bf16<8><<<g, 256>>>(s, N, (uint16_t *)b, nv); });
+    float m6 = best_ms([&] { k_foldpat_bf16<6><<<g, 256>>>(s, N, (uint16_t *)b, nv); });
+    float m12 = best_ms([&] { k_foldpat_bf16<12><<<g, 256>>>(s, N, (uint16_t *)b, nv); });
+    float m4 = best_ms([&] { k_foldpat_bf16<4><<<g, 256>>>(s, N, (uint16_t *)b, nv); });
+    printf("{\"probe\": \"foldpat_bf16_oneshot\", \"N\": %d, \"grid\": %d, \"B8_GBps\": %.1f, \"B6_GBps\": %.1f, "
+           "\"B12_GBps\": %.1f, \"B4_GBps\": %.1f}\n", N, g, alg / (m8 * 1e-3) / 1e9, alg / (m6 * 1e-3) / 1e9,
+           alg / (m12 * 1e-3) / 1e9, alg / (m4 * 1e-3) / 1e9);
   }
   CK(cudaGetLastError());
   return 0;
