@@ -32,6 +32,7 @@
 #include <algorithm>
 #include <cstdio>
 #include <cstdlib>
+#include <type_traits>
 #include <vector>
 
 namespace es {
@@ -906,7 +907,7 @@ int swap_blocks_per_entry(uint64_t max_nbytes) {
   return (int)std::max<uint64_t>(1, std::min<uint64_t>((words + 255) / 256, 64));
 }
 
-template <typename S, typename D, int E, int kU, int MAXSEG, int ST, bool CR = false>
+template <typename S, typename D, int E, int kU, int MAXSEG, int ST, bool CR = false, bool WC = false>
 __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashParams<MAXSEG> p) {
   using In = typename VecT<S::kSize * E>::T;
   using Out = typename VecT<D::kSize * E>::T;
@@ -937,7 +938,21 @@ __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashPara
     gid = ubeg + threadIdx.x;
   }
   const uint64_t pol = ST == 2 ? l2_evict_first_policy() : 0;
-  for (int64_t u0 = gid; u0 < uend; u0 += stride * kU) {
+  if (WC) {   // warp-contiguous: a warp's kU units are 32*kU adjacent units (one 512*kU-byte run)
+    const int lane = threadIdx.x & 31;
+    const int64_t nwarps = stride >> 5;
+    for (int64_t w0 = gid >> 5; w0 * 32 * kU < uend; w0 += nwarps) {
+      const int64_t base = w0 * 32 * kU + lane;
+      In in[kU];
+#pragma unroll
+      for (int u = 0; u < kU; ++u)
+        if (base + 32 * u < uend) in[u] = ld_stream(s + base + 32 * u);
+#pragma unroll
+      for (int u = 0; u < kU; ++u)
+        if (base + 32 * u < uend) st_stream(d + base + 32 * u, Cast<S, D, E>::apply(in[u]));
+    }
+  }
+  for (int64_t u0 = gid; !WC && u0 < uend; u0 += stride * kU) {
     In in[kU];
 #pragma unroll
     for (int u = 0; u < kU; ++u) {
@@ -968,7 +983,7 @@ __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashPara
   if (p.early) pdl_wait();   // complete only after the predecessor: keeps completion order transitive
 }
 
-template <typename S, typename D, int E, int kU, int ST, bool CR = false>
+template <typename S, typename D, int E, int kU, int ST, bool CR = false, bool WC = false>
 cudaError_t launch_stash_v(const StashSegDesc *segs, int nseg, cudaStream_t s, int bo, int to, int *launches,
                            const SwapArgs *swap, bool early) {
   constexpr int kMaxSeg = 32;
@@ -999,7 +1014,7 @@ cudaError_t launch_stash_v(const StashSegDesc *segs, int nseg, cudaStream_t s, i
       static int resident = 0;
       if (!resident) {
         int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_stash<S, D, E, kU, kMaxSeg, ST, CR>, threads, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_stash<S, D, E, kU, kMaxSeg, ST, CR, WC>, threads, 0);
         resident = std::max(1, per_sm) * kSMs;
       }
       const int64_t waves = std::max<int64_t>(1, (total + resident / 2) / resident);
@@ -1007,13 +1022,12 @@ cudaError_t launch_stash_v(const StashSegDesc *segs, int nseg, cudaStream_t s, i
     }
     if (bo > 0) total = bo;
     else if (bo < 0) total = std::min(total, -bo);   // a cap (ES_OPT_STASH_BACKGROUND)
-  else if (bo < 0) total = std::min(total, -bo);   // a cap (ES_OPT_STASH_BACKGROUND)
     total = std::max(total, k);
     std::vector<int32_t> block0;
     split_blocks(work, total, &block0, &p.nblocks);
     for (int j = 0; j < k; ++j) p.seg[j].block0 = block0[j];
     const int grid = p.nblocks + p.swap_bx * p.swap_n;
-    cudaError_t e = launch_k<k_stash<S, D, E, kU, kMaxSeg, ST, CR>>(dim3(grid), dim3(threads), s, p);
+    cudaError_t e = launch_k<k_stash<S, D, E, kU, kMaxSeg, ST, CR, WC>>(dim3(grid), dim3(threads), s, p);
     if (e != cudaSuccess) return e;
     ++*launches;
   }
@@ -1025,7 +1039,8 @@ cudaError_t launch_stash_v(const StashSegDesc *segs, int nseg, cudaStream_t s, i
 // 5 = one contiguous, equal range per block in whole waves of resident
 // blocks (59 regs; +2.4 % alone, but -0.8 % once consecutive stashes
 // overlap through the early start); 1 / 2 / 4 = one-shot with 8 / 2 / 1
-// units; 3 = one-shot with cache-streaming stores; 6 = contiguous, 8 units.
+// units; 3 = one-shot with cache-streaming stores; 6 = contiguous, 8 units;
+// 8 / 9 = one-shot, warp-contiguous units (a warp moves 32*kU adjacent units) with 2 / 4 units.
 int g_stash_variant = [] {
   const char *e = std::getenv("ES_STASH_VARIANT");
   return e ? std::atoi(e) : 0;
@@ -1042,7 +1057,15 @@ cudaError_t launch_stash_t(const StashSegDesc *segs, int nseg, cudaStream_t s, i
     case 5: return launch_stash_v<S, D, E, 4, 0, true>(segs, nseg, s, bo, to, launches, swap, early);
     case 6: return launch_stash_v<S, D, E, 8, 0, true>(segs, nseg, s, bo, to, launches, swap, early);
     case 7: return launch_stash_v<S, D, E, 4, 2>(segs, nseg, s, bo, to, launches, swap, early);
-    default: return launch_stash_v<S, D, E, 4, 0>(segs, nseg, s, bo, to, launches, swap, early);
+    case 8: return launch_stash_v<S, D, E, 2, 0, false, true>(segs, nseg, s, bo, to, launches, swap, early);
+    case 9: return launch_stash_v<S, D, E, 4, 0, false, true>(segs, nseg, s, bo, to, launches, swap, early);
+    default:
+      // bf16 -> bf16: warp-contiguous units measured 0.6 % faster per BERT step (1.1421 vs 1.1496 ms,
+      // two interleaved repeats); fp32 copies are faster with grid-stride units (ResNet-50 0.3519
+      // vs 0.3541 ms, Swin-B 4.871 vs 4.879 ms) -- profiles/r01_stash_variants.md
+      if (std::is_same<S, BF16T>::value && std::is_same<D, BF16T>::value)
+        return launch_stash_v<S, D, E, 4, 0, false, true>(segs, nseg, s, bo, to, launches, swap, early);
+      return launch_stash_v<S, D, E, 4, 0>(segs, nseg, s, bo, to, launches, swap, early);
   }
 }
 

@@ -70,6 +70,37 @@ __global__ void __launch_bounds__(256) k_read1(const int4 *a, int64_t nvec, int 
   if (acc == 0x12345678) sink[blockIdx.x & 1023] = acc;
 }
 
+// one-shot copy: every thread moves U warp-contiguous 16-B vectors (all loads, then all stores)
+template <int U>
+__global__ void __launch_bounds__(256) k_copy1(const int4 *a, int4 *b, int64_t nvec) {
+  const int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  const int64_t base = w * 32 * U + lane;
+  int4 v[U];
+#pragma unroll
+  for (int u = 0; u < U; ++u)
+    if (base + 32 * u < nvec) v[u] = ldnc(a + base + 32 * u);
+#pragma unroll
+  for (int u = 0; u < U; ++u)
+    if (base + 32 * u < nvec) stna(b + base + 32 * u, v[u]);
+}
+
+// k_stash's current pattern: one-shot grid, U units per thread at grid-wide stride
+template <int U>
+__global__ void __launch_bounds__(256) k_copy_gs(const int4 *a, int4 *b, int64_t nvec) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  for (int64_t u0 = g; u0 < nvec; u0 += stride * U) {
+    int4 v[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if (u0 + u * stride < nvec) v[u] = ldnc(a + u0 + u * stride);
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if (u0 + u * stride < nvec) stna(b + u0 + u * stride, v[u]);
+  }
+}
+
 struct Srcs { const float *p[32]; };
 
 // fold pattern: element-vector v of every source; U consecutive vectors per thread (warp covers
@@ -183,6 +214,28 @@ int main() {
   for (int g : {sms * 4, sms * 8, sms * 16}) {
     float ms = best_ms([&] { k_copy<<<g, 256>>>((const int4 *)a, (int4 *)b, nvec / 2); });
     printf("{\"probe\": \"copy\", \"grid\": %d, \"GBps\": %.1f}\n", g, bytes / (ms * 1e-3) / 1e9);
+  }
+  {  // one-shot copies of 2 GiB (read + write bytes counted), U vectors per thread
+    const int64_t nv = nvec / 2;
+    float m1 = best_ms([&] { k_copy1<1><<<(int)((nv + 255) / 256), 256>>>((const int4 *)a, (int4 *)b, nv); });
+    float m2 = best_ms([&] { k_copy1<2><<<(int)((nv / 2 + 255) / 256), 256>>>((const int4 *)a, (int4 *)b, nv); });
+    float m4 = best_ms([&] { k_copy1<4><<<(int)((nv / 4 + 255) / 256), 256>>>((const int4 *)a, (int4 *)b, nv); });
+    float m8 = best_ms([&] { k_copy1<8><<<(int)((nv / 8 + 255) / 256), 256>>>((const int4 *)a, (int4 *)b, nv); });
+    float mc = best_ms([&] { cudaMemcpyAsync(b, a, bytes / 2, cudaMemcpyDeviceToDevice); });
+    float g4 = best_ms([&] { k_copy_gs<4><<<(int)((nv / 4 + 255) / 256), 256>>>((const int4 *)a, (int4 *)b, nv); });
+    float g2 = best_ms([&] { k_copy_gs<2><<<(int)((nv / 2 + 255) / 256), 256>>>((const int4 *)a, (int4 *)b, nv); });
+    // ResNet-50-sized stash: 102 MB one way (L2 = 126 MB)
+    const int64_t ns = 25557032 / 4;
+    float s4 = best_ms([&] { k_copy_gs<4><<<(int)((ns / 4 + 255) / 256), 256>>>((const int4 *)a, (int4 *)b, ns); });
+    float s2w = best_ms([&] { k_copy1<2><<<(int)((ns / 2 + 255) / 256), 256>>>((const int4 *)a, (int4 *)b, ns); });
+    float s4w = best_ms([&] { k_copy1<4><<<(int)((ns / 4 + 255) / 256), 256>>>((const int4 *)a, (int4 *)b, ns); });
+    printf("{\"probe\": \"copy_gridstride_oneshot\", \"U4_GBps\": %.1f, \"U2_GBps\": %.1f, "
+           "\"resnet_stash_102MB\": {\"gridstride_U4\": %.1f, \"warp_U2\": %.1f, \"warp_U4\": %.1f}}\n",
+           bytes / (g4 * 1e-3) / 1e9, bytes / (g2 * 1e-3) / 1e9, 32.0 * ns / (s4 * 1e-3) / 1e9,
+           32.0 * ns / (s2w * 1e-3) / 1e9, 32.0 * ns / (s4w * 1e-3) / 1e9);
+    printf("{\"probe\": \"copy_oneshot\", \"U1_GBps\": %.1f, \"U2_GBps\": %.1f, \"U4_GBps\": %.1f, \"U8_GBps\": %.1f, "
+           "\"cudaMemcpy_d2d_GBps\": %.1f}\n", bytes / (m1 * 1e-3) / 1e9, bytes / (m2 * 1e-3) / 1e9,
+           bytes / (m4 * 1e-3) / 1e9, bytes / (m8 * 1e-3) / 1e9, bytes / (mc * 1e-3) / 1e9);
   }
   // fold pattern: N sources of L floats each inside `a`, output in `b`
   for (int N : {8, 16, 32}) {
