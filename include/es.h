@@ -177,6 +177,17 @@ typedef struct {
  * incremental folds use at most two 256-thread CTAs per SM.  About half the
  * copy bandwidth when nothing else runs.  Same bits. */
 #define ES_OPT_STASH_BACKGROUND 4u
+/* ES_OPT_PEER_PUSH (G > 1, ES_SCHED_PEER buckets, and ES_SCHED_PEER_CHAIN
+ * buckets under ES_OPT_PEER_ROUNDS): the all-gather is fused
+ * into the fold.  Each owner's fold writes its finished shard / chunk into
+ * its own RESULT area AND into every peer's RESULT area over NVLink (posted
+ * stores, riding the fold's egress while its ingress pulls the remote
+ * contributions); after the barrier every rank copies the whole bucket from
+ * its OWN RESULT area into `out` (local HBM) instead of pulling each shard
+ * from its owner.  Same ops, same bits; per GPU the gather's NVLink ingress
+ * moves into the fold phase as egress (PAPER-independent transport choice,
+ * DESIGN.md 7). */
+#define ES_OPT_PEER_PUSH 8u
 
 /* NEXT-3 compatibility variants -- same canonical order, different step
  * arithmetic:

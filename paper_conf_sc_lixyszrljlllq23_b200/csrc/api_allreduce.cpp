@@ -78,6 +78,13 @@ es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *c
     if (!pipe || b.sched != ES_SCHED_PEER_CHAIN) return k;
     return op == ES_OP_GATHER ? 2 : 1;
   };
+  // ES_OPT_PEER_PUSH: buckets whose final results come out of k_fold (not k_fold_pipe) push them
+  // into every peer's RESULT area; their gathers then read the own RESULT area.
+  auto pushes = [&](const es::BucketPlan &b) -> bool {
+    return (p.options & ES_OPT_PEER_PUSH) && p.G > 1 &&
+           (b.sched == ES_SCHED_PEER || (b.sched == ES_SCHED_PEER_CHAIN && !pipe));
+  };
+  std::vector<std::vector<void *>> push_ptrs;   // per fold segment; outlives the launches below
   for (int32_t ph = 0; ph < phases; ++ph) {
     for (int dd = 0; dd < 2; ++dd) {
       std::vector<es::FoldSegDesc> folds;
@@ -100,7 +107,8 @@ es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *c
           if (phase_of(b, k, f[0]) != ph) continue;
           const int64_t lo = f[1], hi = f[2];
           if (f[0] == ES_OP_GATHER) {
-            gathers.push_back({h->peer_ws[f[3]] + p.result_off + p.slot_off[bk] + (uint64_t)lo * esz,
+            const int32_t from = pushes(b) ? p.rank : (int32_t)f[3];   // pushed: already in our RESULT
+            gathers.push_back({h->peer_ws[from] + p.result_off + p.slot_off[bk] + (uint64_t)lo * esz,
                                reinterpret_cast<unsigned char *>(outs[i]) + (uint64_t)lo * esz, hi - lo});
             gbytes += 2 * (uint64_t)(hi - lo) * esz;
             continue;
@@ -132,8 +140,17 @@ es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *c
           d.out_partial = f[7] == ES_BUF_PART;
           d.out = d.out_partial ? (void *)(h->ws + p.peer_parts_off + b.peer_part_base + (uint64_t)f[8])
                                 : (void *)(h->ws + p.result_off + p.slot_off[bk] + (uint64_t)lo * esz);
+          if (!d.out_partial && pushes(b)) {
+            std::vector<void *> dst;
+            for (int32_t g = 0; g < p.G; ++g)
+              if (g != p.rank) dst.push_back(h->peer_ws[g] + p.result_off + p.slot_off[bk] + (uint64_t)lo * esz);
+            push_ptrs.push_back(std::move(dst));
+            d.push = push_ptrs.back().data();
+            d.npush = (int32_t)push_ptrs.back().size();
+          }
           const uint64_t nbytes =
-              (uint64_t)d.n * ((uint64_t)src.size() * esz + (d.part_in ? 4 : 0) + (d.out_partial ? 4 : esz));
+              (uint64_t)d.n * ((uint64_t)src.size() * esz + (d.part_in ? 4 : 0) + (d.out_partial ? 4 : esz) +
+                               (uint64_t)d.npush * esz);
           d.src = src.data();                     // the buffer survives the move below
           srcs.push_back(std::move(src));
           if (pipe && b.sched == ES_SCHED_PEER_CHAIN) {

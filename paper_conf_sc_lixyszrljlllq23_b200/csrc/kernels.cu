@@ -283,6 +283,7 @@ struct FoldSeg {
   int32_t rot, m, src0;   // sources: src[src0 ...]
   int32_t out_partial;
   int32_t block0;         // first block of this segment
+  int32_t npush;          // ES_OPT_PEER_PUSH: extra copies of the final result, pointers in src[] after the sources
 };
 
 template <int MAXSEG, int MAXSRC>
@@ -415,6 +416,7 @@ __global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams
   const FoldSeg &g = p.seg[si];
   const int nb = (si + 1 < p.nseg ? p.seg[si + 1].block0 : p.nblocks) - g.block0;
   const void *const *src = p.src + g.src0;
+  const int cnt_src = g.rot ? p.N : g.m;                             // push pointers follow the sources
   const int64_t nvec = g.n / V;
   const int64_t tid0 = (int64_t)(blockIdx.x - g.block0) * blockDim.x + threadIdx.x;
   const int64_t stride = (int64_t)nb * blockDim.x;
@@ -433,15 +435,25 @@ __global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams
 #pragma unroll
         for (int e = 0; e < V; ++e) acc[e] = __fmul_rn(acc[e], p.r);   // R5: one rounding
       }
-      st_stream(reinterpret_cast<char *>(g.out) + t * T::kSize, T::narrow(acc));  // R13
+      const int4 w = T::narrow(acc);                                   // R13
+      st_stream(reinterpret_cast<char *>(g.out) + t * T::kSize, w);
+      // ES_OPT_PEER_PUSH: the same words into every peer's RESULT area over NVLink (posted
+      // stores), so the all-gather's traffic rides the fold's otherwise idle egress
+      for (int j = 0; j < g.npush; ++j)
+        st_stream(reinterpret_cast<char *>(const_cast<void *>(src[cnt_src + j])) + t * T::kSize, w);
     }
   }
   const int64_t tail0 = nvec * V;                                    // ragged tail (< V elements)
   if (tid0 < g.n - tail0) {
     const int64_t t = tail0 + tid0;
     const float s = fold_scalar<T, COMPAT>(g, src, p.N, t, p.compat, p.r);
-    if (g.out_partial) reinterpret_cast<float *>(g.out)[t] = s;
-    else T::store1(g.out, t, post ? __fmul_rn(s, p.r) : s);
+    if (g.out_partial) {
+      reinterpret_cast<float *>(g.out)[t] = s;
+    } else {
+      const float o = post ? __fmul_rn(s, p.r) : s;
+      T::store1(g.out, t, o);
+      for (int j = 0; j < g.npush; ++j) T::store1(const_cast<void *>(src[cnt_src + j]), t, o);
+    }
   }
 }
 
@@ -680,9 +692,11 @@ cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSeg
     g.m = d[i].m;
     g.src0 = nsrc;
     g.out_partial = d[i].out_partial ? 1 : 0;
+    g.npush = d[i].npush;
     for (int j = 0; j < k; ++j) p.src[nsrc + j] = d[i].src[j];
-    nsrc += k;
-    work[i] = (d[i].n + T::kVec - 1) / T::kVec * (int64_t)(k + 1);   // vectors x streams
+    for (int j = 0; j < d[i].npush; ++j) p.src[nsrc + k + j] = d[i].push[j];
+    nsrc += k + d[i].npush;
+    work[i] = (d[i].n + T::kVec - 1) / T::kVec * (int64_t)(k + 1 + d[i].npush);   // vectors x streams
   }
   const int threads = to > 0 ? to : 256;
   int64_t vecs = 0;
@@ -695,7 +709,7 @@ cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSeg
   split_blocks(work, total, &block0, &p.nblocks);
   for (int i = 0; i < nseg; ++i) p.seg[i].block0 = block0[i];
   bool tma_ok = g_fold_tma > 0 && !compat && N <= 16 && bo == 0 && to == 0;
-  for (int i = 0; i < nseg && tma_ok; ++i) tma_ok = d[i].rot && !d[i].part_in && !d[i].out_partial;
+  for (int i = 0; i < nseg && tma_ok; ++i) tma_ok = d[i].rot && !d[i].part_in && !d[i].out_partial && !d[i].npush;
   if (tma_ok) {
     constexpr int kS = 3;
     const int stage = N * 256 * T::kVec * T::kSize;
@@ -737,7 +751,7 @@ cudaError_t launch_fold_t(int32_t N, float r, uint32_t compat, const FoldSegDesc
   while (i < nseg) {
     int j = i, nsrc = 0;                     // greedy group within the large capacity
     while (j < nseg) {
-      const int k = segs[j].rot ? N : segs[j].m;
+      const int k = (segs[j].rot ? N : segs[j].m) + segs[j].npush;
       if (j - i + 1 > kBigSeg || nsrc + k > kBigSrc) break;
       nsrc += k;
       ++j;
@@ -783,6 +797,7 @@ cudaError_t launch_pipe_group(int32_t N, float r, const PipeSegDesc *d, int nseg
     g.f.src0 = nsrc;
     g.f.out_partial = f.out_partial ? 1 : 0;
     g.f.block0 = 0;
+    g.f.npush = 0;          // k_fold_pipe never pushes (ES_OPT_PEER_PUSH applies to k_fold launches)
     for (int j = 0; j < f.m; ++j) p.src[nsrc + j] = f.src[j];
     nsrc += f.m;
     g.wait = d[i].wait;

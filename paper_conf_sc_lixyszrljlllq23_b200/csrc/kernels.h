@@ -30,6 +30,8 @@ struct FoldSegDesc {
   const float *part_in = nullptr;
   void *out = nullptr;
   bool out_partial = false;
+  void *const *push = nullptr;        // ES_OPT_PEER_PUSH: npush more destinations of the final result
+  int32_t npush = 0;
 };
 
 // Folds all segments (same dtype, same N) with as few launches as the

@@ -364,7 +364,8 @@ bool validate(const es_config *cfg, std::string *err, bool need_comm) {
     return fail(err, "unknown compat bits");
   if ((cfg->compat & ES_COMPAT_PREDIV) && (cfg->compat & ES_COMPAT_PREMUL))
     return fail(err, "compat PREDIV and PREMUL are exclusive");
-  if (cfg->options & ~(uint32_t)(ES_OPT_INCREMENTAL | ES_OPT_PEER_ROUNDS | ES_OPT_STASH_BACKGROUND)) return fail(err, "unknown option bits");
+  if (cfg->options & ~(uint32_t)(ES_OPT_INCREMENTAL | ES_OPT_PEER_ROUNDS | ES_OPT_STASH_BACKGROUND | ES_OPT_PEER_PUSH))
+    return fail(err, "unknown option bits");
   if ((cfg->options & ES_OPT_INCREMENTAL) && cfg->G != 1) return fail(err, "ES_OPT_INCREMENTAL needs G == 1");
   const bool peer_sched = cfg->sched == ES_SCHED_PEER || cfg->sched == ES_SCHED_PEER_CHAIN ||
                           cfg->sched == ES_SCHED_PEER_AUTO;

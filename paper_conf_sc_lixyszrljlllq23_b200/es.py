@@ -28,6 +28,7 @@ ES_COMPAT_PREDIV, ES_COMPAT_PREMUL, ES_COMPAT_BF16_HOP = 1, 2, 4
 ES_OPT_INCREMENTAL = 1
 ES_OPT_PEER_ROUNDS = 2
 ES_OPT_STASH_BACKGROUND = 4
+ES_OPT_PEER_PUSH = 8
 
 EXPORTED = [
     "es_workspace_bytes", "es_init", "es_destroy", "es_sync", "es_register_state", "es_init_state",

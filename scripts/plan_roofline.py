@@ -25,8 +25,11 @@ SCHEDS = {"direct": es.ES_SCHED_DIRECT, "chain": es.ES_SCHED_CHAIN, "peer": es.E
           "peer_chain": es.ES_SCHED_PEER_CHAIN}
 
 
-def rank_costs(name, G, kind, sched):
-    """-> list over ranks of list over phases of (hbm_bytes, nvlink_in_bytes)."""
+def rank_costs(name, G, kind, sched, push=False):
+    """-> list over ranks of list over phases of (hbm_bytes, nvlink_in_bytes).
+    push (ES_OPT_PEER_PUSH, PEER only): every owner's fold also writes its shard into each peer's
+    RESULT area, so a rank's fold phase receives the other shards over NVLink and its gather
+    phase is a local RESULT -> out copy."""
     c = workloads.config(name)
     N = c["N"]
     m = workloads.mapping(N, G, kind)
@@ -59,10 +62,16 @@ def rank_costs(name, G, kind, sched):
                     elif int(f[5]) == es.ES_BUF_PEER_PART:
                         nv += n * 4
                     hb += n * (4 if int(f[7]) == es.ES_BUF_PART else esz)   # write
+                    if push and sched == es.ES_SCHED_PEER and int(f[7]) != es.ES_BUF_PART:
+                        # the other owners' pushes land here in the same phase: L - own shard
+                        nv += (L - n) * esz
+                        hb += (L - n) * esz
                 elif op == es.ES_OP_RECV:
                     w = 4 if int(f[4]) == es.ES_BUF_PART else esz
                     nv += n * w
                     hb += n * w
+                elif op == es.ES_OP_GATHER and push and sched == es.ES_SCHED_PEER:
+                    hb += 2 * n * esz                                       # own RESULT -> out
                 elif op == es.ES_OP_GATHER:
                     if int(f[3]) != g:
                         nv += n * esz
@@ -98,14 +107,18 @@ def main(path):
             "Per phase (between groups / barriers), the slowest rank's max(HBM, NVLink) time, summed.\n",
             "peer_chain = rounds separated by barriers (ES_OPT_PEER_ROUNDS); pipelined = the default k_fold_pipe step "
             "(all rounds overlapped through per-tile flags, then the gather).\n",
-            "| config | G | mapping | direct ms | chain ms | peer ms | peer_chain ms | peer_chain pipelined ms | AUTO picks | "
-            "max NVLink in / rank MB (direct, chain) |",
-            "|---|---|---|---|---|---|---|---|---|---|"]
+            "peer push = ES_OPT_PEER_PUSH (the gather fused into the fold as NVLink stores): the same ingress bytes "
+            "per rank move into the fold phase, so the bandwidth bound does not drop; what it removes is the "
+            "gather's remote loads and one phase boundary (not modelled here).\n",
+            "| config | G | mapping | direct ms | chain ms | peer ms | peer push ms | peer_chain ms | "
+            "peer_chain pipelined ms | AUTO picks | max NVLink in / rank MB (direct, chain) |",
+            "|---|---|---|---|---|---|---|---|---|---|---|"]
     cases = [("resnet50", G, "contiguous") for G in (2, 4, 8)] + [("vgg19", G, "contiguous") for G in (2, 4, 8)] + \
         [("bert_base", 8, "contiguous"), ("bert_base", 8, "round_robin")] + \
         [("swin_b", G, "contiguous") for G in (2, 4, 8)]
     for name, G, kind in cases:
         res = {k: rank_costs(name, G, kind, v) for k, v in SCHEDS.items()}
+        res["peer_push"] = rank_costs(name, G, kind, es.ES_SCHED_PEER, push=True)
         c = workloads.config(name)
         cfg = es.Config(c["N"], G, 0, workloads.mapping(c["N"], G, kind),
                         [(n, es.ES_F32 if d == "f32" else es.ES_BF16) for n, d in c["buckets"]])
@@ -114,7 +127,7 @@ def main(path):
         nvd = max(sum(ph[1] for ph in r.values()) for r in res["direct"]) / 1e6
         nvc = max(sum(ph[1] for ph in r.values()) for r in res["chain"]) / 1e6
         rows.append(f"| {name} | {G} | {kind} | {bound_ms(res['direct']):.3f} | {bound_ms(res['chain']):.3f} | "
-                    f"{bound_ms(res['peer']):.3f} | {bound_ms(res['peer_chain']):.3f} | "
+                    f"{bound_ms(res['peer']):.3f} | {bound_ms(res['peer_push']):.3f} | {bound_ms(res['peer_chain']):.3f} | "
                     f"{bound_ms_pipelined(res['peer_chain']):.3f} | {pick} | {nvd:.0f}, {nvc:.0f} |")
     text = "\n".join(rows) + "\n"
     with open(path, "w") as f:

@@ -257,6 +257,27 @@ def test_mappings_n8_loopback(G, kind, sched):
             assert_bits_equal(res[g][b], want[b], f"G={G} {kind} sched={sched} rank={g} b={b}")
 
 
+@pytest.mark.parametrize("G,kind", [(2, "contiguous"), (4, "random"), (8, "contiguous"), (8, "round_robin"),
+                                    (3, "random")])
+@pytest.mark.parametrize("sched,options", [(es.ES_SCHED_PEER, 0), (es.ES_SCHED_PEER_AUTO, 0),
+                                           (es.ES_SCHED_PEER_CHAIN, es.ES_OPT_PEER_ROUNDS),
+                                           (es.ES_SCHED_PEER_CHAIN, 0)])
+@pytest.mark.parametrize("batched", [False, True])
+def test_peer_push_loopback(G, kind, sched, options, batched):
+    """ES_OPT_PEER_PUSH: owners push their finished shards / chunks into every peer's RESULT area
+    inside the fold; gathers read the own RESULT.  Repeated steps (RESULT reuse across steps and
+    buckets) keep the oracle's bits on every rank.  PEER_CHAIN without PEER_ROUNDS (k_fold_pipe)
+    ignores the option and must be unaffected."""
+    rng = np.random.default_rng(700 + G * 10 + len(kind))
+    xs = [_gauss(rng, 8, 200003), _gauss(rng, 8, 4096 + 5, "bf16"), _gauss(rng, 8, 17)]
+    want = [oracle.reduce(xs[0], "f32"), oracle.reduce(xs[1], "bf16"), oracle.reduce(xs[2], "f32")]
+    res = reduce_loopback(xs, G, workloads.mapping(8, G, kind), sched, steps=3, batched=batched,
+                          options=options | es.ES_OPT_PEER_PUSH)
+    for g in range(G):
+        for b in range(3):
+            assert_bits_equal(res[g][b], want[b], f"push G={G} {kind} sched={sched} opt={options} rank={g} b={b}")
+
+
 @pytest.mark.parametrize("kind", ["contiguous", "round_robin"])
 def test_bert_uneven_n12_g8_loopback(kind):
     """BERT config shape: N=12 on G=8, n = [2,2,2,2,1,1,1,1] (contiguous) and
@@ -650,6 +671,8 @@ def test_random_schedules_mappings_layouts(seed):
     A = int(rng.choice([8, 16, 64, 1024]))
     sched = int(rng.choice(list(SCHED_NAMES)))
     options = int(rng.choice([0, es.ES_OPT_PEER_ROUNDS]))
+    if seed % 3 == 2:                                             # a third of the seeds push the gather
+        options |= es.ES_OPT_PEER_PUSH
     steps = int(rng.integers(1, 4))
     xs = [_gauss(rng, N, L, d) for L, d in zip(sizes, dts)]
     want = [oracle.reduce(x, d, A=A) for x, d in zip(xs, dts)]

@@ -25,7 +25,7 @@ def _port():
     return p
 
 
-def _worker(rank, port, q, sched):
+def _worker(rank, port, q, sched, options=0):
     import sys
     sys.path.insert(0, ROOT)
     sys.path.insert(0, os.path.join(ROOT, "tests"))
@@ -41,7 +41,8 @@ def _worker(rank, port, q, sched):
         torch.cuda.set_device(0)
         N, mapping = 6, [0, 1, 1, 0, 1, 1]        # uneven: 2 and 4 local ESTs
         Ls, dts = [100003, 4096, 17], ["f32", "bf16", "f32"]
-        agg = Aggregator(N, 2, rank, mapping, list(zip(Ls, dts)), transport=es.ES_TRANSPORT_NONE, sched=sched)
+        agg = Aggregator(N, 2, rank, mapping, list(zip(Ls, dts)), transport=es.ES_TRANSPORT_NONE, sched=sched,
+                         options=options)
         agg.peer_connect()
         ok = True
         for step in range(3):
@@ -68,15 +69,17 @@ def _worker(rank, port, q, sched):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("sched_name", ["ES_SCHED_PEER", "ES_SCHED_PEER_CHAIN"])
-def test_peer_schedule_two_processes_real_ipc(sched_name):
+@pytest.mark.parametrize("sched_name,opt_name", [("ES_SCHED_PEER", None), ("ES_SCHED_PEER_CHAIN", None),
+                                                ("ES_SCHED_PEER", "ES_OPT_PEER_PUSH")])
+def test_peer_schedule_two_processes_real_ipc(sched_name, opt_name):
     import sys
     sys.path.insert(0, ROOT)
     from paper_conf_sc_lixyszrljlllq23_b200 import es
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _port()
-    ps = [ctx.Process(target=_worker, args=(r, port, q, getattr(es, sched_name))) for r in range(2)]
+    options = getattr(es, opt_name) if opt_name else 0
+    ps = [ctx.Process(target=_worker, args=(r, port, q, getattr(es, sched_name), options)) for r in range(2)]
     for p in ps:
         p.start()
     for p in ps:
