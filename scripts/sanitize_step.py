@@ -108,10 +108,11 @@ def multi(rng, sched, options=0):
 
 SCHEDS = {"direct": (es.ES_SCHED_DIRECT, 0), "chain": (es.ES_SCHED_CHAIN, 0), "peer": (es.ES_SCHED_PEER, 0),
           "peer_chain": (es.ES_SCHED_PEER_CHAIN, 0),
-          "peer_chain_rounds": (es.ES_SCHED_PEER_CHAIN, es.ES_OPT_PEER_ROUNDS)}
+          "peer_chain_rounds": (es.ES_SCHED_PEER_CHAIN, es.ES_OPT_PEER_ROUNDS),
+          "peer_push": (es.ES_SCHED_PEER, es.ES_OPT_PEER_PUSH)}
 
 if __name__ == "__main__":
-    # argv: which parts to run (default: all): g1 g1_bg direct chain peer peer_chain peer_chain_rounds
+    # argv: which parts to run (default: all): g1 g1_bg direct chain peer peer_chain peer_chain_rounds peer_push
     parts = sys.argv[1:] or ["g1", "g1_bg"] + list(SCHEDS)
     rng = np.random.default_rng(0)
     for part in parts:
