@@ -54,6 +54,8 @@ def parse():
                         "stashed with ES_STASH_INPLACE")
     p.add_argument("--stash-background", action="store_true",
                    help="ES_OPT_STASH_BACKGROUND: one-wave stash grids (for overlap with compute; scripts/overlap_probe.py)")
+    p.add_argument("--peer-push", action="store_true",
+                   help="ES_OPT_PEER_PUSH (G>1, peer schedules): the all-gather fused into the fold as NVLink stores")
     p.add_argument("--rehearse-same-gpu", action="store_true",
                    help="functional rehearsal of the N>1 path on ONE GPU: every rank on cuda:0, gloo process "
                         "group, a peer schedule (CUDA IPC, no NCCL); times are not GPU-scaling numbers")
@@ -300,7 +302,8 @@ def main():
                      transport=es.ES_TRANSPORT_NONE if G == 1 or rehearse else es.ES_TRANSPORT_NCCL, comm=comm,
                      sched=sched,
                      device=dev, options=(es.ES_OPT_INCREMENTAL if args.incremental else 0) |
-                     (es.ES_OPT_STASH_BACKGROUND if args.stash_background else 0))
+                     (es.ES_OPT_STASH_BACKGROUND if args.stash_background else 0) |
+                     (es.ES_OPT_PEER_PUSH if args.peer_push else 0))
     if G > 1 and sched in es.PEER_SCHEDS:
         agg.peer_connect()                       # CUDA IPC map of every peer's workspace (NVLink)
     live = [torch.zeros(n, dtype=torch.uint8, device=dev) for n in snb]
@@ -518,7 +521,8 @@ def main():
                    "api": "per-bucket" if args.per_bucket else ("incremental" if args.incremental else
                                                                ("zero-copy-inplace" if args.inplace else
                                                                 ("batched" if args.no_fuse else "batched+fused-switch")))
-                   + (" +stash-background" if args.stash_background else ""),
+                   + (" +stash-background" if args.stash_background else "")
+                   + (" +peer-push" if args.peer_push else ""),
                    "l2": ("inputs larger than L2 (%.1f MB of EST gradients per GPU per step)" % (in_bytes / 1e6))
                    if flush is None else "L2 flushed between timed steps (512 MB write, then read back: "
                                                   "no flush lines left dirty to drain inside the timed step)"},

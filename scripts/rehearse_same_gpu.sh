@@ -5,4 +5,6 @@ R 4 --config resnet50 --sched peer_chain > gpurun_out/reh_resnet50_g4.json 2>> g
 R 8 --config resnet50 --sched peer --mapping random > gpurun_out/reh_resnet50_g8.json 2>> gpurun_out/reh.err
 R 8 --config bert_base --sched peer_auto --mapping round_robin > gpurun_out/reh_bert_g8rr.json 2>> gpurun_out/reh.err
 R 8 --config bert_base --sched peer_chain > gpurun_out/reh_bert_g8c.json 2>> gpurun_out/reh.err
+R 8 --config resnet50 --sched peer --peer-push > gpurun_out/reh_resnet50_g8_push.json 2>> gpurun_out/reh.err
+R 8 --config bert_base --sched peer --peer-push --mapping round_robin > gpurun_out/reh_bert_g8rr_push.json 2>> gpurun_out/reh.err
 tail -5 gpurun_out/reh.err
