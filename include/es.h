@@ -184,9 +184,10 @@ typedef struct {
  * stores, riding the fold's egress while its ingress pulls the remote
  * contributions); after the barrier every rank copies the whole bucket from
  * its OWN RESULT area into `out` (local HBM) instead of pulling each shard
- * from its owner.  Same ops, same bits; per GPU the gather's NVLink ingress
- * moves into the fold phase as egress (PAPER-independent transport choice,
- * DESIGN.md 7). */
+ * from its owner.  Same ops, same bits, same NVLink bytes per GPU: the other
+ * shards arrive during the fold phase as their owners' posted stores instead
+ * of during the gather as this rank's remote loads.  Ignored
+ * (pull gather) when N + G - 1 > 1024. */
 #define ES_OPT_PEER_PUSH 8u
 
 /* NEXT-3 compatibility variants -- same canonical order, different step

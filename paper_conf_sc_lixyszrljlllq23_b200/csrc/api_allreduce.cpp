@@ -81,7 +81,9 @@ es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *c
   // ES_OPT_PEER_PUSH: buckets whose final results come out of k_fold (not k_fold_pipe) push them
   // into every peer's RESULT area; their gathers then read the own RESULT area.
   auto pushes = [&](const es::BucketPlan &b) -> bool {
-    return (p.options & ES_OPT_PEER_PUSH) && p.G > 1 &&
+    // (sources + push pointers of one segment must fit one launch's 1024-pointer table; the rule
+    //  depends only on N and G, so every rank decides alike)
+    return (p.options & ES_OPT_PEER_PUSH) && p.G > 1 && p.N + p.G - 1 <= 1024 &&
            (b.sched == ES_SCHED_PEER || (b.sched == ES_SCHED_PEER_CHAIN && !pipe));
   };
   std::vector<std::vector<void *>> push_ptrs;   // per fold segment; outlives the launches below
