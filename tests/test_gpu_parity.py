@@ -576,6 +576,19 @@ def test_max_n_1024():
         assert_bits_equal(reduce_g1(xs, batched=batched)[0], oracle.reduce(xs[0], "f32"), f"batched={batched}")
 
 
+@pytest.mark.parametrize("N", [1023, 1024])
+def test_peer_push_at_the_pointer_table_limit(N):
+    """ES_OPT_PEER_PUSH at G = 2: N = 1023 pushes (1023 sources + 1 push pointer fill the 1024-entry
+    table), N = 1024 falls back to the pull gather on every rank (N + G - 1 > 1024)."""
+    rng = np.random.default_rng(N)
+    xs = [_gauss(rng, N, 4099)]
+    m = workloads.mapping(N, 2, "round_robin")
+    res = reduce_loopback(xs, 2, m, es.ES_SCHED_PEER, options=es.ES_OPT_PEER_PUSH)
+    want = oracle.reduce(xs[0], "f32")
+    for g in range(2):
+        assert_bits_equal(res[g][0], want, f"N={N} rank={g}")
+
+
 def test_max_bucket_numel_2p31_minus_1():
     """The largest legal bucket (2^31 - 1 elements, bf16, 4 GiB per EST): the
     32-bit chunk arithmetic and 64-bit offsets hold to the last element."""
