@@ -81,6 +81,7 @@ es_status es_init(const es_config *cfg, void *workspace, size_t workspace_bytes,
   const size_t nslot = (size_t)h->B * h->n_local;
   h->stashed.assign(nslot, 0);
   h->borrowed.assign(nslot, nullptr);
+  h->inc_full.assign(nslot, 0);
   h->stash_ev.assign(nslot, nullptr);
   h->stash_cap.assign(nslot, 0);
   h->ar_ev.assign(h->B, nullptr);
@@ -243,9 +244,13 @@ es_status es_profile_enable(es_handle h, int32_t on) {
 static void drain(es_handle h) {
   for (auto &r : h->recs) {
     float t = 0.f;
-    cudaEventSynchronize(r.b);
-    cudaEventElapsedTime(&t, r.a, r.b);
-    h->ms[r.kind] += t;
+    // A captured pair that was never replayed (or an eager pair that failed)
+    // has no time: skip it and clear the error it raised, so it cannot
+    // surface later as some other call's launch failure.
+    if (cudaEventSynchronize(r.b) == cudaSuccess && cudaEventElapsedTime(&t, r.a, r.b) == cudaSuccess)
+      h->ms[r.kind] += t;
+    else
+      cudaGetLastError();
     std::vector<cudaEvent_t> &dst = r.captured ? h->graph_events : h->pool;
     dst.push_back(r.a);
     dst.push_back(r.b);

@@ -2,7 +2,9 @@
 // slots, EST context export / import (elastic resume), per-EST dropout.
 #include <unistd.h>
 
+#include <chrono>
 #include <cstdlib>
+#include <random>
 
 #include "handle.h"
 
@@ -13,8 +15,10 @@ extern "C" {
 namespace {
 
 struct PeerBlob {
-  char magic[8];            // "ESPEER01"
+  char magic[8];            // "ESPEER02"
   int32_t rank, pid;
+  uint64_t nonce;           // random per process: pid alone is ambiguous across PID namespaces
+  uint64_t plan_hash;       // everything that shapes the peer protocol (must match on every rank)
   uint64_t raw;             // workspace address in the owner's process
   uint64_t offset;          // workspace - allocation base
   uint64_t ws_bytes;
@@ -44,6 +48,46 @@ bool allocation_base(void *p, void **base) {
   return true;
 }
 
+uint64_t fnv1a(uint64_t h, const void *p, size_t n) {
+  const unsigned char *c = reinterpret_cast<const unsigned char *>(p);
+  for (size_t i = 0; i < n; ++i) h = (h ^ c[i]) * 1099511628211ull;
+  return h;
+}
+
+// One random value per process (ranks in different containers may share a pid).
+uint64_t process_nonce() {
+  static const uint64_t n = [] {
+    std::random_device rd;
+    uint64_t x = ((uint64_t)rd() << 32) ^ rd();
+    x ^= (uint64_t)std::chrono::steady_clock::now().time_since_epoch().count();
+    x ^= (uint64_t)getpid() * 0x9E3779B97F4A7C15ull;
+    return x | 1;
+  }();
+  return n;
+}
+
+// Hash of every input that shapes the peer protocol: the layout, N, G, A, the
+// mapping, each bucket's schedule, the compat bits and the options (the
+// executor's phases, barrier count and gather sources depend on them).  Ranks
+// whose plans differ here would wait on barriers the others never reach or
+// gather data never pushed.
+uint64_t peer_plan_hash(const es::Plan &p) {
+  uint64_t h = 1469598103934665603ull;
+  h = fnv1a(h, &p.N, sizeof p.N);
+  h = fnv1a(h, &p.G, sizeof p.G);
+  h = fnv1a(h, &p.A, sizeof p.A);
+  h = fnv1a(h, p.est_to_gpu.data(), p.est_to_gpu.size() * sizeof(int32_t));
+  for (const es::BucketPlan &b : p.bp) {
+    h = fnv1a(h, &b.L, sizeof b.L);
+    const int32_t d = (int32_t)b.dtype;
+    h = fnv1a(h, &d, sizeof d);
+    h = fnv1a(h, &b.sched, sizeof b.sched);
+  }
+  h = fnv1a(h, &p.compat, sizeof p.compat);
+  h = fnv1a(h, &p.options, sizeof p.options);
+  return h;
+}
+
 }  // namespace
 
 es_status es_peer_blob(es_handle h, void *blob, size_t bytes) {
@@ -52,9 +96,11 @@ es_status es_peer_blob(es_handle h, void *blob, size_t bytes) {
   if (!blob || bytes < ES_PEER_BLOB_BYTES) return set_err(ES_EINVAL, "blob must hold ES_PEER_BLOB_BYTES");
   PeerBlob b;
   std::memset(&b, 0, sizeof b);
-  std::memcpy(b.magic, "ESPEER01", 8);
+  std::memcpy(b.magic, "ESPEER02", 8);
   b.rank = h->plan.rank;
   b.pid = (int32_t)getpid();
+  b.nonce = process_nonce();
+  b.plan_hash = peer_plan_hash(h->plan);
   b.raw = (uint64_t)(uintptr_t)h->ws;
   b.ws_bytes = h->ws_bytes;
   void *base = nullptr;
@@ -83,6 +129,8 @@ es_status es_peer_open(es_handle h, const void *blobs, size_t bytes) {
   std::vector<unsigned char *> ws(p.G, nullptr);
   std::vector<void *> mapped;
   const int32_t me = (int32_t)getpid();
+  const uint64_t my_nonce = process_nonce();
+  const uint64_t my_hash = peer_plan_hash(p);
   // Ranks sharing this process (loopback) share one device: their barrier
   // kernels spin concurrently on different streams, which needs one hardware
   // queue per rank -- more ranks than CUDA_DEVICE_MAX_CONNECTIONS (default 8)
@@ -91,7 +139,7 @@ es_status es_peer_open(es_handle h, const void *blobs, size_t bytes) {
   for (int32_t g = 0; g < p.G; ++g) {
     PeerBlob b;
     std::memcpy(&b, reinterpret_cast<const unsigned char *>(blobs) + (size_t)g * ES_PEER_BLOB_BYTES, sizeof b);
-    same_process += b.pid == me;
+    same_process += b.pid == me && b.nonce == my_nonce;
   }
   const char *mc = std::getenv("CUDA_DEVICE_MAX_CONNECTIONS");
   const int32_t max_conn = mc ? std::atoi(mc) : 8;
@@ -100,9 +148,14 @@ es_status es_peer_open(es_handle h, const void *blobs, size_t bytes) {
   for (int32_t g = 0; g < p.G; ++g) {
     PeerBlob b;
     std::memcpy(&b, reinterpret_cast<const unsigned char *>(blobs) + (size_t)g * ES_PEER_BLOB_BYTES, sizeof b);
-    if (std::memcmp(b.magic, "ESPEER01", 8) != 0 || b.rank != g) {
+    if (std::memcmp(b.magic, "ESPEER02", 8) != 0 || b.rank != g) {
       for (void *m : mapped) cudaIpcCloseMemHandle(m);
       return set_err(ES_EINVAL, "blob g is not rank g's es_peer_blob");
+    }
+    if (b.plan_hash != my_hash) {
+      for (void *m : mapped) cudaIpcCloseMemHandle(m);
+      return set_err(ES_EINVAL, "rank " + std::to_string(g) +
+                                    "'s plan differs (N, G, A, mapping, layout, schedules, compat or options)");
     }
     int32_t n_g = 0;
     for (int32_t e = 0; e < p.N; ++e) n_g += p.est_to_gpu[e] == g;
@@ -112,7 +165,7 @@ es_status es_peer_open(es_handle h, const void *blobs, size_t bytes) {
     }
     if (g == p.rank) {
       ws[g] = h->ws;
-    } else if (b.pid == me) {
+    } else if (b.pid == me && b.nonce == my_nonce) {
       ws[g] = reinterpret_cast<unsigned char *>((uintptr_t)b.raw);     // same process (loopback)
     } else {
       if (!b.ipc_ok) {
@@ -216,6 +269,15 @@ es_status es_export_context(es_handle h, int32_t est, void *host_dst, size_t byt
   if (li < 0) return set_err(ES_ESTATE, "est is not mapped to this rank");
   const int32_t nst = (int32_t)p.state_nbytes.size();
   if (nst > 0 && !h->state_registered) return set_err(ES_ESTATE, "es_register_state has not been called");
+  // NEXT-1: a COPY stash of a bucket being folded incrementally keeps only
+  // the chunks that wait for the wrap in the slot (the rest went into the
+  // fp32 partials), so the slot is not this EST's gradient: refuse.
+  for (int32_t b = 0; b < h->B; ++b) {
+    const size_t k = (size_t)li * h->B + b;
+    if (h->inc_next[b] > 0 && h->stashed[k] && !h->borrowed[k] && h->inc_full[k] == 0)
+      return set_err(ES_ESTATE, "bucket is being folded incrementally (es_stash_fold_grads): its slot holds "
+                                "only part of the EST's gradient and cannot be exported");
+  }
   cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
   unsigned char *o = reinterpret_cast<unsigned char *>(host_dst);
   CtxHeader hd;
@@ -283,6 +345,13 @@ es_status es_import_context(es_handle h, int32_t est, const void *host_src, size
   const int32_t nst = (int32_t)p.state_nbytes.size();
   if (nst > 0 && li == h->cur_local && !h->state_registered)
     return set_err(ES_ESTATE, "es_register_state has not been called");
+  {
+    const unsigned char *m = reinterpret_cast<const unsigned char *>(host_src) + sizeof hd;
+    for (int32_t b = 0; b < h->B; ++b)
+      if (m[b] && h->inc_next[b] > 0)
+        return set_err(ES_ESTATE, "bucket is being folded incrementally this step: an imported contribution "
+                                  "would bypass the running partials");
+  }
   cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
   const unsigned long long cap = capture_id(cs);
   const unsigned char *in = reinterpret_cast<const unsigned char *>(host_src);

@@ -225,6 +225,8 @@ es_status es_stash_fold_grads(es_handle h, int32_t est, int32_t n, const int32_t
     h->stash_cap[k] = cap;
     h->stashed[k] = 1;
     h->inc_next[buckets[i]] = est + 1;
+    // the slot holds the whole gradient iff nothing of it was folded here (EST 0, the last EST)
+    h->inc_full[k] = mode == ES_STASH_COPY && (est == 0 || est == p.N - 1) ? 1 : 0;
   }
   return ES_OK;
 }

@@ -93,6 +93,9 @@ struct es_ctx {
 
   // NEXT-1 incremental fold: next EST expected per bucket (0: none folded yet)
   std::vector<int32_t> inc_next;
+  // [local EST index * B + bucket]: 1 if an incremental COPY stash left the EST's
+  // whole gradient in the slot (exportable), 0 if part of it lives only in the partials
+  std::vector<uint8_t> inc_full;
 
   // ES_SCHED_PEER
   std::vector<unsigned char *> peer_ws;   // [G] workspace base of every rank, mapped here

@@ -114,47 +114,6 @@ __device__ __forceinline__ void st_stream(uint2 *p, const uint2 &v) {
   asm volatile("st.global.L1::no_allocate.v2.u32 [%0], {%1, %2};" ::"l"(p), "r"(v.x), "r"(v.y) : "memory");
 }
 __device__ __forceinline__ void st_stream(int4 *p, const int4 &v) { st_stream(static_cast<void *>(p), v); }
-// Cache-streaming (evict-first) stores: experiment for the stash (ES_STASH_VARIANT=3).
-__device__ __forceinline__ void st_cs(int4 *p, const int4 &v) {
-  asm volatile("st.global.cs.v4.s32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
-               : "memory");
-}
-__device__ __forceinline__ void st_cs(uint2 *p, const uint2 &v) {
-  asm volatile("st.global.cs.v2.u32 [%0], {%1, %2};" ::"l"(p), "r"(v.x), "r"(v.y) : "memory");
-}
-
-// L2 evict-first loads/stores (experiment for the stash, ES_STASH_VARIANT=7:
-// a stream copied once should not push a concurrent kernel's working set out
-// of L2).
-__device__ __forceinline__ uint64_t l2_evict_first_policy() {
-  uint64_t pol;
-  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-  return pol;
-}
-__device__ __forceinline__ int4 ld_ef(const int4 *p, uint64_t pol) {
-  int4 r;
-  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
-               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
-               : "l"(p), "l"(pol));
-  return r;
-}
-__device__ __forceinline__ uint2 ld_ef(const uint2 *p, uint64_t pol) {
-  uint2 r;
-  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0, %1}, [%2], %3;"
-               : "=r"(r.x), "=r"(r.y)
-               : "l"(p), "l"(pol));
-  return r;
-}
-__device__ __forceinline__ void st_ef(int4 *p, const int4 &v, uint64_t pol) {
-  asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.s32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p), "r"(v.x),
-               "r"(v.y), "r"(v.z), "r"(v.w), "l"(pol)
-               : "memory");
-}
-__device__ __forceinline__ void st_ef(uint2 *p, const uint2 &v, uint64_t pol) {
-  asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.u32 [%0], {%1, %2}, %3;" ::"l"(p), "r"(v.x), "r"(v.y),
-               "l"(pol)
-               : "memory");
-}
 
 __device__ __forceinline__ uint32_t smem_addr(const void *p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -186,8 +145,9 @@ cudaError_t launch(K kernel, dim3 grid, dim3 block, cudaStream_t s, const P &par
   at[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = at;
   cfg.numAttrs = g_pdl ? 1 : 0;
-  cudaError_t e = cudaLaunchKernelEx(&cfg, kernel, params);
-  return e != cudaSuccess ? e : cudaGetLastError();
+  // Only this launch's own status: cudaGetLastError() here would report (and
+  // clear) an unrelated earlier non-sticky error as this kernel's failure.
+  return cudaLaunchKernelEx(&cfg, kernel, params);
 }
 
 template <auto F, typename P>
@@ -487,7 +447,6 @@ struct PipeParams {
   const uint64_t *epoch;  // this rank's barrier epoch counter
   unsigned int *ticket;   // zeroed before the launch
   uint64_t timeout_ns;
-  int32_t debug;          // ES_PIPE_DEBUG=1: on timeout print the stuck wait and skip it (wrong bits) instead of trapping
   PipeSeg seg[MAXSEG];
   const void *src[MAXSRC];
 };
@@ -532,13 +491,7 @@ __global__ void __launch_bounds__(256) k_fold_pipe(const __grid_constant__ PipeP
         if (f >= v) break;
         __nanosleep(64);
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now));
-        if (now - t0 > p.timeout_ns) {                // the producer never published: fail loudly
-          if (!p.debug) __trap();
-          printf("k_fold_pipe stuck: block %d ticket %d seg lo %lld n %lld tile %lld flag %llu want %llu wait %p\n",
-                 (int)blockIdx.x, tk, (long long)g.lo, (long long)g.n, (long long)tile, (unsigned long long)f,
-                 (unsigned long long)v, (const void *)fl);
-          break;
-        }
+        if (now - t0 > p.timeout_ns) __trap();         // the producer never published: fail loudly
       }
     }
     __syncthreads();
@@ -736,8 +689,7 @@ cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSeg
     cfg.attrs = at;
     cfg.numAttrs = g_pdl ? 1 : 0;
     (void)KernelReg<k_fold_tma<T, MAXSEG, MAXSRC, kS>>::token;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, k_fold_tma<T, MAXSEG, MAXSRC, kS>, p);
-    return e != cudaSuccess ? e : cudaGetLastError();
+    return cudaLaunchKernelEx(&cfg, k_fold_tma<T, MAXSEG, MAXSRC, kS>, p);
   }
   if (compat) return launch_k<k_fold<T, MAXSEG, MAXSRC, true>>(dim3(p.nblocks), dim3(threads), s, p);
   return launch_k<k_fold<T, MAXSEG, MAXSRC, false>>(dim3(p.nblocks), dim3(threads), s, p);
@@ -778,11 +730,6 @@ cudaError_t launch_pipe_group(int32_t N, float r, const PipeSegDesc *d, int nseg
   p.epoch = epoch;
   p.ticket = ticket;
   p.timeout_ns = barrier_timeout_ns();
-  static const int dbg = [] {
-    const char *e = std::getenv("ES_PIPE_DEBUG");
-    return e && e[0] == '1' ? 1 : 0;
-  }();
-  p.debug = dbg;
   int nsrc = 0, tiles = 0;
   for (int i = 0; i < nseg; ++i) {
     PipeSeg &g = p.seg[i];
@@ -814,11 +761,6 @@ cudaError_t launch_pipe_group(int32_t N, float r, const PipeSegDesc *d, int nseg
     }
     return std::max(b, 1);
   }();
-  static const int share_env = [] {   // ES_PIPE_SHARE: diagnostic override of the device share
-    const char *e = std::getenv("ES_PIPE_SHARE");
-    return e ? std::atoi(e) : 0;
-  }();
-  if (share_env > 0) share = share_env;
   const int grid = std::max(1, std::min(tiles, kSMs * occ / std::max(share, 1)));
   cudaError_t e = cudaMemsetAsync(ticket, 0, sizeof(unsigned int), s);
   if (e != cudaSuccess) return e;
@@ -922,7 +864,9 @@ int swap_blocks_per_entry(uint64_t max_nbytes) {
   return (int)std::max<uint64_t>(1, std::min<uint64_t>((words + 255) / 256, 64));
 }
 
-template <typename S, typename D, int E, int kU, int MAXSEG, int ST, bool CR = false, bool WC = false>
+// WC (warp-contiguous): a warp's kU units are 32*kU adjacent units (one
+// 512*kU-byte run); otherwise a thread's kU units are a grid stride apart.
+template <typename S, typename D, int E, int kU, int MAXSEG, bool WC>
 __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashParams<MAXSEG> p) {
   using In = typename VecT<S::kSize * E>::T;
   using Out = typename VecT<D::kSize * E>::T;
@@ -942,52 +886,39 @@ __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashPara
   const In *s = reinterpret_cast<const In *>(g.src);
   Out *d = reinterpret_cast<Out *>(g.dst);
   const int64_t nunits = g.n / E;
-  int64_t stride = (int64_t)nb * blockDim.x;
-  int64_t gid = (int64_t)(bid - g.block0) * blockDim.x + threadIdx.x;
-  int64_t ubeg = 0, uend = nunits;
-  if (CR) {   // contiguous, equal range per block (balanced: every block finishes together)
-    const int64_t per = ((nunits + nb - 1) / nb + blockDim.x - 1) / blockDim.x * blockDim.x;
-    ubeg = min(nunits, (int64_t)(bid - g.block0) * per);
-    uend = min(nunits, ubeg + per);
-    stride = blockDim.x;
-    gid = ubeg + threadIdx.x;
-  }
-  const uint64_t pol = ST == 2 ? l2_evict_first_policy() : 0;
-  if (WC) {   // warp-contiguous: a warp's kU units are 32*kU adjacent units (one 512*kU-byte run)
+  const int64_t stride = (int64_t)nb * blockDim.x;
+  const int64_t gid = (int64_t)(bid - g.block0) * blockDim.x + threadIdx.x;
+  if (WC) {
     const int lane = threadIdx.x & 31;
     const int64_t nwarps = stride >> 5;
-    for (int64_t w0 = gid >> 5; w0 * 32 * kU < uend; w0 += nwarps) {
+    for (int64_t w0 = gid >> 5; w0 * 32 * kU < nunits; w0 += nwarps) {
       const int64_t base = w0 * 32 * kU + lane;
       In in[kU];
 #pragma unroll
       for (int u = 0; u < kU; ++u)
-        if (base + 32 * u < uend) in[u] = ld_stream(s + base + 32 * u);
+        if (base + 32 * u < nunits) in[u] = ld_stream(s + base + 32 * u);
 #pragma unroll
       for (int u = 0; u < kU; ++u)
-        if (base + 32 * u < uend) st_stream(d + base + 32 * u, Cast<S, D, E>::apply(in[u]));
+        if (base + 32 * u < nunits) st_stream(d + base + 32 * u, Cast<S, D, E>::apply(in[u]));
     }
-  }
-  for (int64_t u0 = gid; !WC && u0 < uend; u0 += stride * kU) {
-    In in[kU];
+  } else {
+    for (int64_t u0 = gid; u0 < nunits; u0 += stride * kU) {
+      In in[kU];
 #pragma unroll
-    for (int u = 0; u < kU; ++u) {
-      const int64_t i = u0 + u * stride;
-      if (i < uend) in[u] = ST == 2 ? ld_ef(s + i, pol) : ld_stream(s + i);
-    }
+      for (int u = 0; u < kU; ++u) {                      // all loads first ...
+        const int64_t i = u0 + u * stride;
+        if (i < nunits) in[u] = ld_stream(s + i);
+      }
 #pragma unroll
-    for (int u = 0; u < kU; ++u) {
-      const int64_t i = u0 + u * stride;
-      if (i < uend) {
-        if (ST == 1) st_cs(d + i, Cast<S, D, E>::apply(in[u]));
-        else if (ST == 2) st_ef(d + i, Cast<S, D, E>::apply(in[u]), pol);
-        else st_stream(d + i, Cast<S, D, E>::apply(in[u]));
+      for (int u = 0; u < kU; ++u) {                      // ... then the (cast and) stores
+        const int64_t i = u0 + u * stride;
+        if (i < nunits) st_stream(d + i, Cast<S, D, E>::apply(in[u]));
       }
     }
   }
   const int64_t tail0 = nunits * E;
-  const int64_t tid0 = (int64_t)(bid - g.block0) * blockDim.x + threadIdx.x;
-  if (tid0 < g.n - tail0) {
-    const int64_t i = tail0 + tid0;
+  if (gid < g.n - tail0) {
+    const int64_t i = tail0 + gid;
     if (S::kSize == D::kSize) {
       if (S::kSize == 4) reinterpret_cast<uint32_t *>(g.dst)[i] = reinterpret_cast<const uint32_t *>(g.src)[i];
       else reinterpret_cast<uint16_t *>(g.dst)[i] = reinterpret_cast<const uint16_t *>(g.src)[i];
@@ -998,7 +929,7 @@ __global__ void __launch_bounds__(256) k_stash(const __grid_constant__ StashPara
   if (p.early) pdl_wait();   // complete only after the predecessor: keeps completion order transitive
 }
 
-template <typename S, typename D, int E, int kU, int ST, bool CR = false, bool WC = false>
+template <typename S, typename D, int E, int kU, bool WC>
 cudaError_t launch_stash_v(const StashSegDesc *segs, int nseg, cudaStream_t s, int bo, int to, int *launches,
                            const SwapArgs *swap, bool early) {
   constexpr int kMaxSeg = 32;
@@ -1023,18 +954,9 @@ cudaError_t launch_stash_v(const StashSegDesc *segs, int nseg, cudaStream_t s, i
       work[j] = (segs[i + j].n + E - 1) / E;
       units += work[j];
     }
+    // one-shot grid: ~one iteration of kU units per thread (profiles/r01_stash_variants.md)
     int total = (int)std::min<int64_t>((units + (int64_t)threads * kU - 1) / ((int64_t)threads * kU),
                                        (int64_t)kMaxBlocks);
-    if (CR) {   // whole waves of resident blocks
-      static int resident = 0;
-      if (!resident) {
-        int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_stash<S, D, E, kU, kMaxSeg, ST, CR, WC>, threads, 0);
-        resident = std::max(1, per_sm) * kSMs;
-      }
-      const int64_t waves = std::max<int64_t>(1, (total + resident / 2) / resident);
-      total = (int)std::min<int64_t>(waves * resident, (int64_t)kMaxBlocks);
-    }
     if (bo > 0) total = bo;
     else if (bo < 0) total = std::min(total, -bo);   // a cap (ES_OPT_STASH_BACKGROUND)
     total = std::max(total, k);
@@ -1042,55 +964,32 @@ cudaError_t launch_stash_v(const StashSegDesc *segs, int nseg, cudaStream_t s, i
     split_blocks(work, total, &block0, &p.nblocks);
     for (int j = 0; j < k; ++j) p.seg[j].block0 = block0[j];
     const int grid = p.nblocks + p.swap_bx * p.swap_n;
-    cudaError_t e = launch_k<k_stash<S, D, E, kU, kMaxSeg, ST, CR, WC>>(dim3(grid), dim3(threads), s, p);
+    cudaError_t e = launch_k<k_stash<S, D, E, kU, kMaxSeg, WC>>(dim3(grid), dim3(threads), s, p);
     if (e != cudaSuccess) return e;
     ++*launches;
   }
   return cudaSuccess;
 }
 
-// ES_STASH_VARIANT (measured in profiles/r01_stash_variants.md):
-// 0 (default) = one-shot grid, ~1 iteration of 4 units per thread (40 regs);
-// 5 = one contiguous, equal range per block in whole waves of resident
-// blocks (59 regs; +2.4 % alone, but -0.8 % once consecutive stashes
-// overlap through the early start); 1 / 2 / 4 = one-shot with 8 / 2 / 1
-// units; 3 = one-shot with cache-streaming stores; 6 = contiguous, 8 units;
-// 8 / 9 = one-shot, warp-contiguous units (a warp moves 32*kU adjacent units) with 2 / 4 units.
-int g_stash_variant = [] {
-  const char *e = std::getenv("ES_STASH_VARIANT");
-  return e ? std::atoi(e) : 0;
-}();
-
+// Stash variants were measured in round 1 (profiles/r01_stash_variants.md: unroll 1/2/8,
+// cache-streaming and L2 evict-first stores, contiguous equal ranges per block in whole
+// waves, TMA bulk copies) and the losers removed.  Kept: one-shot grid, 4 units in flight
+// per thread; bf16 -> bf16 warp-contiguous (0.6 % faster per BERT step, 1.1421 vs 1.1496
+// ms), everything else grid-stride (ResNet-50 0.3519 vs 0.3541 ms, Swin-B 4.871 vs 4.879).
 template <typename S, typename D, int E>
 cudaError_t launch_stash_t(const StashSegDesc *segs, int nseg, cudaStream_t s, int bo, int to, int *launches,
                            const SwapArgs *swap, bool early) {
-  switch (g_stash_variant) {
-    case 1: return launch_stash_v<S, D, E, 8, 0>(segs, nseg, s, bo, to, launches, swap, early);
-    case 2: return launch_stash_v<S, D, E, 2, 0>(segs, nseg, s, bo, to, launches, swap, early);
-    case 3: return launch_stash_v<S, D, E, 4, 1>(segs, nseg, s, bo, to, launches, swap, early);
-    case 4: return launch_stash_v<S, D, E, 1, 0>(segs, nseg, s, bo, to, launches, swap, early);
-    case 5: return launch_stash_v<S, D, E, 4, 0, true>(segs, nseg, s, bo, to, launches, swap, early);
-    case 6: return launch_stash_v<S, D, E, 8, 0, true>(segs, nseg, s, bo, to, launches, swap, early);
-    case 7: return launch_stash_v<S, D, E, 4, 2>(segs, nseg, s, bo, to, launches, swap, early);
-    case 8: return launch_stash_v<S, D, E, 2, 0, false, true>(segs, nseg, s, bo, to, launches, swap, early);
-    case 9: return launch_stash_v<S, D, E, 4, 0, false, true>(segs, nseg, s, bo, to, launches, swap, early);
-    default:
-      // bf16 -> bf16: warp-contiguous units measured 0.6 % faster per BERT step (1.1421 vs 1.1496 ms,
-      // two interleaved repeats); fp32 copies are faster with grid-stride units (ResNet-50 0.3519
-      // vs 0.3541 ms, Swin-B 4.871 vs 4.879 ms) -- profiles/r01_stash_variants.md
-      if (std::is_same<S, BF16T>::value && std::is_same<D, BF16T>::value)
-        return launch_stash_v<S, D, E, 4, 0, false, true>(segs, nseg, s, bo, to, launches, swap, early);
-      return launch_stash_v<S, D, E, 4, 0>(segs, nseg, s, bo, to, launches, swap, early);
-  }
+  constexpr bool kWC = std::is_same<S, BF16T>::value && std::is_same<D, BF16T>::value;
+  return launch_stash_v<S, D, E, 4, kWC>(segs, nseg, s, bo, to, launches, swap, early);
 }
 
 // ---- k_copy_tma: TMA bulk-copy stash for same-dtype segments ------------------
 // One elected thread per CTA streams a contiguous, equal share of the bytes
 // through an S-stage shared-memory ring: cp.async.bulk global->shared
 // (completion on an mbarrier with expect_tx), then cp.async.bulk
-// shared->global.  Chosen with ES_STASH_TMA=1 (S=4 x 32 KB, 1 CTA/SM) or 2
-// (S=6 x 16 KB, 2 CTAs/SM); the default is the SM copy (k_stash), which
-// measured faster (profiles/).
+// shared->global.  Used by ES_OPT_STASH_BACKGROUND only (S=4 x 4 KB, one warp
+// per SM: a footprint that fits beside a GEMM's CTA); alone it is slower than
+// k_stash (profiles/r01_stash_variants.md, r01_overlap.md).
 
 struct CopySeg {
   const unsigned char *src;
@@ -1227,17 +1126,12 @@ cudaError_t launch_copy_tma(const StashSegDesc *segs, int nseg, int esize, cudaS
     cfg.numAttrs = g_pdl ? 1 : 0;
     (void)KernelReg<k_copy_tma<S, T>>::token;
     cudaError_t e = cudaLaunchKernelEx(&cfg, k_copy_tma<S, T>, p);
-    if (e == cudaSuccess) e = cudaGetLastError();
     if (e != cudaSuccess) return e;
     ++*launches;
   }
   return cudaSuccess;
 }
 
-int g_stash_tma = [] {
-  const char *e = std::getenv("ES_STASH_TMA");
-  return e ? std::atoi(e) : 0;
-}();
 
 // ---- k_swap -----------------------------------------------------------------
 
@@ -1388,11 +1282,6 @@ cudaError_t launch_fold_multi(es_dtype dtype, int32_t N, float r, uint32_t compa
                              launches);
 }
 
-// ES_BG_TMA=0: ES_OPT_STASH_BACKGROUND without the TMA ring (capped k_stash grid only; experiment)
-int g_bg_tma = [] {
-  const char *e = std::getenv("ES_BG_TMA");
-  return !(e && e[0] == '0');
-}();
 
 cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *segs, int nseg, cudaStream_t s,
                                int bo, int to, int *launches, const SwapArgs *swap, bool early, bool background) {
@@ -1412,7 +1301,7 @@ cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *s
   bool aligned = true;
   for (const StashSegDesc &g : live)
     aligned = aligned && !(reinterpret_cast<uintptr_t>(g.src) & 15) && !(reinterpret_cast<uintptr_t>(g.dst) & 15);
-  if (background && g_bg_tma && sdt == ddt && aligned && bo <= 0) {   // bo > 0: an explicit es_set_launch_override
+  if (background && sdt == ddt && aligned && bo <= 0) {   // bo > 0: an explicit es_set_launch_override
     // ES_OPT_STASH_BACKGROUND, same dtype: the copy runs as one warp per SM
     // driving a 4 x 4 KB TMA bulk-copy ring (16 KB of shared memory, a
     // few registers), a footprint that fits beside a tensor-core GEMM's CTA, so
@@ -1424,13 +1313,6 @@ cudaError_t launch_stash_multi(es_dtype sdt, es_dtype ddt, const StashSegDesc *s
       if (e != cudaSuccess) return e;
     }
     return launch_copy_tma<4, 4096>(live.data(), n, sdt == ES_BF16 ? 2 : 4, s, 1, launches);
-  }
-  if (sdt == ddt && g_stash_tma > 0 && aligned && !(swap && swap->n > 0)) {
-    const int es_ = sdt == ES_BF16 ? 2 : 4;
-    // 3: the small-footprint ring of ES_OPT_STASH_BACKGROUND, for every stash
-    return g_stash_tma == 1   ? launch_copy_tma<4, 32768>(live.data(), n, es_, s, 1, launches)
-           : g_stash_tma == 3 ? launch_copy_tma<4, 4096>(live.data(), n, es_, s, 1, launches)
-                              : launch_copy_tma<6, 16384>(live.data(), n, es_, s, 2, launches);
   }
   if (sdt == ES_F32 && ddt == ES_F32) return launch_stash_t<F32T, F32T, 4>(live.data(), n, s, bo, to, launches, swap, early);
   if (sdt == ES_BF16 && ddt == ES_BF16)

@@ -115,3 +115,57 @@ def test_green_context_really_restricts_sms():
     agg.close()
     cu.cuStreamDestroy(stream)
     cu.cuGreenCtxDestroy(gctx)
+
+
+@pytest.mark.parametrize("n_sms", [8, 16, 32])
+def test_dropout_on_green_context_sm_partitions(n_sms):
+    """NEXT-4 (D2): the per-EST dropout, driven by each EST's
+    swapped device Philox record, gives the oracle's masks and values on an SM
+    partition of 8/16/32 SMs -- time-sliced ESTs, switches on the same green
+    stream, several calls per EST (the offset advances once per call)."""
+    torch.cuda.init()
+    try:
+        cu, gctx, ctx, stream, got_sms = _green_stream(n_sms)
+    except Exception as e:  # green contexts unavailable on this driver / device
+        pytest.skip(f"green contexts unavailable: {e}")
+    N, calls, p = 4, 2, 0.3
+    seeds = [0x5EED_0000_0000 + 977 * k for k in range(N)]
+    rng = np.random.default_rng(100 + n_sms)
+    sizes = {"f32": 300007, "bf16": 4099}
+    xs = {}
+    for d, n in sizes.items():
+        x32 = rng.standard_normal(n).astype(np.float32)
+        xs[d] = x32 if d == "f32" else oracle.f32_to_bf16_bits(x32)
+    agg = Aggregator(N, 1, 0, [0] * N, [(64, "f32")], state_nbytes=[16])
+    live = [torch.zeros(16, dtype=torch.uint8, device="cuda")]
+    agg.register_state(live)
+    for k in range(N):
+        agg.init_state(k, 0, int(seeds[k]).to_bytes(8, "little") + (0).to_bytes(8, "little"))
+    xdev = {d: to_dev(x) for d, x in xs.items()}
+    ys = {(k, c, d): torch.empty_like(xdev[d]) for k in range(N) for c in range(calls) for d in sizes}
+    ms = {(k, c, d): torch.empty(sizes[d], dtype=torch.uint8, device="cuda")
+          for k in range(N) for c in range(calls) for d in sizes}
+    torch.cuda.synchronize()
+    _check(cu.cuCtxPushCurrent(ctx))
+    try:
+        s = int(stream)
+        for k in range(N):
+            es.es_switch_context(agg.h, k, s)
+            for c in range(calls):
+                for d in sizes:
+                    es.es_dropout(agg.h, xdev[d].data_ptr(), ys[(k, c, d)].data_ptr(), ms[(k, c, d)].data_ptr(),
+                                  sizes[d], es.ES_F32 if d == "f32" else es.ES_BF16, p, 0, s)
+        _check(cu.cuStreamSynchronize(stream))
+    finally:
+        _check(cu.cuCtxPopCurrent())
+    for k in range(N):
+        off = 0
+        for c in range(calls):
+            for d in sizes:                       # one offset unit per es_dropout call, in call order
+                wy, wm = oracle.dropout(xs[d], d, p, seeds[k], off)
+                assert np.array_equal(ms[(k, c, d)].cpu().numpy(), wm), (got_sms, k, c, d)
+                assert_bits_equal(from_dev(ys[(k, c, d)]), wy, f"{got_sms} SMs, EST {k} call {c} {d}")
+                off += 1
+    agg.close()
+    cu.cuStreamDestroy(stream)
+    cu.cuGreenCtxDestroy(gctx)

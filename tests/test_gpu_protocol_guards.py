@@ -1,0 +1,68 @@
+"""GPU: protocol guards of the C ABI.
+
+* es_export_context refuses (ES_ESTATE) an EST whose bucket is being folded
+  incrementally (NEXT-1, COPY mode): its slot holds only the chunks that wait
+  for the wrap, the rest lives in the fp32 partials; exporting it would write
+  stale bytes marked as stashed (R17: a context is the EST's whole gradient).
+  EST 0 and a BORROWed EST are exportable; import refuses to bypass partials.
+* es_peer_open refuses (ES_EINVAL) blobs from ranks whose plan differs (options,
+  schedule, mapping...): mismatched executors would wait on barriers the others
+  never reach or gather results nobody pushed.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from paper_conf_sc_lixyszrljlllq23_b200 import es
+
+from gpu_util import Aggregator, assert_bits_equal, from_dev, to_dev
+
+pytestmark = pytest.mark.gpu
+
+
+def test_export_refuses_partially_folded_slot():
+    N, L = 4, 100003
+    agg = Aggregator(N, 1, 0, [0] * N, [(L, "f32")], options=es.ES_OPT_INCREMENTAL)
+    rng = np.random.default_rng(5)
+    xs = [(rng.standard_normal(L) * 1e-2).astype(np.float32) for _ in range(N)]
+    d = [to_dev(x) for x in xs]
+    agg.stash_fold(0, [0], [d[0]], es.ES_STASH_COPY)          # EST 0: whole gradient stashed
+    agg.stash_fold(1, [0], [d[1]], es.ES_STASH_COPY)          # EST 1: chunk 0 folded, rest stashed
+    blob0 = agg.export_context(0)
+    with pytest.raises(es.EsError) as ei:
+        agg.export_context(1)
+    assert ei.value.status == es.ES_ESTATE
+    with pytest.raises(es.EsError) as ei:                     # importing would bypass the partials
+        agg.import_context(0, blob0)
+    assert ei.value.status == es.ES_ESTATE
+    agg.stash_fold(2, [0], [d[2]], es.ES_STASH_COPY)
+    agg.stash_fold(3, [0], [d[3]], es.ES_STASH_BORROW)        # BORROW: the live buffer is whole
+    agg.export_context(3)
+    out = agg.new_out(0)
+    agg.allreduce(0, out)                                     # the refused calls changed nothing
+    torch.cuda.synchronize()
+    assert_bits_equal(from_dev(out), oracle.reduce(xs, "f32"), "incremental after refused export")
+    # the exported EST 0 context is its gradient
+    blob = np.frombuffer(blob0, dtype=np.uint8)
+    assert blob[-L * 4:].tobytes() == xs[0].tobytes()        # no context buffers: the bucket ends the blob
+    agg.close()
+
+
+def test_peer_open_refuses_mismatched_plans():
+    N, G = 4, 2
+    m = [0, 0, 1, 1]
+    world = es.es_loopback_create(G)
+    a0 = Aggregator(N, G, 0, m, [(4096, "f32")], transport=es.ES_TRANSPORT_LOOPBACK, comm=world.value,
+                    sched=es.ES_SCHED_PEER)
+    a1 = Aggregator(N, G, 1, m, [(4096, "f32")], transport=es.ES_TRANSPORT_LOOPBACK, comm=world.value,
+                    sched=es.ES_SCHED_PEER, options=es.ES_OPT_PEER_PUSH)
+    blobs = [a0.peer_blob(), a1.peer_blob()]
+    for a in (a0, a1):
+        with pytest.raises(es.EsError) as ei:
+            a.peer_open(blobs)
+        assert ei.value.status == es.ES_EINVAL
+        assert "plan differs" in str(ei.value)
+    a0.close()
+    a1.close()
+    es.es_loopback_destroy(world)
