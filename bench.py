@@ -8,8 +8,15 @@ each bucket (k_stash; the last local EST is borrowed),
 then es_allreduce of every bucket (exchange + canonical fold + 1/N + gather).
 value = N * sum_b L_b * bytes / step time (whole job; inputs resident in HBM).
 
-  python bench.py [--gpus N --steps K --warmup W] [--config resnet50] [--impl reference]
-  (N > 1: torchrun --nproc-per-node N ... bench.py --gpus N ...; NCCL transport)
+  python bench.py [--gpus N --steps K --warmup W] [--config swin_b] [--impl reference]
+  (N > 1: torchrun --nproc-per-node N ... bench.py --gpus N ...; peer-memory
+   schedules over NVLink with a fallback ladder down to the NCCL transport)
+
+Default workload: Swin-B, N=32 ESTs (BASELINE configs[4], the largest config
+that fits one GPU: 11.2 GB of EST gradients per step, a Philox/BN context swap
+at every switch).  The inputs are drawn on the host (workloads.host_inputs,
+NumPy Philox) and copied to HBM before anything is timed; rank 0 checks the
+WHOLE output against the C oracle on every host core.
 
 Prints ONE JSON line on rank 0.  See DESIGN.md "Measurement".
 """
@@ -29,26 +36,29 @@ sys.path.insert(0, ROOT)
 METRIC = "EST-gradient GB/s reduced (bit-exact across G) at 1/2/4/8 B200; % of roofline"
 L2_BYTES = 126 * 1024 * 1024
 HBM_NOMINAL_GBPS = 8000.0     # B200 HBM3e nominal (SURVEY 8(d) t_roof uses 8.0 TB/s); `frac` uses the measured peak
+NVL_MEASURED_GBPS = 770.0     # B200_PROFILING.md: measured peer copy per direction per GPU
+NVL_NOMINAL_GBPS = 900.0      # NVLink 5, per direction per GPU
 
 
-def parse():
+def parse(argv=None):
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=50)
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--impl", default="es200", choices=["es200", "reference"])
-    p.add_argument("--config", default="resnet50",
+    p.add_argument("--config", default="swin_b",
                    choices=["tiny", "resnet50", "vgg19", "bert_base", "swin_b"])
     p.add_argument("--mapping", default="contiguous", choices=["contiguous", "round_robin", "random"])
     p.add_argument("--sched", default=None, choices=["auto", "direct", "chain", "peer", "peer_chain", "peer_auto"],
-                   help="default: auto at G=1; peer_auto at G>1 (fused folds over NVLink peer memory, CUDA IPC)")
+                   help="default: auto at G=1; peer_auto at G>1 (fused folds over NVLink peer memory, CUDA IPC), "
+                        "falling back to peer_auto + ES_OPT_PEER_ROUNDS, then to the NCCL transport (auto)")
     p.add_argument("--no-graph", action="store_true", help="eager launches instead of one CUDA graph per step")
     p.add_argument("--per-bucket", action="store_true",
                    help="one es_stash_grad / es_allreduce call per bucket (DDP-style) instead of the batched calls")
     p.add_argument("--no-fuse", action="store_true",
                    help="separate es_switch_context and es_stash_grads launches instead of es_stash_and_switch")
     p.add_argument("--incremental", action="store_true",
-                   help="NEXT-1: fold each EST into running partials at its switch (es_stash_fold_grads, G == 1)")
+                   help="NEXT-1: fold each EST into running partials at its switch (es_stash_fold_grads)")
     p.add_argument("--inplace", action="store_true",
                    help="NEXT-2 zero-copy stash: each EST's gradients are produced in its slot (es_slot_ptr) and "
                         "stashed with ES_STASH_INPLACE")
@@ -59,10 +69,20 @@ def parse():
     p.add_argument("--rehearse-same-gpu", action="store_true",
                    help="functional rehearsal of the N>1 path on ONE GPU: every rank on cuda:0, gloo process "
                         "group, a peer schedule (CUDA IPC, no NCCL); times are not GPU-scaling numbers")
+    p.add_argument("--simulate-peer-failure", default=None, choices=["open", "parity"],
+                   help="test hook (G>1): the first rung of the schedule ladder fails as if es_peer_open had "
+                        "returned ES_EUNSUPPORTED on the last rank (open) or its first-step oracle check had "
+                        "failed on rank 0 (parity); bench must fall back and still print a bit-exact line")
+    p.add_argument("--no-ring-check", action="store_true", help="skip NEXT-3 (iii), the NCCL ring cross-check (N == G)")
+    p.add_argument("--no-full-parity", action="store_true", help="check sampled windows only (not the whole output)")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     p.add_argument("--cpu-seconds", type=float, default=10.0)
-    return p.parse_args()
+    return p.parse_args(argv)
+
+
+def default_sched(args, world):
+    return args.sched or ("peer_auto" if world > 1 else "auto")
 
 
 def peaks():
@@ -79,6 +99,24 @@ def cores_used():
         return len(os.sched_getaffinity(0))
     except Exception:
         return os.cpu_count()
+
+
+def cpu_model():
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            if line.startswith("Model name:"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return None
 
 
 # ---- clocks sampler ------------------------------------------------------------------------
@@ -101,9 +139,6 @@ class Clocks:
         except Exception:
             self.proc = None
         self.t0 = time.time()
-
-    def mark(self):
-        return time.time()
 
     def stop(self, t_start, t_end):
         if self.proc is None:
@@ -134,12 +169,196 @@ class Clocks:
                 "reasons": reasons, "samples": len(win)}
 
 
-# ---- oracle legs (cpu_baseline / --impl reference) -----------------------------------------
+# ---- NVLink: device facts and byte counters (NVML) --------------------------------------------
 
-def oracle_windows(name, fetch, budget_s, seed=0):
-    """Times the oracle, as it stands (single thread), on windows of every
-    bucket until ~budget_s of CPU work.  fetch(k, b, s, n) -> EST k's bucket b
-    elements [s, s+n) as numpy.  Returns (GB/s, sample text, [(b, s, n, out)])."""
+class NvLink:
+    """Per-GPU NVLink facts and data counters through NVML (nvidia_ml_py).
+    Data counters: NVML_FI_DEV_NVLINK_THROUGHPUT_DATA_TX/RX (KiB, per link,
+    payload only), summed over the active links."""
+    FI_TX, FI_RX = 138, 139
+
+    def __init__(self, uuid):
+        self.ok, self.why, self.links = False, None, []
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            u = str(uuid)
+            self.h = pynvml.nvmlDeviceGetHandleByUUID(u if u.startswith("GPU-") else "GPU-" + u)
+            for l in range(18):
+                try:
+                    if pynvml.nvmlDeviceGetNvLinkState(self.h, l) == 1:
+                        self.links.append(l)
+                except Exception:
+                    break
+            self.ok = True
+        except Exception as e:  # NVML missing or no such device
+            self.why = f"NVML unavailable: {e}"
+
+    def read(self):
+        """(tx_bytes, rx_bytes) summed over active links, or None."""
+        if not self.ok or not self.links:
+            return None
+        try:
+            fields = [(self.FI_TX, l) for l in self.links] + [(self.FI_RX, l) for l in self.links]
+            vals = self.nv.nvmlDeviceGetFieldValues(self.h, fields)
+            tx = rx = 0
+            for i, v in enumerate(vals):
+                if v.nvmlReturn != 0:
+                    self.why = f"NVML field {fields[i]} returned {v.nvmlReturn}"
+                    return None
+                kib = int(v.value.ullVal)
+                if i < len(self.links):
+                    tx += kib
+                else:
+                    rx += kib
+            return tx * 1024, rx * 1024
+        except Exception as e:
+            self.why = f"NVML field read failed: {e}"
+            return None
+
+
+# ---- the multi-GPU roofline of the exported plan (SURVEY 8(d)) ---------------------------------
+
+def plan_costs(buckets, N, G, mapping, sched, options=0, borrow_last=True):
+    """Per-rank algorithmic bytes of one es_allreduce_many over every bucket, from the op lists
+    each rank EXPORTS (es_plan_ops: the plan the executor walks), for the roofline.
+
+    Returns (costs, scheds): costs[g] = {"hbm", "nvl_in", "nvl_out", "phases": [(hbm, in, out), ...],
+    "kinds": {kind: [hbm, nvl_in]}} and scheds[b] = the schedule bucket b runs.
+      * FOLD: every contribution read (a remote EST's slot under a PEER schedule = NVLink in from its
+        GPU, else HBM: own slot / borrowed gradient / staging), the incoming partial (HBM, or NVLink
+        for a PEER_CHAIN producer), the output write (HBM);
+      * SEND / RECV (NCCL transport): NVLink out / in, plus the HBM read / write of the buffer;
+      * GATHER (PEER): a remote owner's RESULT = NVLink in + HBM write; the own = HBM read + write;
+      * PEER buckets with a BORROWed last EST: the slot copy of the ranges peers read (HBM, 2x).
+    Phases are the executor's: barriers (PEER*: phase k of every bucket is one merged launch),
+    groups (NCCL transport: bucket by bucket); a pipelined PEER_CHAIN step (k_fold_pipe, the
+    default) runs all its fold rounds as one phase."""
+    from paper_conf_sc_lixyszrljlllq23_b200 import es
+    pipelined = not (options & es.ES_OPT_PEER_ROUNDS)
+    costs, scheds = [], None
+    bl = [(n, es.ES_F32 if d in ("f32", es.ES_F32) else es.ES_BF16) for n, d in buckets]
+    for g in range(G):
+        cfg = es.Config(N, G, g, mapping, bl, sched=sched, options=options & ~es.ES_OPT_INCREMENTAL)
+        ph = {}
+        kinds = {}
+        sch = []
+
+        def add(p, kind, hbm=0, nvl_in=0, src=None):
+            e = ph.setdefault(p, [0, 0, [0] * G])
+            e[0] += hbm
+            e[1] += nvl_in
+            if src is not None and nvl_in:
+                e[2][src] += nvl_in
+            k = kinds.setdefault(kind, [0, 0])
+            k[0] += hbm
+            k[1] += nvl_in
+        for b, (L, dt) in enumerate(bl):
+            esz = 2 if dt == es.ES_BF16 else 4
+            ops, s = es.es_plan_ops(cfg, b)
+            sch.append(s)
+            peer = s in (es.ES_SCHED_PEER, es.ES_SCHED_PEER_CHAIN)
+            if s == es.ES_SCHED_PEER and borrow_last and L > 0:
+                own = [o for o in ops if int(o[0]) == es.ES_OP_FOLD]
+                shard = int(own[0][2] - own[0][1]) if own else 0
+                add((0, -1), "stash", hbm=2 * (L - shard) * esz)
+            k = 0
+            for f in ops:
+                op = int(f[0])
+                if op in (es.ES_OP_BARRIER, es.ES_OP_GROUP_BEGIN, es.ES_OP_GROUP_END):
+                    k += 1
+                    continue
+                # peer schedules: phase k of every bucket runs as one merged launch (peer_allreduce);
+                # NCCL transport: bucket after bucket, group by group
+                if peer and s == es.ES_SCHED_PEER_CHAIN and pipelined:
+                    p = (0, 2) if op == es.ES_OP_GATHER else (0, 1)
+                elif peer:
+                    p = (0, k)
+                else:
+                    p = (1 + b, k)
+                lo, hi = int(f[1]), int(f[2])
+                n = hi - lo
+                if op == es.ES_OP_FOLD:
+                    ests = range(N) if int(f[3]) < 0 else [(int(f[3]) + t) % N for t in range(int(f[4]))]
+                    for e in ests:
+                        if peer and mapping[e] != g:
+                            add(p, "fold", nvl_in=n * esz, src=mapping[e])
+                        else:
+                            add(p, "fold", hbm=n * esz)
+                    if int(f[5]) == es.ES_BUF_PART:
+                        add(p, "fold", hbm=n * 4)
+                    elif int(f[5]) == es.ES_BUF_PEER_PART:
+                        add(p, "fold", nvl_in=n * 4, src=int(f[6]))
+                    add(p, "fold", hbm=n * (4 if int(f[7]) == es.ES_BUF_PART else esz))
+                elif op in (es.ES_OP_SEND, es.ES_OP_RECV):
+                    w = 4 if int(f[4]) == es.ES_BUF_PART else esz
+                    if op == es.ES_OP_RECV:
+                        add(p, "xfer", hbm=n * w, nvl_in=n * w, src=int(f[3]))
+                    else:
+                        add(p, "xfer", hbm=n * w)
+                elif op == es.ES_OP_GATHER:
+                    src = int(f[3])
+                    if src != g:
+                        add(p, "gather", hbm=n * esz, nvl_in=n * esz, src=src)
+                    else:
+                        add(p, "gather", hbm=2 * n * esz)
+        costs.append({"phases": ph, "kinds": kinds})
+        scheds = scheds or sch
+    # NVLink out of rank h = what every other rank reads / receives from h
+    for g in range(G):
+        c = costs[g]
+        out_by_phase = {}
+        for h in range(G):
+            for p, (_, _, src) in costs[h]["phases"].items():
+                out_by_phase[p] = out_by_phase.get(p, 0) + src[g]
+        c["phase_list"] = [(v[0], v[1], out_by_phase.get(p, 0)) for p, v in sorted(c["phases"].items())]
+        c["hbm"] = sum(v[0] for v in c["phase_list"])
+        c["nvl_in"] = sum(v[1] for v in c["phase_list"])
+        c["nvl_out"] = sum(v[2] for v in c["phase_list"])
+    for c in costs:
+        del c["phases"]
+    return costs, scheds
+
+
+def plan_roofline(costs, t_ms, hbm_gbps, nvl_gbps=NVL_MEASURED_GBPS):
+    """t_roof = max over ranks of max(HBM / HBM peak, NVLink in or out / NVLink peak)
+    (every byte overlapped); t_roof_phased = the slowest rank's sum over its executor phases of
+    the same max (phases separated by barriers / groups cannot overlap).  `bound` names the term
+    that sets t_roof; frac = t_roof / measured time."""
+    def ms(b, gbps):
+        return b / (gbps * 1e9) * 1e3
+    worst, bound, t_roof = None, None, 0.0
+    for g, c in enumerate(costs):
+        th, tn = ms(c["hbm"], hbm_gbps), ms(max(c["nvl_in"], c["nvl_out"]), nvl_gbps)
+        t = max(th, tn)
+        if t > t_roof:
+            t_roof, worst, bound = t, g, ("nvlink" if tn > th else "hbm")
+    phased = max(sum(max(ms(h, hbm_gbps), ms(max(i, o), nvl_gbps)) for h, i, o in c["phase_list"]) for c in costs)
+    w = costs[worst] if worst is not None else {"hbm": 0, "nvl_in": 0, "nvl_out": 0}
+    nvl_bytes = max(w["nvl_in"], w["nvl_out"])
+    achieved = (nvl_bytes if bound == "nvlink" else w["hbm"]) / (t_ms / 1e3) / 1e9 if t_ms > 0 else None
+    peak = nvl_gbps if bound == "nvlink" else hbm_gbps
+    return {"bound": bound, "achieved": round(achieved, 1) if achieved else None, "peak": peak, "unit": "GB/s",
+            "frac": round(achieved / peak, 4) if achieved else None,
+            "t_roof_ms": round(t_roof, 4), "t_roof_phased_ms": round(phased, 4), "t_measured_ms": round(t_ms, 4),
+            "frac_of_t_roof": round(t_roof / t_ms, 4) if t_ms > 0 else None,
+            "frac_of_t_roof_phased": round(phased / t_ms, 4) if t_ms > 0 else None,
+            "slowest_rank": worst,
+            "per_rank_MB": [{"hbm": round(c["hbm"] / 1e6, 2), "nvl_in": round(c["nvl_in"] / 1e6, 2),
+                             "nvl_out": round(c["nvl_out"] / 1e6, 2)} for c in costs],
+            "peaks": {"hbm_gbps": hbm_gbps, "nvlink_gbps": nvl_gbps,
+                      "nvlink_source": "B200_PROFILING.md measured peer copy per direction (900 nominal)"}}
+
+
+# ---- oracle legs (cpu_baseline / --impl reference / parity) ------------------------------------
+
+def oracle_windows(name, fetch_all, budget_s, seed=0, per_bucket=1):
+    """Times the oracle, as it stands (single thread), on a bounded sample of the
+    workload: `per_bucket` windows of <= 2^18 elements of every bucket (all N ESTs'
+    inputs fetched before the clock starts), folded repeatedly until ~budget_s of
+    CPU time.  fetch_all(b, s, n) -> [EST k's bucket b elements [s, s+n) for k < N].
+    Returns (GB/s, sample text, [(b, s, n, out)] of the first pass)."""
     import numpy as np
     import oracle
     from paper_conf_sc_lixyszrljlllq23_b200 import workloads
@@ -147,28 +366,30 @@ def oracle_windows(name, fetch, budget_s, seed=0):
     N = cfg["N"]
     esz = 2 if cfg["dtype"] == "bf16" else 4
     rng = np.random.default_rng(seed)
-    done_bytes, t_oracle, windows = 0, 0.0, []
     win = 1 << 18
-    t_begin = time.time()
-    while t_oracle < budget_s and time.time() - t_begin < 3 * budget_s:
-        for b, (L, d) in enumerate(cfg["buckets"]):
+    jobs = []
+    for b, (L, d) in enumerate(cfg["buckets"]):
+        for _ in range(per_bucket):
             n = min(win, L)
             s = int(rng.integers(0, L - n + 1))
-            xs = [fetch(k, b, s, n) for k in range(N)]
+            jobs.append((b, s, n, d, L, fetch_all(b, s, n)))
+    done_bytes, t_oracle, windows, passes = 0, 0.0, [], 0
+    while passes == 0 or t_oracle < budget_s:
+        for b, s, n, d, L, xs in jobs:
             t0 = time.perf_counter()
             out = oracle.reduce(xs, d, L=L, first=s)
             t_oracle += time.perf_counter() - t0
             done_bytes += N * n * esz
-            windows.append((b, s, n, out))
-            if t_oracle >= budget_s:
-                break
+            if passes == 0:
+                windows.append((b, s, n, out))
+        passes += 1
     gbs = done_bytes / t_oracle / 1e9
-    sample = (f"{len(windows)} windows of <= {win} elements x {N} ESTs across the {len(cfg['buckets'])} buckets "
-              f"({done_bytes / 1e6:.1f} MB of EST gradients, {t_oracle:.1f} s single-thread C oracle)")
+    sample = (f"{len(jobs)} windows of <= {win} elements x {N} ESTs (one per bucket, {passes} passes; "
+              f"{done_bytes / 1e6:.1f} MB of EST gradients, {t_oracle:.1f} s single-thread C oracle)")
     return gbs, sample, windows
 
 
-def oracle_all_cores(name, fetch, threads, budget_s=3.0, max_bytes=512 << 20, seed=7):
+def oracle_all_cores(name, fetch_all, threads, budget_s=3.0, max_bytes=512 << 20, seed=7):
     """The same unmodified single-thread oracle, one window per host thread at a
     time on every available core (ctypes releases the GIL inside the C call;
     each element's fold order is unchanged).  Inputs are fetched before the
@@ -189,7 +410,7 @@ def oracle_all_cores(name, fetch, threads, budget_s=3.0, max_bytes=512 << 20, se
         L, d = cfg["buckets"][b]
         n = min(win, L)
         s = int(rng.integers(0, L - n + 1))
-        jobs.append(([fetch(k, b, s, n) for k in range(N)], d, L, s, N * n * esz))
+        jobs.append((fetch_all(b, s, n), d, L, s, N * n * esz))
     reps = 0
     with cf.ThreadPoolExecutor(max_workers=threads) as ex:
         t0 = time.perf_counter()
@@ -202,10 +423,63 @@ def oracle_all_cores(name, fetch, threads, budget_s=3.0, max_bytes=512 << 20, se
                              f"EST gradients) on {threads} threads, {dt:.2f} s wall")
 
 
+def oracle_full(buckets, host, N, outs_np, threads, win=1 << 21):
+    """The WHOLE step's output against the oracle on every host core: each bucket in windows,
+    oracle.reduce (the unmodified plain definition) per window on a thread pool.  Returns
+    (mismatched words, oracle SHA-256 of all buckets in order, seconds)."""
+    import concurrent.futures as cf
+    import numpy as np
+    import oracle
+    t0 = time.perf_counter()
+    jobs = []
+    for b, (L, d) in enumerate(buckets):
+        for s in range(0, L, win):
+            jobs.append((b, s, min(win, L - s)))
+
+    def run(j):
+        b, s, n = j
+        L, d = buckets[b]
+        want = oracle.reduce([host[(k, b)][s:s + n] for k in range(N)], d, L=L, first=s)
+        got = outs_np[b][s:s + n]
+        w = want.view(np.uint32 if want.dtype == np.float32 else np.uint16)
+        return want, int((w != got.view(w.dtype)).sum())
+    h, mism = hashlib.sha256(), 0
+    with cf.ThreadPoolExecutor(max_workers=threads) as ex:
+        for want, m in ex.map(run, jobs):           # in order: the hash is over the buckets in bucket order
+            h.update(want.tobytes())
+            mism += m
+    return mism, h.hexdigest(), time.perf_counter() - t0
+
+
+def first_step_check(name, buckets, N, outs, host, seed=11, n=4099):
+    """Sampled first-step parity (fallback ladder): 3 windows of every bucket of the first eager
+    step's output against the oracle; remote ESTs' windows are drawn from their seeded streams."""
+    import numpy as np
+    import oracle
+    from paper_conf_sc_lixyszrljlllq23_b200 import workloads
+    rng = np.random.default_rng(seed)
+    bad = 0
+    for b, (L, d) in enumerate(buckets):
+        if L == 0:
+            continue
+        for s in sorted({0, max(0, L - n), int(rng.integers(0, max(1, L - n)))}):
+            m = min(n, L - s)
+            miss = [k for k in range(N) if (k, b) not in host]
+            drawn = dict(zip(miss, workloads.window_np(name, b, miss, s, s + m))) if miss else {}
+            xs = [host[(k, b)][s:s + m] if (k, b) in host else drawn[k] for k in range(N)]
+            want = oracle.reduce(xs, d, L=L, first=s)
+            got = outs[b][s:s + m].cpu()
+            got = got.numpy() if d == "f32" else got.view(__import__("torch").int16).numpy().view(np.uint16)
+            bad += int((want.view(got.dtype) != got).sum()) if d == "bf16" else \
+                int((want.view(np.uint32) != got.view(np.uint32)).sum())
+    return bad
+
+
 def workload_config(args, cfg, G):
     """The `config` keys both arms share (the same workload)."""
-    return {"workload": args.config, "N": cfg["N"], "G": G, "mapping": args.mapping, "sched": args.sched,
-            "buckets": len(cfg["buckets"]), "elements": sum(n for n, _ in cfg["buckets"]), "desc": cfg["desc"]}
+    return {"workload": args.config, "N": cfg["N"], "G": G, "mapping": args.mapping,
+            "sched": default_sched(args, G), "buckets": len(cfg["buckets"]),
+            "elements": sum(n for n, _ in cfg["buckets"]), "desc": cfg["desc"]}
 
 
 def run_reference(args, rank, world):
@@ -214,21 +488,21 @@ def run_reference(args, rank, world):
     from paper_conf_sc_lixyszrljlllq23_b200 import workloads
     name = args.config
     cfg = workloads.config(name)
+
     cache = {}
 
-    def fetch(k, b, s, n):
-        if (k, b) not in cache:
-            t = workloads.est_bucket(name, k, b, device="cpu")
-            cache[(k, b)] = t.numpy() if cfg["dtype"] == "f32" else t.view(__import__("torch").int16).numpy().view("uint16")
-        return cache[(k, b)][s:s + n]
+    def fetch_all(b, s, n):             # the seeded host inputs (the GPU arm copies the same arrays)
+        if (b, s, n) not in cache:
+            cache[(b, s, n)] = workloads.window_np(name, b, range(cfg["N"]), s, s + n)
+        return cache[(b, s, n)]
 
     # one "step" = one bounded sample of the workload; K timed samples after W warm-ups
     budget = max(0.5, min(args.cpu_seconds, 60.0 / max(1, args.steps + args.warmup)))
     for _ in range(args.warmup):
-        oracle_windows(name, fetch, budget * 0.2, seed=1)
+        oracle_windows(name, fetch_all, budget * 0.2, seed=100)
     rates, sample = [], ""
     for i in range(args.steps):
-        gbs, sample, _ = oracle_windows(name, fetch, budget, seed=100 + i)
+        gbs, sample, _ = oracle_windows(name, fetch_all, budget, seed=100)   # the same drawn sample per step
         rates.append(gbs)
     value = statistics.median(rates)
     payload = workloads.payload_bytes(name)
@@ -237,10 +511,10 @@ def run_reference(args, rank, world):
         "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GB/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 3), "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": cfg["dtype"], "data": "synthetic",
-        "config": dict(workload_config(args, cfg, world), graph=False, api="C oracle (single thread)",
-                       l2="host memory"),
+        "config": workload_config(args, cfg, world),
+        "arm": {"api": "C oracle (single thread)", "memory": "host"},
         "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-                         "sample": sample + "; ms_per_step extrapolates the full step"},
+                         "sample": sample + "; ms_per_step extrapolates the full step", "cpu_model": cpu_model()},
         "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -248,38 +522,66 @@ def run_reference(args, rank, world):
 
 # ---- the GPU arm ------------------------------------------------------------------------------
 
+class PeerFailure(RuntimeError):
+    pass
+
+
+def ladder(args, world, rehearse):
+    """Schedules to try, in order (G > 1).  Peer schedules map the peers' workspaces through CUDA
+    IPC; if that fails (es_peer_open: ES_EUNSUPPORTED for a non-exportable allocation, ES_ECUDA)
+    or the first step misses the oracle, the next rung runs: PEER_CHAIN without tile pipelining
+    (no cross-GPU per-tile flags), then the NCCL transport (not in the one-GPU rehearsal: NCCL
+    refuses two ranks per device)."""
+    s = default_sched(args, world)
+    if world == 1:
+        return [(s, 0)]
+    if s in ("peer", "peer_chain", "peer_auto"):
+        rungs = [(s, 0), (s, "rounds")]
+        if not rehearse:
+            rungs.append(("auto", 0))
+        return rungs
+    return [(s, 0)]
+
+
 def main():
     args = parse()
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
-    if args.sched is None:
-        args.sched = "peer_auto" if world > 1 else "auto"
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    local_world = int(os.environ.get("LOCAL_WORLD_SIZE", str(world)))
     if args.impl == "reference":
         return run_reference(args, rank, world)
+
+    from paper_conf_sc_lixyszrljlllq23_b200 import workloads
+    name = args.config
+    cfg = workloads.config(name)
+    N, G = cfg["N"], world
+    mapping = workloads.mapping(N, G, args.mapping)
+    local = [k for k in range(N) if mapping[k] == rank]
+    buckets = cfg["buckets"]
+    B = len(buckets)
+    rehearse = args.rehearse_same_gpu and world > 1
+    # Host inputs BEFORE CUDA is initialised (forked workers draw them on this rank's share of the
+    # cores).  Rank 0 also draws the remote ESTs: it checks the whole output against the oracle.
+    need = list(range(N)) if rank == 0 and not args.no_full_parity else local
+    t_gen = time.time()
+    host = workloads.host_inputs(name, need, procs=max(1, cores_used() // max(1, local_world)))
+    t_gen = time.time() - t_gen
 
     import numpy as np
     import torch
     import torch.distributed as dist
 
-    from paper_conf_sc_lixyszrljlllq23_b200 import es, workloads
+    from paper_conf_sc_lixyszrljlllq23_b200 import es
     from paper_conf_sc_lixyszrljlllq23_b200.aggregator import Aggregator, nccl_comm_ptr
 
-    rehearse = args.rehearse_same_gpu and world > 1
-    if rehearse and args.sched not in ("peer", "peer_chain", "peer_auto"):
+    if rehearse and default_sched(args, world) not in ("peer", "peer_chain", "peer_auto"):
         raise SystemExit("--rehearse-same-gpu needs --sched peer|peer_chain|peer_auto (NCCL refuses two ranks per GPU)")
     if rehearse:
         local_rank = 0
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
     comm = None
-
-    def max_over_ranks(x):
-        if world == 1:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device="cpu" if rehearse else dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
     if rehearse:
         dist.init_process_group("gloo")
     elif world > 1:
@@ -288,35 +590,115 @@ def main():
         dist.all_reduce(t)                       # create the NCCL communicator
         torch.cuda.synchronize()
         comm = nccl_comm_ptr()
-    name = args.config
-    cfg = workloads.config(name)
-    N, G = cfg["N"], world
-    mapping = workloads.mapping(N, G, args.mapping)
-    local = [k for k in range(N) if mapping[k] == rank]
-    buckets = cfg["buckets"]
-    B = len(buckets)
-    sched = {"auto": es.ES_SCHED_AUTO, "direct": es.ES_SCHED_DIRECT, "chain": es.ES_SCHED_CHAIN,
-             "peer": es.ES_SCHED_PEER, "peer_chain": es.ES_SCHED_PEER_CHAIN, "peer_auto": es.ES_SCHED_PEER_AUTO}[args.sched]
+
+    def reduce_over_ranks(x, op):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cpu" if rehearse else dev)
+        dist.all_reduce(t, op=op)
+        return float(t.item())
+
+    def max_over_ranks(x):
+        return reduce_over_ranks(x, dist.ReduceOp.MAX) if world > 1 else x
+
+    def gather_objects(obj):
+        if world == 1:
+            return [obj]
+        out = [None] * world
+        dist.all_gather_object(out, obj)
+        return out
+
+    # ---- preflight: device, peer access, NVLink links (every rank, recorded in the line) ----
+    props = torch.cuda.get_device_properties(dev)
+    nvl = NvLink(props.uuid)
+    peer_access = [bool(torch.cuda.can_device_access_peer(local_rank, j)) if j != local_rank else None
+                   for j in range(torch.cuda.device_count())]
+    pre = {"rank": rank, "device": local_rank, "name": props.name,
+           "pci_bus": f"{props.pci_domain_id:04x}:{props.pci_bus_id:02x}:{props.pci_device_id:02x}",
+           "nvlink_links_active": len(nvl.links) if nvl.ok else None, "peer_access": peer_access,
+           "nvml": nvl.why}
+    preflight = gather_objects(pre)
+
     snb = workloads.state_nbytes()
-    agg = Aggregator(N, G, rank, mapping, buckets, state_nbytes=snb,
-                     transport=es.ES_TRANSPORT_NONE if G == 1 or rehearse else es.ES_TRANSPORT_NCCL, comm=comm,
-                     sched=sched,
-                     device=dev, options=(es.ES_OPT_INCREMENTAL if args.incremental else 0) |
-                     (es.ES_OPT_STASH_BACKGROUND if args.stash_background else 0) |
-                     (es.ES_OPT_PEER_PUSH if args.peer_push else 0))
-    if G > 1 and sched in es.PEER_SCHEDS:
-        agg.peer_connect()                       # CUDA IPC map of every peer's workspace (NVLink)
-    live = [torch.zeros(n, dtype=torch.uint8, device=dev) for n in snb]
-    agg.register_state(live)
-    for k in local:
-        for i, blob in enumerate(workloads.est_state(name, k)):
-            agg.init_state(k, i, blob)
-    if args.inplace:       # the synthetic "backward" writes straight into the EST's slots
-        grads = {k: [workloads.est_bucket(name, k, b, device=dev, out=agg.slot(k, b)) for b in range(B)]
-                 for k in local}
-    else:
-        grads = {k: [workloads.est_bucket(name, k, b, device=dev) for b in range(B)] for k in local}
-    outs = [agg.new_out(b) for b in range(B)]
+    grads_host = {k: [host[(k, b)] for b in range(B)] for k in local}
+    opts_base = ((es.ES_OPT_INCREMENTAL if args.incremental else 0) |
+                 (es.ES_OPT_STASH_BACKGROUND if args.stash_background else 0) |
+                 (es.ES_OPT_PEER_PUSH if args.peer_push else 0))
+    sched_ids = {"auto": es.ES_SCHED_AUTO, "direct": es.ES_SCHED_DIRECT, "chain": es.ES_SCHED_CHAIN,
+                 "peer": es.ES_SCHED_PEER, "peer_chain": es.ES_SCHED_PEER_CHAIN, "peer_auto": es.ES_SCHED_PEER_AUTO}
+    fuse = not (args.per_bucket or args.no_fuse or args.incremental or args.inplace)
+
+    def build(sched_name, extra, attempt):
+        sched = sched_ids[sched_name]
+        options = opts_base | (es.ES_OPT_PEER_ROUNDS if extra == "rounds" else 0)
+        peer = G > 1 and sched in es.PEER_SCHEDS
+        agg = Aggregator(N, G, rank, mapping, buckets, state_nbytes=snb,
+                         transport=es.ES_TRANSPORT_NONE if G == 1 or peer else es.ES_TRANSPORT_NCCL,
+                         comm=comm, sched=sched, device=dev, options=options)
+        if peer:
+            fail = ""
+            try:
+                if attempt == 0 and args.simulate_peer_failure == "open" and rank == world - 1:
+                    raise PeerFailure("simulated: es_peer_open returned ES_EUNSUPPORTED (test hook)")
+                agg.peer_connect()               # CUDA IPC map of every peer's workspace (NVLink)
+            except (es.EsError, PeerFailure) as e:
+                fail = f"rank {rank}: {e}"
+            fails = [f for f in gather_objects(fail) if f]
+            if fails:
+                agg.close()
+                raise PeerFailure("; ".join(fails))
+        return agg, sched, options
+
+    attempts = []
+    agg = None
+    for attempt, (sched_name, extra) in enumerate(ladder(args, world, rehearse)):
+        try:
+            agg, sched, options = build(sched_name, extra, attempt)
+        except PeerFailure as e:
+            attempts.append({"sched": sched_name, "executor": extra or "default", "failed": str(e)})
+            continue
+        live = [torch.zeros(n, dtype=torch.uint8, device=dev) for n in snb]
+        agg.register_state(live)
+        for k in local:
+            for i, blob in enumerate(workloads.est_state(name, k)):
+                agg.init_state(k, i, blob)
+        if args.inplace:       # the synthetic "backward" writes straight into the EST's slots
+            grads = {k: [agg.slot(k, b).copy_(workloads.to_torch(grads_host[k][b])) for b in range(B)]
+                     for k in local}
+        else:
+            grads = {k: [workloads.to_torch(grads_host[k][b], dev) for b in range(B)] for k in local}
+        outs = [agg.new_out(b) for b in range(B)]
+        torch.cuda.synchronize()
+        if world > 1:
+            stream0 = torch.cuda.Stream(device=dev)
+            with torch.cuda.stream(stream0):     # first step, eager: the fallback decision's evidence
+                agg.switch(local[0])
+                for i, k in enumerate(local):
+                    agg.stash_many(k, range(B), grads[k], es.ES_STASH_BORROW if i == len(local) - 1
+                                   else es.ES_STASH_COPY)
+                agg.allreduce_many(range(B), outs)
+            torch.cuda.synchronize()
+            agg.sync()
+            bad = first_step_check(name, buckets, N, outs, host)
+            if attempt == 0 and args.simulate_peer_failure == "parity" and rank == 0:
+                bad += 1
+            bads = gather_objects(bad)
+            if any(bads):
+                attempts.append({"sched": sched_name, "executor": extra or "default",
+                                 "failed": f"first-step oracle check: {bads} mismatched words per rank"})
+                del grads, outs, live
+                agg.close()
+                agg = None
+                continue
+        attempts.append({"sched": sched_name, "executor": extra or "default", "ok": True})
+        break
+    if agg is None:
+        if rank == 0:
+            print(json.dumps({"metric": METRIC, "error": "every schedule rung failed", "attempts": attempts,
+                              "preflight": preflight}), flush=True)
+        raise SystemExit(2)
+    args.sched = sched_name                      # the schedule that runs (the line's config says it)
+
     esz = 2 if cfg["dtype"] == "bf16" else 4
     in_bytes = len(local) * sum(n for n, _ in buckets) * esz
     flush = None if in_bytes > 2 * L2_BYTES else torch.empty(4 * L2_BYTES, dtype=torch.uint8, device=dev)
@@ -324,8 +706,6 @@ def main():
         flush_words = flush.view(torch.int32)
         flush_sink = torch.zeros((), dtype=torch.int32, device=dev)
     torch.cuda.synchronize()
-
-    fuse = not (args.per_bucket or args.no_fuse or args.incremental or args.inplace)
 
     def step(marks=None):
         # marks: three external CUDA events recorded at the phase boundaries
@@ -392,9 +772,9 @@ def main():
     marks = [torch.cuda.Event(enable_timing=True, external=use_graph) for _ in range(3)]
     if use_graph:
         # Three captures of the same step: without timing events (the K steps
-        # we time), with phase-boundary events only (replayed once after the
-        # timed region: stash and allreduce phases with every overlap intact),
-        # and with per-kernel event nodes (replayed once after that: per-kind
+        # we time), with phase-boundary events only (replayed after the timed
+        # region: stash and allreduce phases with every overlap intact), and
+        # with per-kernel event nodes (replayed once after that: per-kind
         # durations).
         graph = torch.cuda.CUDAGraph()
         with torch.cuda.graph(graph, stream=stream):
@@ -431,6 +811,7 @@ def main():
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
+    nvl0 = nvl.read()
     t_start = time.time()
     with torch.cuda.stream(stream):
         for i in range(args.steps):
@@ -445,23 +826,41 @@ def main():
             ends[i].record(stream)
     torch.cuda.synchronize()
     t_end = time.time()
+    nvl1 = nvl.read()
+    phase_samples = []
     if graph is not None:
         # after (outside) the timed region, in the same steady state (queued back to back behind
-        # plain replays, no host sync in between): one replay with phase-boundary events, one with
-        # per-kernel event pairs, each prepared like a timed step
+        # plain replays, no host sync in between): 5 replays with phase-boundary events (each
+        # read before the next), then one with per-kernel event pairs
+        for _ in range(5):
+            with torch.cuda.stream(stream):
+                for g_ in (graph, graph, graph_phase):
+                    if flush is not None:
+                        flush.zero_()
+                        flush_sink.copy_(flush_words.amax())
+                    g_.replay()
+            torch.cuda.synchronize()
+            phase_samples.append((marks[0].elapsed_time(marks[1]), marks[1].elapsed_time(marks[2])))
         with torch.cuda.stream(stream):
-            for g_ in (graph, graph, graph_phase, graph, graph_prof):
+            for g_ in (graph, graph_prof):
                 if flush is not None:
                     flush.zero_()
                     flush_sink.copy_(flush_words.amax())
                 g_.replay()
         torch.cuda.synchronize()
+    elif args.steps >= 2:
+        phase_samples.append((marks[0].elapsed_time(marks[1]), marks[1].elapsed_time(marks[2])))
     if world > 1:
         dist.barrier()
     clk = clocks.stop(t_start, t_end)
     step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
     ms = sum(step_ms) / len(step_ms)
     ms = max_over_ranks(ms)
+    # phase times of this rank (median of the samples), then max over ranks
+    stash_ph = statistics.median(p[0] for p in phase_samples) if phase_samples else None
+    ar_ph = statistics.median(p[1] for p in phase_samples) if phase_samples else None
+    if world > 1 and ar_ph is not None:
+        stash_ph, ar_ph = max_over_ranks(stash_ph), max_over_ranks(ar_ph)
 
     kinds = {"stash": es.ES_KERNEL_STASH, "fold": es.ES_KERNEL_FOLD, "swap": es.ES_KERNEL_SWAP,
              "gather": es.ES_KERNEL_GATHER, "barrier": es.ES_KERNEL_BARRIER}
@@ -469,12 +868,9 @@ def main():
     agg.profile(False)
     steps_profiled = 1 if graph is not None else args.steps
     launches_per_step = sum(p[0] for p in prof.values()) / (1 if graph is not None else args.steps)
-    fl_n, fl_ms, fl_bytes = prof["fold"]
     payload = workloads.payload_bytes(name)
     value = payload / (ms / 1e3) / 1e9
     peak, peak_src = peaks()
-    # Roofline of every HBM kernel of the step; `roofline` is the dominant one
-    # (largest share of the profiled step's device time).
     traffic_all = {}
     tfile = os.path.join(ROOT, "profiles", f"traffic_{name}_g{G}.json")
     if os.path.exists(tfile) and not (args.incremental or args.per_bucket or args.no_fuse or args.no_graph
@@ -482,30 +878,52 @@ def main():
         with open(tfile) as f:
             traffic_all = json.load(f)
 
-    # Phase timing (fused G=1 step only, where the stash phase holds nothing but stash kernels with
-    # their fused switches and the allreduce phase nothing but the fold): events at the phase
-    # boundaries of one timed step, no event between kernels, so early start and PDL overlap stay
-    # intact.  The per-kernel event pairs of the profiled step add ~1-5 us per launch.
-    phase_ms = None
-    if fuse and G == 1 and (graph is not None or args.steps >= 2):
-        phase_ms = {"stash": marks[0].elapsed_time(marks[1]), "fold": marks[1].elapsed_time(marks[2])}
+    # The plan this rank runs (schedules per bucket) and its per-rank byte model.
+    costs, scheds = (None, None)
+    if G > 1:
+        costs, scheds = plan_costs(buckets, N, G, mapping, sched, options)
+    sched_name_of = {0: "single", es.ES_SCHED_DIRECT: "direct", es.ES_SCHED_CHAIN: "chain",
+                     es.ES_SCHED_PEER: "peer", es.ES_SCHED_PEER_CHAIN: "peer_chain"}
+
+    # Phase timing: events only at the phase boundaries of one step (no event between kernels,
+    # so early start / PDL overlap stay intact).  The stash phase holds the stash kernels (with
+    # their fused switches) of the fused step; the allreduce phase everything es_allreduce_many
+    # launches (G == 1: the fold; G > 1: barrier, folds, gathers).  Per-kernel event pairs of the
+    # profiled step add ~1-5 us per launch and serialise the overlap.
+    phase_ms = {}
+    if stash_ph is not None and fuse:
+        phase_ms["stash"] = stash_ph
+    if ar_ph is not None and G == 1 and not args.incremental:
+        phase_ms["fold"] = ar_ph
 
     def roof(kind, kname):
         n_, ms_, bytes_ = prof[kind]
         if n_ == 0 or ms_ <= 0:
             return None
         ev_us = ms_ / n_ * 1e3                                       # per-kernel event pairs
-        if phase_ms is not None and kind in phase_ms:
+        if kind in phase_ms:
             us, how = phase_ms[kind] * 1e3 / (n_ / steps_profiled), "phase events (no event between launches)"
         else:
             us, how = ev_us, "per-launch event pairs"
-        a = bytes_ / n_ / (us / 1e6) / 1e9
-        return {"bound": "hbm", "kernel": kname, "achieved": round(a, 1), "peak": peak, "unit": "GB/s",
-                "frac": round(a / peak, 4), "traffic": traffic_all.get(f"{kname}_dram_bytes_per_launch"),
-                "algorithmic_bytes_per_launch": int(bytes_ / n_), "launches_per_step": int(n_ / steps_profiled),
-                "avg_launch_us": round(us, 2), "timing": how, "avg_launch_us_event_pairs": round(ev_us, 2),
-                "share_of_step": round(us * n_ / steps_profiled / 1e3 / ms, 3), "peak_source": peak_src,
-                "frac_of_nominal": round(a / HBM_NOMINAL_GBPS, 4)}
+        bound, bpl, pk = "hbm", bytes_ / n_, peak
+        if costs is not None and kind in ("fold", "gather"):
+            # G > 1: the kernel reads peer memory over NVLink (PEER*) -- its bound is the slower of
+            # its HBM and NVLink bytes; achieved is measured against that resource
+            hb, nv = costs[rank]["kinds"].get(kind, [0, 0])
+            per = n_ / steps_profiled
+            if nv / NVL_MEASURED_GBPS > hb / peak:
+                bound, bpl, pk = "nvlink", nv / per, NVL_MEASURED_GBPS
+            else:
+                bpl = hb / per
+        a = bpl / (us / 1e6) / 1e9
+        r = {"bound": bound, "kernel": kname, "achieved": round(a, 1), "peak": pk, "unit": "GB/s",
+             "frac": round(a / pk, 4), "traffic": traffic_all.get(f"{kname}_dram_bytes_per_launch"),
+             "algorithmic_bytes_per_launch": int(bpl), "launches_per_step": int(n_ / steps_profiled),
+             "avg_launch_us": round(us, 2), "timing": how, "avg_launch_us_event_pairs": round(ev_us, 2),
+             "share_of_step": round(us * n_ / steps_profiled / 1e3 / ms, 3),
+             "peak_source": peak_src if bound == "hbm" else "B200_PROFILING.md measured peer copy per direction",
+             "frac_of_nominal": round(a / (HBM_NOMINAL_GBPS if bound == "hbm" else NVL_NOMINAL_GBPS), 4)}
+        return r
 
     roofs = {k: r for k, r in (("k_fold", roof("fold", "k_fold")), ("k_stash", roof("stash", "k_stash")),
                                ("k_gather", roof("gather", "k_gather"))) if r is not None}
@@ -526,6 +944,9 @@ def main():
                    "l2": ("inputs larger than L2 (%.1f MB of EST gradients per GPU per step)" % (in_bytes / 1e6))
                    if flush is None else "L2 flushed between timed steps (512 MB write, then read back: "
                                                   "no flush lines left dirty to drain inside the timed step)"},
+        "inputs": {"generator": "NumPy Philox per (config, EST, bucket, 2^20-element block), drawn on the host "
+                                "(workloads.host_inputs) and copied to HBM before timing",
+                   "host_seconds": round(t_gen, 2)},
         "roofline": dominant,
         "roofline_by_kernel": roofs,
         # the whole step against the same peak: every kernel's algorithmic bytes of one step divided by
@@ -535,18 +956,51 @@ def main():
                           "frac": round(sum(v[2] for v in prof.values()) / steps_profiled / (ms / 1e3) / 1e9 / peak, 4),
                           "bytes_per_step": int(sum(v[2] for v in prof.values()) / steps_profiled),
                           "frac_of_nominal": round(sum(v[2] for v in prof.values()) / steps_profiled / (ms / 1e3) / 1e9
-                                                   / HBM_NOMINAL_GBPS, 4)},
+                                                   / HBM_NOMINAL_GBPS, 4),
+                          "note": "all kernels' algorithmic bytes (HBM and, at G > 1, NVLink) of this rank's step"},
         "breakdown_ms_per_step": {k: round(v[1] / steps_profiled, 4) for k, v in prof.items()},
         "per_kernel": {k: {"launches_per_step": int(v[0] / steps_profiled),
                            "algorithmic_GBps": round(v[2] / (v[1] / 1e3) / 1e9, 1) if v[1] > 0 else None,
                            "us_per_launch": round(v[1] / max(v[0], 1) * 1e3, 2)} for k, v in prof.items()},
-        # SURVEY 8(d)'s narrower metric: es_allreduce time only (stashes already done)
-        "allreduce_only": {"ms": round(fl_ms / steps_profiled, 4),
-                           "GBps": round(payload / (fl_ms / steps_profiled / 1e3) / 1e9, 1) if fl_ms > 0 else None},
         "gpu_launches": int(round(launches_per_step * args.steps)),
         "step_ms_p10_p50_p90": [round(float(np.percentile(step_ms, q)), 4) for q in (10, 50, 90)],
         "clocks": clk,
     }
+    # SURVEY 8(d)'s narrower metric: es_allreduce time only (stashes already done) -- exchange +
+    # fold + scale + gather, from phase events (stash-done -> allreduce-done), max over ranks
+    if ar_ph is not None:
+        ar = {"ms": round(ar_ph, 4), "GBps": round(payload / (ar_ph / 1e3) / 1e9, 1),
+              "timing": f"phase events, median of {len(phase_samples)} replays, max over ranks",
+              "stash_phase_ms": round(stash_ph, 4) if stash_ph is not None else None}
+        if costs is not None:
+            ar["roofline"] = plan_roofline(costs, ar_ph, peak)
+        elif not args.incremental:
+            fold_bytes = (N + 1) * sum(n for n, _ in buckets) * esz          # (N+1) L b: SURVEY 8(d), G = 1
+            a = fold_bytes / (ar_ph / 1e3) / 1e9
+            ar["roofline"] = {"bound": "hbm", "achieved": round(a, 1), "peak": peak, "unit": "GB/s",
+                              "frac": round(a / peak, 4), "bytes": fold_bytes,
+                              "t_roof_ms": round(fold_bytes / (peak * 1e9) * 1e3, 4),
+                              "frac_of_nominal": round(a / HBM_NOMINAL_GBPS, 4)}
+        line["allreduce_only"] = ar
+    if G > 1:
+        line["schedule"] = {"ladder": attempts,
+                            "per_bucket": [sched_name_of.get(s, str(s)) for s in scheds],
+                            "peer_chain_executor": ("rounds (ES_OPT_PEER_ROUNDS)" if options & es.ES_OPT_PEER_ROUNDS
+                                                    else "tile-pipelined (k_fold_pipe)"),
+                            "transport": "CUDA IPC peer memory" if sched in es.PEER_SCHEDS else "NCCL P2P"}
+        line["preflight"] = preflight
+        # NVLink bytes this rank's links carried over the K timed steps (NVML data counters)
+        if nvl0 is not None and nvl1 is not None:
+            mine = {"tx_bytes_per_step": (nvl1[0] - nvl0[0]) / args.steps, "rx_bytes_per_step":
+                    (nvl1[1] - nvl0[1]) / args.steps}
+        else:
+            mine = {"unavailable": nvl.why or "no active NVLink"}
+        per_rank = gather_objects(mine)
+        plan_nv = [{"in_bytes": c["nvl_in"], "out_bytes": c["nvl_out"]} for c in costs]
+        line["nvlink_counters"] = {"per_rank": per_rank, "plan_per_rank": plan_nv,
+                                   "source": "NVML NVLINK_THROUGHPUT_DATA_TX/RX (KiB, payload), active links",
+                                   **({"note": "rehearsal: every rank on one GPU, peer traffic stays in HBM"}
+                                      if rehearse else {})}
 
     # ---- context-switch latency (reported separately) ----
     if len(local) > 1:
@@ -575,62 +1029,55 @@ def main():
                           "timed": f"{10 * n_sw} back-to-back es_switch_context in a CUDA graph",
                           "share_of_step": round(us * len(local) / 1e3 / ms, 4)}
 
-    # ---- parity of the timed outputs against the oracle on sampled windows (+ cpu_baseline) ----
-    if rank == 0:
-        import oracle  # test infrastructure: the cpu_baseline leg and parity check only
-        gen_cache = {}
+    # ---- NEXT-3 (iii): ncclAllReduce (Ring, Simple, one channel) vs the canonical order --------
+    line["ring_crosscheck"] = ring_crosscheck(args, name, N, G, rank, rehearse, dev, host)
 
-        def fetch(k, b, s, n):
-            if k in grads:
-                t = grads[k][b][s:s + n]
-            else:                                   # remote EST: regenerate its seeded input
-                if (k, b) not in gen_cache:
-                    gen_cache[(k, b)] = workloads.est_bucket(name, k, b, device=dev)
-                t = gen_cache[(k, b)][s:s + n]
-            t = t.cpu()
-            return t.numpy() if t.dtype == torch.float32 else t.view(torch.int16).numpy().view(np.uint16)
+    # ---- parity of the timed outputs against the oracle (+ cpu_baseline) ----
+    if rank == 0:
+        import oracle  # test infrastructure: the parity and cpu_baseline legs only
+
+        def fetch_all(b, s, n):
+            miss = [k for k in range(N) if (k, b) not in host]       # remote ESTs: their seeded streams
+            drawn = dict(zip(miss, workloads.window_np(name, b, miss, s, s + n))) if miss else {}
+            return [host[(k, b)][s:s + n] if (k, b) in host else drawn[k] for k in range(N)]
 
         budget = args.cpu_seconds if (world == 1 and not args.no_cpu) else 1.0
-        gbs, sample, windows = oracle_windows(name, fetch, budget)
-        mism = 0
-        checked = 0
+        gbs, sample, windows = oracle_windows(name, fetch_all, budget)
+        outs_np = []
+        for o in outs:
+            t = o.cpu()
+            outs_np.append(t.numpy() if t.dtype == torch.float32 else t.view(torch.int16).numpy().view(np.uint16))
+        mism, checked = 0, 0
         for b, s, n, want in windows:
-            got = outs[b][s:s + n].cpu()
-            got = got.numpy() if got.dtype == torch.float32 else got.view(torch.int16).numpy().view(np.uint16)
             w = want.view(np.uint32 if want.dtype == np.float32 else np.uint16)
-            g_ = got.view(w.dtype)
-            mism += int((w != g_).sum())
+            mism += int((w != outs_np[b][s:s + n].view(w.dtype)).sum())
             checked += n
         line["parity"] = {"checked_elements": checked, "mismatched_words": mism, "vs": "CPU oracle, bit-exact"}
         # SURVEY 8(d) bit-exact flag: SHA-256 of the whole reduced bucket set (bucket order, raw
         # words).  Equal across G and mappings (D1); the scaling run's lines can be compared.
         h = hashlib.sha256()
-        for o in outs:
-            h.update(o.view(torch.uint8).cpu().numpy().tobytes())
+        for o in outs_np:
+            h.update(o.tobytes())
         line["output_sha256"] = h.hexdigest()
-        if payload <= 3e9:
-            # the whole output against the oracle (seconds of single-thread C for these sizes)
-            ho, mism_all = hashlib.sha256(), 0
-            for b, (L_b, d_b) in enumerate(buckets):
-                want = oracle.reduce([fetch(k, b, 0, L_b) for k in range(N)], d_b)
-                ho.update(want.tobytes())
-                got = outs[b].view(torch.uint8).cpu().numpy()
-                mism_all += int((got.view(want.dtype) != want).sum()) if want.dtype != np.float32 else \
-                    int((got.view(np.uint32) != want.view(np.uint32)).sum())
+        if not args.no_full_parity:
+            # the WHOLE output against the oracle, every bucket, on every host core
+            mism_all, osha, secs = oracle_full(buckets, host, N, outs_np, cores_used())
             line["parity"].update({"full_output_checked": True, "full_output_mismatched_words": mism_all,
-                                   "oracle_sha256": ho.hexdigest(),
-                                   "sha256_equal": ho.hexdigest() == line["output_sha256"]})
+                                   "full_output_elements": sum(n for n, _ in buckets),
+                                   "oracle_sha256": osha, "sha256_equal": osha == line["output_sha256"],
+                                   "oracle_threads": cores_used(), "oracle_seconds": round(secs, 2)})
         if world == 1 and not args.no_cpu:
             line["cpu_baseline"] = {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-                                    "sample": sample, "host_cores_available": cores_used()}
+                                    "sample": sample, "host_cores_available": cores_used(),
+                                    "cpu_model": cpu_model()}
             # the oracle also on all host cores (same code, one window per thread)
-            gbs_mc, sample_mc = oracle_all_cores(name, fetch, cores_used())
+            gbs_mc, sample_mc = oracle_all_cores(name, fetch_all, cores_used())
             line["cpu_baseline_all_cores"] = {"value": round(gbs_mc, 4), "unit": "GB/s", "cores": cores_used(),
-                                              "kind": "oracle", "sample": sample_mc}
+                                              "kind": "oracle", "sample": sample_mc, "cpu_model": cpu_model()}
 
     # ---- e2e: public API with host buffers (pinned H2D in, D2H out, inside the timed region) ----
     if not args.no_e2e:
-        host = {k: [g.cpu().pin_memory() for g in grads[k]] for k in local}
+        hostp = {k: [workloads.to_torch(grads_host[k][b]).pin_memory() for b in range(B)] for k in local}
         # two live-gradient buffers: EST i+1's H2D (copy stream) overlaps EST i's stash (compute stream)
         live_grad = [[torch.empty_like(grads[local[0]][b]) for b in range(B)] for _ in range(2)]
         host_out = [torch.empty(o.shape, dtype=o.dtype).pin_memory() for o in outs]
@@ -657,7 +1104,7 @@ def main():
                 h2d_stream.wait_event(free[j])
                 with torch.cuda.stream(h2d_stream):
                     for b in range(B):                 # "backward" lands in a live buffer
-                        live_grad[j][b].copy_(host[k][b], non_blocking=True)
+                        live_grad[j][b].copy_(hostp[k][b], non_blocking=True)
                 landed[j].record(h2d_stream)
                 stream.wait_event(landed[j])
                 if i == 0:
@@ -698,7 +1145,7 @@ def main():
         # The e2e ceiling: the step's H2D bytes over this host link, the link's rate measured as plain
         # pinned H2D copies of the step's input tensors, repeated to >= 256 MB so small steps are not
         # latency-bound (the D2H runs in the other direction, overlapped).
-        flat = [t for k in local for t in host[k]]
+        flat = [t for k in local for t in hostp[k]]
         dst = [torch.empty_like(live_grad[0][b]) for b in range(B)]
         rounds = max(1, -(-(256 << 20) // h2d))
         h2d_ms = float("inf")
@@ -726,6 +1173,64 @@ def main():
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
+
+
+def ring_crosscheck(args, name, N, G, rank, rehearse, dev, host):
+    """NEXT-3 (iii): with N == G (one EST per GPU) run ncclAllReduce(sum) with
+    NCCL_ALGO=Ring, NCCL_PROTO=Simple on a one-channel communicator (min/max CTAs = 1) over a
+    buffer whose per-rank ring chunk equals R1's chunk (L_x = N * 65536 fp32: C = L_x / N, one
+    NCCL loop), then compare its words, times fl32(1/N) (a power of two here: exact), with the
+    oracle's canonical fold of the same inputs.  Agreement 1.0 pins reading R2 to NCCL's ring;
+    anything less says the readings differ from NCCL's order.  Outside the timed region."""
+    if args.no_ring_check:
+        return {"skipped": "--no-ring-check"}
+    if N != G:
+        return {"skipped": f"needs N == G (here N={N}, G={G})"}
+    if rehearse:
+        return {"skipped": "rehearsal: NCCL refuses two ranks on one GPU"}
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_lixyszrljlllq23_b200 import workloads
+    cfg = workloads.config(name)
+    b = max(range(len(cfg["buckets"])), key=lambda i: cfg["buckets"][i][0] if cfg["buckets"][i][1] == "f32" else -1)
+    L_b, d = cfg["buckets"][b]
+    if d != "f32" or (N & (N - 1)):
+        return {"skipped": "needs an fp32 bucket and a power-of-two N (exact 1/N scale on both sides)"}
+    per = 65536
+    Lx = min(N * per, (L_b // (N * 16)) * N * 16)
+    saved = {k: os.environ.get(k) for k in ("NCCL_ALGO", "NCCL_PROTO")}
+    os.environ["NCCL_ALGO"], os.environ["NCCL_PROTO"] = "Ring", "Simple"
+    try:
+        opts = dist.ProcessGroupNCCL.Options()
+        opts.config.min_ctas = 1
+        opts.config.max_ctas = 1
+        pg = dist.new_group(list(range(G)), backend="nccl", pg_options=opts)
+        x = workloads.to_torch(workloads.est_bucket_np(name, rank, b, 0, Lx), dev)
+        dist.all_reduce(x, group=pg)
+        torch.cuda.synchronize()
+        got = (x * (1.0 / N)).cpu().numpy()
+        dist.destroy_process_group(pg)
+    except Exception as e:
+        return {"error": f"{type(e).__name__}: {e}"}
+    finally:
+        for k, v in saved.items():
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
+    if rank != 0:
+        return None
+    import oracle
+    miss = [k for k in range(N) if (k, b) not in host]
+    drawn = dict(zip(miss, workloads.window_np(name, b, miss, 0, Lx))) if miss else {}
+    xs = [host[(k, b)][:Lx] if (k, b) in host else drawn[k] for k in range(N)]
+    want = oracle.reduce(xs, "f32", L=Lx)
+    eq = int((want.view(np.uint32) == got.view(np.uint32)).sum())
+    return {"bucket": b, "elements": Lx, "ring_chunk_elements": Lx // N, "words_equal": eq, "frac_equal": eq / Lx,
+            "nccl": "ncclAllReduce sum, NCCL_ALGO=Ring NCCL_PROTO=Simple, min/max CTAs 1, times fl32(1/N)",
+            "nccl_sha256": hashlib.sha256(got.tobytes()).hexdigest(),
+            "oracle_sha256": hashlib.sha256(want.tobytes()).hexdigest()}
 
 
 if __name__ == "__main__":
