@@ -162,7 +162,7 @@ typedef struct {
 } es_config;
 
 /* ES_OPT_INCREMENTAL: reserve fp32 partials so that es_stash_fold_grads can
- * fold each EST into the running partials at its switch (NEXT-1, G == 1). */
+ * fold each EST into the running partials at its switch (NEXT-1, any G). */
 #define ES_OPT_INCREMENTAL 1u
 /* ES_OPT_PEER_ROUNDS: PEER_CHAIN without tile pipelining (a device barrier
  * between rounds).  Same bits; kept for comparison and as a fallback. */
@@ -284,22 +284,28 @@ es_status es_stash_and_switch(es_handle h, int32_t est, int32_t n, const int32_t
                               const es_dtype *grad_dtypes, es_stash_mode mode, int32_t next_est, es_stream stream);
 
 /* NEXT-1 incremental canonical fold (PAPER.md:599-606 overlaps
- * the gradient swap with the next EST's compute): at EST `est`'s switch,
- * fold its contribution straight into the running unrounded fp32 partials of
- * the chunks c < est -- for them `est` comes after c+1..est-1 in canonical
- * order (R2), and ESTs run in index order -- and stash only chunks >= est,
- * which wait for the wrap.  The last EST (N-1) folds nothing at its call
- * (COPY stashes the whole bucket, BORROW keeps the buffer): es_allreduce of
- * the bucket folds, per chunk c, the partial (ESTs c+1..N-2), EST N-1 and
- * the stashed 0..c, so the end-of-step critical path reads the partial plus
- * c+2 contributions per element -- ~(N+3)/2 on average -- instead of N,
- * with the same bits (segmentability, R14).  Total bytes grow by the
- * partials' round trips, which the paper's overlap hides.
- * Requirements: G == 1, cfg.options has ES_OPT_INCREMENTAL, every EST of the
- * step calls this for the bucket in order 0, 1, ..., N-1 (ES_ESTATE
+ * the gradient swap with the next EST's compute).  Every fold this rank runs
+ * whose canonical sequence (R2: c+1, c+2, ... for chunk c) STARTS here -- at
+ * G == 1 every chunk's whole sequence, for DIRECT / PEER the own shard's
+ * chunks with EST c+1 local, for CHAIN / PEER_CHAIN a chain's first segment --
+ * has a prefix of local ESTs c+1, c+2, ... (ascending, up to the wrap
+ * N-1 -> 0, never the rank's last local EST, leaving the segment at least one
+ * EST).  At the stash of a prefix EST its contribution is folded straight into
+ * the running unrounded fp32 partial of that chunk (the first prefix EST opens
+ * it); everything else of its gradient -- ranges peers or the exchange read,
+ * chunks after the wrap -- is copied to the slot (COPY) or kept (BORROW).
+ * es_allreduce then continues each such fold from its partial over the
+ * remaining ESTs, so the end-of-step critical path reads fewer contributions
+ * (G == 1: ~(N+3)/2 instead of N per element), with the same bits
+ * (segmentability, R14).  Total bytes grow by the partials' round trips,
+ * which the paper's overlap hides.
+ * Requirements: cfg.options has ES_OPT_INCREMENTAL; every local EST of the
+ * step calls this for the bucket, in ascending EST order (ES_ESTATE
  * otherwise; mixing with es_stash_grad for the same bucket and step is an
- * ES_ESTATE error).  mode: COPY (the stashed part is copied) or BORROW (the
- * buffer is kept until es_allreduce completes). */
+ * ES_ESTATE error).  mode: COPY (the unfolded part is copied) or BORROW (the
+ * buffer is kept until es_allreduce completes).  A COPY-stashed EST whose
+ * contribution was partly folded cannot be exported (es_export_context:
+ * ES_ESTATE). */
 es_status es_stash_fold_grads(es_handle h, int32_t est, int32_t n, const int32_t *buckets, const void *const *grads,
                               const es_dtype *grad_dtypes, es_stash_mode mode, es_stream stream);
 
@@ -423,6 +429,15 @@ enum {
 /* All [lo, hi) ranges are in bucket element coordinates. */
 es_status es_plan_ops(const es_config *cfg, int32_t bucket, int64_t *ops, size_t cap_ops,
                       size_t *n_ops, int32_t *sched_out);
+
+/* Host-only, like es_plan_ops: the NEXT-1 incremental prefixes of cfg->rank
+ * for `bucket` (cfg->options must hold ES_OPT_INCREMENTAL, else *n_rows = 0).
+ * Row i = rows[5i .. 5i+4] = {c, first, q, lo, hi}: at their stashes ESTs
+ * first, first+1, ..., first+q-1 (first = (c+1) mod N) are folded into the
+ * fp32 partial of bucket elements [lo, hi) of chunk c; es_allreduce
+ * continues from it (see es_stash_fold_grads).  Rows ascend in c.  Same
+ * two-call protocol as es_plan_ops (rows NULL: count only). */
+es_status es_plan_incremental(const es_config *cfg, int32_t bucket, int64_t *rows, size_t cap_rows, size_t *n_rows);
 
 /* ---- loopback transport (testing; see es_transport) ---------------------- */
 

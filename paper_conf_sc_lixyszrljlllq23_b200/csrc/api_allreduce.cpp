@@ -12,6 +12,43 @@ extern "C" {
 namespace {
 es_status finish_allreduce(es_handle h, int32_t n, const int32_t *buckets, cudaStream_t cs, unsigned long long cap);
 
+// NEXT-1 end of step.  A planned fold over [lo, hi) that starts its sequence
+// fresh -- rot (every chunk's whole canonical sequence: G == 1, DIRECT, PEER)
+// or a chain's first segment (ESTs e0, e0+1, ..., m of them) -- is cut into
+// per-chunk pieces; where plan_incremental folded the first q ESTs of chunk c
+// into the fp32 partial at their stashes, the piece continues from that
+// partial over the remaining ESTs of the sequence (segmentability, R14).
+// Chunks without a partial stay rot pieces (merged when adjacent).
+struct Piece {
+  int64_t lo, hi;
+  bool rot;
+  int32_t e0, m;
+  bool part;
+};
+void inc_pieces(const es::Plan &p, const es::BucketPlan &b, bool inc, int64_t lo, int64_t hi, int64_t e0, int32_t m,
+                std::vector<Piece> *out) {
+  out->clear();
+  if (!inc) {
+    out->push_back({lo, hi, e0 < 0, (int32_t)e0, m, false});
+    return;
+  }
+  const int64_t C = (int64_t)b.C;
+  for (int64_t a = lo; a < hi;) {
+    const int32_t c = (int32_t)(a / C);
+    const int64_t z = std::min<int64_t>(hi, (int64_t)(c + 1) * C);
+    const int32_t q = b.inc_q[c];
+    if (q == 0) {
+      if (e0 < 0 && !out->empty() && out->back().rot && out->back().hi == a) out->back().hi = z;
+      else out->push_back({a, z, e0 < 0, (int32_t)e0, m, false});
+    } else if (e0 < 0) {
+      out->push_back({a, z, false, (int32_t)(((int64_t)c + 1 + q) % p.N), p.N - q, true});
+    } else {
+      out->push_back({a, z, false, (int32_t)((e0 + q) % p.N), m - q, true});
+    }
+    a = z;
+  }
+}
+
 es_status peer_barrier(es_handle h, cudaStream_t cs) {
   const es::Plan &p = h->plan;
   std::vector<uint64_t *> pf(p.G);
@@ -32,6 +69,7 @@ es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *c
   if (!h->peer_open) return set_err(ES_ESTATE, "peer-memory schedules need es_peer_open before es_allreduce");
   const bool pipe = !(p.options & ES_OPT_PEER_ROUNDS) && p.compat == 0;
   es_status s;
+  auto inc_done = [&](int32_t bk) { return (p.options & ES_OPT_INCREMENTAL) && h->inc_next[bk] == h->n_local; };
   auto slot_of = [&](int32_t rank, int32_t e, int32_t b) {
     return h->peer_ws[rank] + p.grad_off + (uint64_t)p.owner_index[e] * p.slot_block + p.slot_off[b];
   };
@@ -115,10 +153,13 @@ es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *c
             gbytes += 2 * (uint64_t)(hi - lo) * esz;
             continue;
           }
-          // ES_OP_FOLD
+          // ES_OP_FOLD (NEXT-1: pieces continuing from the incremental partials)
+          std::vector<Piece> pcs;
+          inc_pieces(p, b, inc_done(bk) && f[5] == ES_BUF_NONE, lo, hi, f[3], (int32_t)f[4], &pcs);
+          for (const Piece &pc : pcs) {
           es::FoldSegDesc d;
-          d.lo = lo;
-          d.n = hi - lo;
+          d.lo = pc.lo;
+          d.n = pc.hi - pc.lo;
           d.C = (uint32_t)b.C;
           std::vector<const void *> src;
           auto contrib = [&](int32_t e) -> const unsigned char * {
@@ -126,26 +167,28 @@ es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *c
             const void *bw = li >= 0 ? h->borrowed[(size_t)li * h->B + bk] : nullptr;
             const unsigned char *base = bw ? reinterpret_cast<const unsigned char *>(bw)
                                            : slot_of(p.est_to_gpu[e], e, bk);   // local or peer slot
-            return base + (uint64_t)lo * esz;
+            return base + (uint64_t)pc.lo * esz;
           };
-          if (f[3] < 0) {
+          if (pc.rot) {
             d.rot = true;
             for (int32_t e = 0; e < p.N; ++e) src.push_back(contrib(e));
           } else {
             d.rot = false;
-            d.m = (int32_t)f[4];
-            for (int32_t t = 0; t < d.m; ++t) src.push_back(contrib((int32_t)((f[3] + t) % p.N)));
+            d.m = pc.m;
+            for (int32_t t = 0; t < d.m; ++t) src.push_back(contrib((int32_t)((pc.e0 + t) % p.N)));
           }
           if (f[5] == ES_BUF_PEER_PART)         // the previous GPU's partial, over NVLink
             d.part_in = reinterpret_cast<const float *>(h->peer_ws[f[6]] + p.peer_parts_off + b.peer_part_base +
                                                         (uint64_t)f[9]);
+          else if (pc.part)                     // NEXT-1: this rank's incremental partial
+            d.part_in = reinterpret_cast<const float *>(h->ws + p.inc_off + p.inc_bucket_off[bk]) + pc.lo;
           d.out_partial = f[7] == ES_BUF_PART;
           d.out = d.out_partial ? (void *)(h->ws + p.peer_parts_off + b.peer_part_base + (uint64_t)f[8])
-                                : (void *)(h->ws + p.result_off + p.slot_off[bk] + (uint64_t)lo * esz);
+                                : (void *)(h->ws + p.result_off + p.slot_off[bk] + (uint64_t)pc.lo * esz);
           if (!d.out_partial && pushes(b)) {
             std::vector<void *> dst;
             for (int32_t g = 0; g < p.G; ++g)
-              if (g != p.rank) dst.push_back(h->peer_ws[g] + p.result_off + p.slot_off[bk] + (uint64_t)lo * esz);
+              if (g != p.rank) dst.push_back(h->peer_ws[g] + p.result_off + p.slot_off[bk] + (uint64_t)pc.lo * esz);
             push_ptrs.push_back(std::move(dst));
             d.push = push_ptrs.back().data();
             d.npush = (int32_t)push_ptrs.back().size();
@@ -157,20 +200,21 @@ es_status peer_allreduce(es_handle h, int32_t n, const int32_t *buckets, void *c
           srcs.push_back(std::move(src));
           if (pipe && b.sched == ES_SCHED_PEER_CHAIN) {
             const int32_t rd = k - 1;                     // round of this segment
-            const uint64_t c = (uint64_t)lo / b.C;        // its chunk (segments span whole chunks)
+            const uint64_t c = (uint64_t)pc.lo / b.C;     // its chunk (segments span whole chunks)
             auto flag = [&](unsigned char *base, int32_t round) {
               return reinterpret_cast<uint64_t *>(base + p.pipe_flags_off) + b.pipe_flag_base +
                      (c * (uint64_t)b.chain_rounds + (uint64_t)round) * b.tiles_per_chunk;
             };
             es::PipeSegDesc q;
             q.f = d;
-            q.wait = d.part_in ? flag(h->peer_ws[f[6]], rd - 1) : nullptr;
+            q.wait = f[5] == ES_BUF_PEER_PART ? flag(h->peer_ws[f[6]], rd - 1) : nullptr;
             q.pub = d.out_partial ? flag(h->ws, rd) : nullptr;
             pipes.push_back({rd, q});
             pbytes += nbytes;
           } else {
             folds.push_back(d);
             fbytes += nbytes;
+          }
           }
         }
       }
@@ -233,7 +277,7 @@ es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void
     for (int32_t li = 0; li < h->n_local; ++li)
       if (!h->stashed[(size_t)li * h->B + buckets[i]])
         return set_err(ES_ESTATE, "es_allreduce before every local EST stashed this bucket");
-    if (h->inc_next[buckets[i]] != 0 && h->inc_next[buckets[i]] != p.N)
+    if (h->inc_next[buckets[i]] != 0 && h->inc_next[buckets[i]] != h->n_local)
       return set_err(ES_ESTATE, "incremental fold of this bucket is incomplete");
   }
   cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
@@ -293,62 +337,39 @@ es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void
       return h->ws + p.parts_off + pt.off + (uint64_t)(lo - pt.lo) * 4;
     };
     unsigned char *outp = reinterpret_cast<unsigned char *>(outs[i]);
-    if (h->inc_next[bucket] == p.N && b.L > 0) {
-      // NEXT-1 end of step (the last EST's fold was deferred to here): chunk
-      // c < N-2 continues from its partial (ESTs c+1..N-2) over EST N-1 and
-      // the stashed ESTs 0..c; chunk N-2 folds N-1, 0..N-2 (EST N-1 is its
-      // first); chunk N-1 folds 0..N-1.
-      if (!pend.empty() && pend_dt != b.dtype && (s = flush()) != ES_OK) return s;
-      pend_dt = b.dtype;
-      const float *part = reinterpret_cast<const float *>(h->ws + p.inc_off + p.inc_bucket_off[bucket]);
-      for (int32_t c = 0; c < p.N; ++c) {
-        const int64_t lo = std::min<int64_t>((int64_t)b.L, (int64_t)c * (int64_t)b.C);
-        const int64_t hi = std::min<int64_t>((int64_t)b.L, (int64_t)(c + 1) * (int64_t)b.C);
-        if (hi <= lo) continue;
-        es::FoldSegDesc d;
-        d.lo = lo;
-        d.n = hi - lo;
-        d.C = (uint32_t)b.C;
-        d.rot = false;
-        const bool cont = c < p.N - 2;
-        std::vector<const void *> src;
-        if (c < p.N - 1) src.push_back(src_base(p.N - 1) + (uint64_t)lo * esz);
-        for (int32_t e = 0; e <= (c < p.N - 1 ? c : p.N - 1); ++e) src.push_back(src_base(e) + (uint64_t)lo * esz);
-        d.m = (int32_t)src.size();
-        d.part_in = cont ? part + lo : nullptr;
-        d.out = outp + (uint64_t)lo * esz;
-        pend_bytes += (uint64_t)d.n * ((uint64_t)d.m * esz + (cont ? 4 : 0) + esz);
-        pend.push_back(d);
-        pend_src.push_back(std::move(src));
-      }
-      continue;
-    }
+    const bool inc = (p.options & ES_OPT_INCREMENTAL) && h->inc_next[bucket] == h->n_local;
     for (const es::Op &op : b.ops) {
       const int64_t *f = op.f;
       switch (f[0]) {
         case ES_OP_FOLD: {
           if (!pend.empty() && pend_dt != b.dtype && (s = flush()) != ES_OK) return s;
           pend_dt = b.dtype;
-          const int64_t lo = f[1], hi = f[2];
-          es::FoldSegDesc d;
-          d.lo = lo;
-          d.n = hi - lo;
-          d.C = (uint32_t)b.C;
-          std::vector<const void *> src;
-          if (f[3] < 0) {
-            d.rot = true;
-            for (int32_t e = 0; e < p.N; ++e) src.push_back(contrib_at(e, lo));
-          } else {
-            d.rot = false;
-            d.m = (int32_t)f[4];
-            for (int32_t t = 0; t < d.m; ++t) src.push_back(contrib_at((int32_t)((f[3] + t) % p.N), lo));
+          std::vector<Piece> pcs;   // NEXT-1: pieces continuing from the incremental partials
+          inc_pieces(p, b, inc && f[5] == ES_BUF_NONE, f[1], f[2], f[3], (int32_t)f[4], &pcs);
+          for (const Piece &pc : pcs) {
+            const int64_t lo = pc.lo;
+            es::FoldSegDesc d;
+            d.lo = lo;
+            d.n = pc.hi - lo;
+            d.C = (uint32_t)b.C;
+            std::vector<const void *> src;
+            if (pc.rot) {
+              d.rot = true;
+              for (int32_t e = 0; e < p.N; ++e) src.push_back(contrib_at(e, lo));
+            } else {
+              d.rot = false;
+              d.m = pc.m;
+              for (int32_t t = 0; t < d.m; ++t) src.push_back(contrib_at((int32_t)((pc.e0 + t) % p.N), lo));
+            }
+            if (f[5] == ES_BUF_PART) d.part_in = reinterpret_cast<const float *>(part_at(f[6], lo));
+            else if (pc.part) d.part_in = reinterpret_cast<const float *>(h->ws + p.inc_off + p.inc_bucket_off[bucket]) + lo;
+            d.out_partial = f[7] == ES_BUF_PART;
+            d.out = d.out_partial ? (void *)part_at(f[8], lo) : (void *)(outp + (uint64_t)lo * esz);
+            pend_bytes +=
+                (uint64_t)d.n * ((uint64_t)src.size() * esz + (d.part_in ? 4 : 0) + (d.out_partial ? 4 : esz));
+            pend.push_back(d);
+            pend_src.push_back(std::move(src));
           }
-          d.part_in = f[5] == ES_BUF_PART ? reinterpret_cast<const float *>(part_at(f[6], lo)) : nullptr;
-          d.out_partial = f[7] == ES_BUF_PART;
-          d.out = d.out_partial ? (void *)part_at(f[8], lo) : (void *)(outp + (uint64_t)lo * esz);
-          pend_bytes += (uint64_t)d.n * ((uint64_t)src.size() * esz + (d.part_in ? 4 : 0) + (d.out_partial ? 4 : esz));
-          pend.push_back(d);
-          pend_src.push_back(std::move(src));
           break;
         }
         case ES_OP_GROUP_BEGIN:

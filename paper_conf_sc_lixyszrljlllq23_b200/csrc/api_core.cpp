@@ -56,6 +56,25 @@ es_status es_plan_ops(const es_config *cfg, int32_t bucket, int64_t *ops, size_t
   return ES_OK;
 }
 
+es_status es_plan_incremental(const es_config *cfg, int32_t bucket, int64_t *rows, size_t cap_rows,
+                              size_t *n_rows) {
+  if (!n_rows) return set_err(ES_EINVAL, "n_rows is NULL");
+  es::Plan p;
+  std::string err;
+  es_status s = es::build_plan(cfg, &p, &err, false);
+  if (s != ES_OK) return set_err(s, err);
+  if (bucket < 0 || bucket >= (int32_t)p.bp.size()) return set_err(ES_EINVAL, "bucket out of range");
+  const es::BucketPlan &b = p.bp[bucket];
+  *n_rows = b.inc.size();
+  if (rows)
+    for (size_t i = 0; i < b.inc.size() && i < cap_rows; ++i) {
+      const es::IncChunk &ic = b.inc[i];
+      const int64_t r[5] = {ic.c, ic.first, ic.q, ic.lo, ic.hi};
+      std::memcpy(rows + 5 * i, r, sizeof r);
+    }
+  return ES_OK;
+}
+
 es_status es_init(const es_config *cfg, void *workspace, size_t workspace_bytes, es_handle *out) {
   ES_NVTX();
   if (!out) return set_err(ES_EINVAL, "out is NULL");

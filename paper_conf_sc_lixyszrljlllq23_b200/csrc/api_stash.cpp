@@ -127,11 +127,13 @@ es_status es_stash_fold_grads(es_handle h, int32_t est, int32_t n, const int32_t
   es_status s = check_handle(h);
   if (s != ES_OK) return s;
   const es::Plan &p = h->plan;
-  if (!(p.options & ES_OPT_INCREMENTAL) || p.G != 1)
-    return set_err(ES_EUNSUPPORTED, "es_stash_fold_grads needs G == 1 and ES_OPT_INCREMENTAL");
+  if (!(p.options & ES_OPT_INCREMENTAL))
+    return set_err(ES_EUNSUPPORTED, "es_stash_fold_grads needs ES_OPT_INCREMENTAL");
   if (n < 0 || (n > 0 && (!buckets || !grads || !gdts))) return set_err(ES_EINVAL, "bad bucket/grad arrays");
   if (est < 0 || est >= p.N) return set_err(ES_EINVAL, "est out of range");
   if (mode != ES_STASH_COPY && mode != ES_STASH_BORROW) return set_err(ES_EINVAL, "mode must be COPY or BORROW");
+  const int32_t li = p.local_index[est];
+  if (li < 0) return set_err(ES_ESTATE, "est is not mapped to this rank");
   for (int32_t i = 0; i < n; ++i) {
     const int32_t bk = buckets[i];
     if (bk < 0 || bk >= h->B) return set_err(ES_EINVAL, "bucket out of range");
@@ -141,14 +143,13 @@ es_status es_stash_fold_grads(es_handle h, int32_t est, int32_t n, const int32_t
       return set_err(ES_EINVAL, "grad must be a 16-byte aligned device pointer");
     for (int32_t j = 0; j < i; ++j)
       if (buckets[j] == bk) return set_err(ES_EINVAL, "bucket listed twice");
-    if (h->inc_next[bk] != est)
-      return set_err(ES_ESTATE, "incremental fold expects the ESTs of a bucket in order 0, 1, ..., N-1");
-    if (est == 0)
-      for (int32_t li = 0; li < h->n_local; ++li)
-        if (h->stashed[(size_t)li * h->B + bk])
+    if (h->inc_next[bk] != li)
+      return set_err(ES_ESTATE, "incremental fold expects the local ESTs of a bucket in ascending order");
+    if (li == 0)
+      for (int32_t lj = 0; lj < h->n_local; ++lj)
+        if (h->stashed[(size_t)lj * h->B + bk])
           return set_err(ES_ESTATE, "bucket already stashed this step with es_stash_grad(s)");
   }
-  const int32_t li = p.local_index[est];
   cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
   const unsigned long long cap = capture_id(cs);
   for (int32_t i = 0; i < n; ++i) {
@@ -157,12 +158,14 @@ es_status es_stash_fold_grads(es_handle h, int32_t est, int32_t n, const int32_t
       return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
   }
   const float r = 1.0f / (float)p.N;
+  std::vector<uint8_t> folded(n, 0);
   for (int dd = 0; dd < 2; ++dd) {
-    // (i) fold x_est into the partials of chunks c < est (R2: est follows c+1..est-1)
+    // (i) fold x_est into the partials of the chunks whose planned prefix holds it
+    //     (plan_incremental): est is position t of the sequence first, first+1, ...
     std::vector<es::FoldSegDesc> segs;
     std::vector<std::vector<const void *>> srcs;
     uint64_t fbytes = 0;
-    // (ii) stash chunks >= est (they wait for the wrap)
+    // (ii) stash the rest: what the end fold, the exchange or peers still read
     std::vector<es::StashSegDesc> st;
     uint64_t sbytes = 0;
     for (int32_t i = 0; i < n; ++i) {
@@ -171,34 +174,44 @@ es_status es_stash_fold_grads(es_handle h, int32_t est, int32_t n, const int32_t
       if ((int)b.dtype != dd || b.L == 0) continue;
       const unsigned char *x = reinterpret_cast<const unsigned char *>(grads[i]);
       float *part = reinterpret_cast<float *>(h->ws + p.inc_off + p.inc_bucket_off[bk]);
-      const int64_t L = (int64_t)b.L, C = (int64_t)b.C;
-      // The last EST's fold is deferred into the end-of-step fold (which reads
-      // its gradient right after the partials), so the partials make no extra
-      // round trip through HBM on the critical path: nothing is folded here.
-      const bool last = est == p.N - 1;
-      const int64_t cont_hi = last ? 0 : std::min<int64_t>(L, (int64_t)std::max(est - 1, 0) * C);   // chunks < est-1
-      const int64_t inc_hi = last ? 0 : std::min<int64_t>(L, (int64_t)est * C);                     // chunks < est
-      auto add = [&](int64_t lo, int64_t hi, bool cont) {
-        if (hi <= lo) return;
-        es::FoldSegDesc d;
-        d.lo = lo;
-        d.n = hi - lo;
-        d.C = (uint32_t)b.C;
-        d.rot = false;
-        d.m = 1;
-        d.part_in = cont ? part + lo : nullptr;
-        d.out_partial = true;
-        d.out = part + lo;
-        segs.push_back(d);
-        srcs.push_back({x + (uint64_t)lo * b.esize});
-        fbytes += (uint64_t)(hi - lo) * (b.esize + (cont ? 8 : 4));
-      };
-      add(0, cont_hi, true);           // partial continues
-      add(cont_hi, inc_hi, false);     // chunk est-1: est is its first EST (c+1)
-      if (mode == ES_STASH_COPY && inc_hi < L) {
+      std::vector<std::pair<int64_t, int64_t>> used;   // ranges consumed here, ascending
+      for (const es::IncChunk &ic : b.inc) {
+        const int32_t t = (int32_t)(((int64_t)est - ic.first + p.N) % p.N);
+        if (t >= ic.q) continue;
+        const bool cont = t > 0;                 // t == 0: est opens the partial (c+1)
+        // adjacent ranges with the same continuation merge into one segment
+        if (!segs.empty() && srcs.back()[0] == (const void *)(x + (uint64_t)segs.back().lo * b.esize) &&
+            segs.back().lo + segs.back().n == ic.lo && (segs.back().part_in != nullptr) == cont) {
+          segs.back().n += ic.hi - ic.lo;
+        } else {
+          es::FoldSegDesc d;
+          d.lo = ic.lo;
+          d.n = ic.hi - ic.lo;
+          d.C = (uint32_t)b.C;
+          d.rot = false;
+          d.m = 1;
+          d.part_in = cont ? part + ic.lo : nullptr;
+          d.out_partial = true;
+          d.out = part + ic.lo;
+          segs.push_back(d);
+          srcs.push_back({x + (uint64_t)ic.lo * b.esize});
+        }
+        fbytes += (uint64_t)(ic.hi - ic.lo) * (b.esize + (cont ? 8 : 4));
+        if (!used.empty() && used.back().second == ic.lo) used.back().second = ic.hi;
+        else used.push_back({ic.lo, ic.hi});
+      }
+      folded[i] = !used.empty();
+      if (mode == ES_STASH_COPY) {
         unsigned char *slot = h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[bk];
-        st.push_back({x + (uint64_t)inc_hi * b.esize, slot + (uint64_t)inc_hi * b.esize, L - inc_hi});
-        sbytes += 2 * (uint64_t)(L - inc_hi) * b.esize;
+        int64_t at = 0;
+        used.push_back({(int64_t)b.L, (int64_t)b.L});
+        for (const auto &u : used) {
+          if (u.first > at) {
+            st.push_back({x + (uint64_t)at * b.esize, slot + (uint64_t)at * b.esize, u.first - at});
+            sbytes += 2 * (uint64_t)(u.first - at) * b.esize;
+          }
+          at = u.second;
+        }
       }
     }
     if (!segs.empty()) {
@@ -224,9 +237,9 @@ es_status es_stash_fold_grads(es_handle h, int32_t est, int32_t n, const int32_t
     if (cudaEventRecord(h->stash_ev[k], cs) != cudaSuccess) return h->poison(ES_ECUDA, "cudaEventRecord failed");
     h->stash_cap[k] = cap;
     h->stashed[k] = 1;
-    h->inc_next[buckets[i]] = est + 1;
-    // the slot holds the whole gradient iff nothing of it was folded here (EST 0, the last EST)
-    h->inc_full[k] = mode == ES_STASH_COPY && (est == 0 || est == p.N - 1) ? 1 : 0;
+    h->inc_next[buckets[i]] = li + 1;
+    // the slot holds the whole gradient iff nothing of it was folded here
+    h->inc_full[k] = mode == ES_STASH_COPY && !folded[i] ? 1 : 0;
   }
   return ES_OK;
 }

@@ -323,6 +323,48 @@ void plan_peer_chain(const Plan &p, BucketPlan *b) {
       b->ops.push_back(make_op(ES_OP_GATHER, sh.rng[c].lo, sh.rng[c].hi, p.est_to_gpu[c]));
 }
 
+// NEXT-1 (PAPER.md:599-606 overlaps the gradient swap with the
+// next EST's compute): which ESTs of which chunks this rank can fold into a
+// running fp32 partial at their stashes, before any exchange.  A left fold is
+// segmentable (R14), so the partial of the first q ESTs of a sequence that
+// starts here, continued by the end fold over the rest, gives the same bits.
+// Local ESTs stash in ascending order, so the prefix stops at the wrap
+// N-1 -> 0; it never takes the last local EST (nothing is left to overlap
+// with after its stash, and the end fold reads it straight from its stash)
+// and leaves the segment's end fold at least one source.
+void plan_incremental(const Plan &p, BucketPlan *b) {
+  b->inc.clear();
+  b->inc_q.assign(p.N, 0);
+  if (b->L == 0 || p.local_ests.empty()) return;
+  const int32_t g = p.rank, last_local = p.local_ests.back();
+  const bool shard = b->sched == ES_SCHED_DIRECT || b->sched == ES_SCHED_PEER;
+  std::vector<Seg> segs;
+  for (int32_t c = 0; c < p.N; ++c) {
+    Range r = chunk_range(b->L, b->C, c);
+    const int32_t first = (int32_t)(((int64_t)c + 1) % p.N);
+    if (p.est_to_gpu[first] != g) continue;   // the sequence does not start here
+    if (shard) {
+      r.lo = std::max<int64_t>(r.lo, b->shard_lo);
+      r.hi = std::min<int64_t>(r.hi, b->shard_hi);
+    }
+    if (r.hi <= r.lo) continue;
+    int32_t seg_len = p.N;                    // G == 1, DIRECT, PEER: the whole sequence folds here
+    if (b->sched == ES_SCHED_CHAIN || b->sched == ES_SCHED_PEER_CHAIN) {
+      chunk_segments(p, c, &segs);
+      seg_len = segs[0].m;                    // the chain's first segment (on this rank)
+    }
+    int32_t q = 0;
+    while (q < seg_len - 1) {
+      const int32_t e = first + q;
+      if (e >= p.N || p.est_to_gpu[e] != g || e == last_local) break;
+      ++q;
+    }
+    if (q == 0) continue;
+    b->inc_q[c] = q;
+    b->inc.push_back({c, first, q, r.lo, r.hi});
+  }
+}
+
 bool fail(std::string *err, const char *msg) {
   if (err) *err = msg;
   return false;
@@ -366,7 +408,6 @@ bool validate(const es_config *cfg, std::string *err, bool need_comm) {
     return fail(err, "compat PREDIV and PREMUL are exclusive");
   if (cfg->options & ~(uint32_t)(ES_OPT_INCREMENTAL | ES_OPT_PEER_ROUNDS | ES_OPT_STASH_BACKGROUND | ES_OPT_PEER_PUSH))
     return fail(err, "unknown option bits");
-  if ((cfg->options & ES_OPT_INCREMENTAL) && cfg->G != 1) return fail(err, "ES_OPT_INCREMENTAL needs G == 1");
   const bool peer_sched = cfg->sched == ES_SCHED_PEER || cfg->sched == ES_SCHED_PEER_CHAIN ||
                           cfg->sched == ES_SCHED_PEER_AUTO;
   if (cfg->G > 1 && need_comm && !peer_sched) {
@@ -431,6 +472,7 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
       else if (s == ES_SCHED_PEER_CHAIN) plan_peer_chain(*p, &b);
       else plan_direct(*p, &b);
     }
+    if (p->options & ES_OPT_INCREMENTAL) plan_incremental(*p, &b);
     max_stage = std::max(max_stage, b.stage_bytes);
     max_parts = std::max(max_parts, b.part_bytes);
     b.peer_part_base = sum_peer_parts;   // buckets of one batched call run their rounds together

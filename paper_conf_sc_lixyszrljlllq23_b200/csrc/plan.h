@@ -27,6 +27,19 @@ struct Part {
   uint64_t off;
 };
 
+// NEXT-1 (incremental fold): a chunk whose canonical sequence starts on this
+// rank (the first segment of a chain, or the local run opening a DIRECT/PEER
+// shard fold) folds its first q ESTs into fp32 partials at their stashes.
+// [lo, hi): the elements this rank folds for the chunk (chunk, or chunk and
+// shard); first = (c+1) mod N.  q >= 1 only; q ends before the wrap N-1 -> 0
+// (ESTs run in ascending order), never takes this rank's last local EST (its
+// contribution joins the end fold straight from its stash) and leaves at least
+// one source of the segment to the end fold.
+struct IncChunk {
+  int32_t c, first, q;
+  int64_t lo, hi;
+};
+
 struct BucketPlan {
   uint64_t L = 0;
   es_dtype dtype = ES_F32;
@@ -46,6 +59,8 @@ struct BucketPlan {
   uint64_t pipe_flag_base = 0;          // PEER_CHAIN: first tile flag (u64 words) of this bucket;
                                         //   chunk c, round r, tile t at base + (c*R + r)*tiles_per_chunk + t
   std::vector<Op> ops;
+  std::vector<IncChunk> inc;            // NEXT-1 (ES_OPT_INCREMENTAL): chunks with q >= 1, ascending c
+  std::vector<int32_t> inc_q;           // NEXT-1: [N] q of chunk c on this rank (0: none)
 };
 
 struct Plan {

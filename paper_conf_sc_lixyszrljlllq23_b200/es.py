@@ -35,7 +35,7 @@ EXPORTED = [
     "es_read_state", "es_switch_context", "es_stash_grad", "es_stash_grads", "es_stash_and_switch", "es_stash_fold_grads", "es_allreduce",
     "es_allreduce_many", "es_chunk_elems", "es_slot_ptr", "es_context_bytes", "es_export_context",
     "es_import_context", "es_dropout", "es_peer_blob", "es_peer_open",
-    "es_plan_ops", "es_loopback_create", "es_loopback_destroy", "es_profile_enable",
+    "es_plan_ops", "es_plan_incremental", "es_loopback_create", "es_loopback_destroy", "es_profile_enable",
     "es_profile_reset", "es_profile_query", "es_set_launch_override", "es_status_string",
     "es_last_error", "es_abi_version",
 ]
@@ -109,6 +109,7 @@ def lib():
         "es_export_context": (st, [P, i32, P, sz, P]),
         "es_import_context": (st, [P, i32, P, sz, P]),
         "es_plan_ops": (st, [cfgp, i32, ctypes.POINTER(i64), sz, ctypes.POINTER(sz), ctypes.POINTER(i32)]),
+        "es_plan_incremental": (st, [cfgp, i32, ctypes.POINTER(i64), sz, ctypes.POINTER(sz)]),
         "es_loopback_create": (st, [i32, ctypes.POINTER(P)]),
         "es_loopback_destroy": (st, [P]),
         "es_profile_enable": (st, [P, i32]),
@@ -290,6 +291,16 @@ def es_plan_ops(cfg, bucket):
     _check(lib().es_plan_ops(cfg.ptr(), bucket, ops.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)), n.value,
                              ctypes.byref(n), ctypes.byref(sched)), "es_plan_ops")
     return ops[: n.value], sched.value
+
+
+def es_plan_incremental(cfg, bucket):
+    """-> int64 array [n_rows, 5]: (c, first, q, lo, hi) per chunk with an incremental prefix."""
+    n = ctypes.c_size_t()
+    _check(lib().es_plan_incremental(cfg.ptr(), bucket, None, 0, ctypes.byref(n)), "es_plan_incremental")
+    rows = np.zeros((max(n.value, 1), 5), dtype=np.int64)
+    _check(lib().es_plan_incremental(cfg.ptr(), bucket, rows.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
+                                     n.value, ctypes.byref(n)), "es_plan_incremental")
+    return rows[: n.value]
 
 
 def es_loopback_create(G):

@@ -12,4 +12,7 @@ R 8 reh_bert_g8rr --config bert_base --mapping round_robin
 R 2 reh_swin_g2 --config swin_b
 R 2 reh_resnet50_g2_failopen --config resnet50 --simulate-peer-failure open
 R 2 reh_resnet50_g2_failparity --config resnet50 --simulate-peer-failure parity
-echo done > $O/done.txt
+echo done1 > $O/done.txt
+# launch list of the default command (swin_b), cold-cache serialised per-launch times
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 600 --csv --log-file $O/launches_swin_b_default.csv python bench.py --steps 2 --warmup 3 --no-cpu --no-e2e --no-full-parity > $O/ncu_launch.log 2>&1
+echo done2 >> $O/done.txt

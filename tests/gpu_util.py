@@ -125,7 +125,9 @@ def reduce_loopback(xs_per_bucket, G, mapping, sched=es.ES_SCHED_AUTO, A=16, bor
                     loc = a.local_ests
                     for i, k in enumerate(loc):
                         mode = es.ES_STASH_BORROW if (borrow_last and i == len(loc) - 1) else es.ES_STASH_COPY
-                        if batched:
+                        if options & es.ES_OPT_INCREMENTAL:      # NEXT-1: fold at the stash
+                            a.stash_fold(k, range(len(buckets)), [devs[b][k] for b in range(len(buckets))], mode)
+                        elif batched:
                             a.stash_many(k, range(len(buckets)), [devs[b][k] for b in range(len(buckets))], mode)
                         else:
                             for b in range(len(buckets)):

@@ -560,10 +560,78 @@ def test_incremental_fold_protocol_and_graph():
     torch.cuda.synchronize()
     assert_bits_equal(from_dev(out), oracle.reduce(xs, "f32"))
     agg.close()
-    with pytest.raises(es.EsError) as e:              # G > 1 is refused at init
-        Aggregator(4, 2, 0, [0, 0, 1, 1], [(L, "f32")], options=es.ES_OPT_INCREMENTAL,
-                   transport=es.ES_TRANSPORT_LOOPBACK, comm=es.es_loopback_create(2).value)
-    assert e.value.status == es.ES_EINVAL
+
+
+def _inc_want(xs, dts):
+    return [oracle.reduce(x, d) for x, d in zip(xs, dts)]
+
+
+@pytest.mark.parametrize("G,kind", [(2, "contiguous"), (4, "contiguous"), (8, "contiguous"), (2, "round_robin"),
+                                    (4, "round_robin"), (8, "round_robin"), (2, "random"), (4, "random"),
+                                    (3, "random")])
+@pytest.mark.parametrize("sched", [es.ES_SCHED_AUTO, es.ES_SCHED_DIRECT, es.ES_SCHED_CHAIN, es.ES_SCHED_PEER,
+                                   es.ES_SCHED_PEER_CHAIN, es.ES_SCHED_PEER_AUTO])
+def test_incremental_fold_loopback_n8(G, kind, sched):
+    """NEXT-1 at G > 1: every rank folds the local prefix of each sequence that
+    starts on it (chain first segments, the local run opening a DIRECT/PEER
+    shard fold) into fp32 partials at the stashes; the end fold continues from
+    them.  Two steps on the same handles (partials reused), oracle bits on
+    every rank, for every schedule and mapping kind."""
+    rng = np.random.default_rng(1500 + G * 10 + len(kind))
+    dts = ["f32", "bf16", "f32"]
+    xs = [_gauss(rng, 8, 200003), _gauss(rng, 8, 4096 + 5, "bf16"), _gauss(rng, 8, 40)]
+    res = reduce_loopback(xs, G, workloads.mapping(8, G, kind), sched, steps=2,
+                          options=es.ES_OPT_INCREMENTAL)
+    want = _inc_want(xs, dts)
+    for g in range(G):
+        for b in range(3):
+            assert_bits_equal(res[g][b], want[b], f"inc G={G} {kind} sched={sched} rank={g} b={b}")
+
+
+@pytest.mark.parametrize("kind", ["contiguous", "round_robin"])
+@pytest.mark.parametrize("sched", [es.ES_SCHED_AUTO, es.ES_SCHED_PEER_AUTO, es.ES_SCHED_CHAIN,
+                                   es.ES_SCHED_PEER_CHAIN])
+def test_incremental_fold_bert_n12_g8(kind, sched):
+    """NEXT-1 on the BERT shape: N=12 bf16 on G=8, uneven n_g, both maps."""
+    rng = np.random.default_rng(1600 + len(kind))
+    xs = [_gauss(rng, 12, 120011, "bf16"), _gauss(rng, 12, 30000, "bf16")]
+    res = reduce_loopback(xs, 8, workloads.mapping(12, 8, kind), sched, steps=2, options=es.ES_OPT_INCREMENTAL)
+    want = _inc_want(xs, ["bf16", "bf16"])
+    for g in range(8):
+        for b in range(2):
+            assert_bits_equal(res[g][b], want[b], f"inc bert {kind} sched={sched} rank={g} b={b}")
+
+
+@pytest.mark.parametrize("G", [2, 3, 4])
+def test_incremental_fold_all_maps_n4(G):
+    """Every surjective map of N=4 onto G ranks, AUTO and PEER_AUTO, with NEXT-1."""
+    rng = np.random.default_rng(1700 + G)
+    xs = [_gauss(rng, 4, 1000), _gauss(rng, 4, 77, "bf16")]
+    want = _inc_want(xs, ["f32", "bf16"])
+    for m in _surjections(4, G):
+        for sched in (es.ES_SCHED_AUTO, es.ES_SCHED_PEER_AUTO):
+            res = reduce_loopback(xs, G, m, sched, options=es.ES_OPT_INCREMENTAL)
+            for g in range(G):
+                for b in range(2):
+                    assert_bits_equal(res[g][b], want[b], f"inc map={m} sched={sched} rank={g} b={b}")
+
+
+def test_incremental_fold_g2_protocol():
+    """G > 1: local ESTs must come in ascending order; a remote EST is refused."""
+    from gpu_util import Aggregator, to_dev
+    L = 5000
+    world = es.es_loopback_create(2)
+    agg = Aggregator(4, 2, 0, [0, 0, 1, 1], [(L, "f32")], options=es.ES_OPT_INCREMENTAL,
+                     transport=es.ES_TRANSPORT_LOOPBACK, comm=world.value)
+    x = to_dev(np.ones(L, np.float32))
+    with pytest.raises(es.EsError) as e:              # EST 1 before EST 0
+        agg.stash_fold(1, [0], [x])
+    assert e.value.status == es.ES_ESTATE
+    with pytest.raises(es.EsError) as e:              # EST 2 lives on rank 1
+        agg.stash_fold(2, [0], [x])
+    assert e.value.status == es.ES_ESTATE
+    agg.close()
+    es.es_loopback_destroy(world)
 
 
 # ---- maximum sizes ----------------------------------------------------------------------------
@@ -686,6 +754,8 @@ def test_random_schedules_mappings_layouts(seed):
     options = int(rng.choice([0, es.ES_OPT_PEER_ROUNDS]))
     if seed % 3 == 2:                                             # a third of the seeds push the gather
         options |= es.ES_OPT_PEER_PUSH
+    if seed % 4 == 1:                                             # a quarter fold at the stash (NEXT-1)
+        options |= es.ES_OPT_INCREMENTAL
     steps = int(rng.integers(1, 4))
     xs = [_gauss(rng, N, L, d) for L, d in zip(sizes, dts)]
     want = [oracle.reduce(x, d, A=A) for x, d in zip(xs, dts)]

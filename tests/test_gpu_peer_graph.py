@@ -28,7 +28,10 @@ def _inputs(rng, N, Ls, dts):
 
 
 @pytest.mark.parametrize("sched,options", [(es.ES_SCHED_PEER, 0), (es.ES_SCHED_PEER_CHAIN, 0),
-                                           (es.ES_SCHED_PEER_CHAIN, es.ES_OPT_PEER_ROUNDS)])
+                                           (es.ES_SCHED_PEER_CHAIN, es.ES_OPT_PEER_ROUNDS),
+                                           (es.ES_SCHED_PEER, es.ES_OPT_INCREMENTAL),
+                                           (es.ES_SCHED_PEER_CHAIN, es.ES_OPT_INCREMENTAL),
+                                           (es.ES_SCHED_PEER_AUTO, es.ES_OPT_INCREMENTAL | es.ES_OPT_PEER_ROUNDS)])
 @pytest.mark.parametrize("G,N,kind", [(2, 8, "contiguous"), (4, 12, "random")])
 def test_peer_schedules_under_graph_replay(sched, options, G, N, kind):
     Ls, dts = [120011, 4099, 33], ["f32", "bf16", "f32"]
@@ -51,8 +54,11 @@ def test_peer_schedules_under_graph_replay(sched, options, G, N, kind):
     def step(g):
         a = aggs[g]
         for i, k in enumerate(a.local_ests):
-            a.stash_many(k, range(B), devs[k],
-                         es.ES_STASH_BORROW if i == len(a.local_ests) - 1 else es.ES_STASH_COPY)
+            mode = es.ES_STASH_BORROW if i == len(a.local_ests) - 1 else es.ES_STASH_COPY
+            if options & es.ES_OPT_INCREMENTAL:     # NEXT-1 at G > 1: fold at the stash
+                a.stash_fold(k, range(B), devs[k], mode)
+            else:
+                a.stash_many(k, range(B), devs[k], mode)
         a.allreduce_many(range(B), outs[g])
 
     def on_threads(fn):
