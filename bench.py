@@ -638,9 +638,11 @@ def main():
         if peer:
             fail = ""
             try:
+                blobs = [None] * world           # every rank takes part in the blob exchange
+                dist.all_gather_object(blobs, agg.peer_blob())
                 if attempt == 0 and args.simulate_peer_failure == "open" and rank == world - 1:
                     raise PeerFailure("simulated: es_peer_open returned ES_EUNSUPPORTED (test hook)")
-                agg.peer_connect()               # CUDA IPC map of every peer's workspace (NVLink)
+                agg.peer_open(blobs)             # CUDA IPC map of every peer's workspace (NVLink)
             except (es.EsError, PeerFailure) as e:
                 fail = f"rank {rank}: {e}"
             fails = [f for f in gather_objects(fail) if f]
@@ -906,7 +908,12 @@ def main():
         else:
             us, how = ev_us, "per-launch event pairs"
         bound, bpl, pk = "hbm", bytes_ / n_, peak
-        if costs is not None and kind in ("fold", "gather"):
+        if costs is not None and kind in ("fold", "gather") and rehearse:
+            # rehearsal: every rank on one GPU -- "peer" reads never leave its HBM, so the kernel's
+            # HBM and would-be NVLink bytes are all HBM bytes (and the ranks share that HBM)
+            hb, nv = costs[rank]["kinds"].get(kind, [0, 0])
+            bpl = (hb + nv) / (n_ / steps_profiled)
+        elif costs is not None and kind in ("fold", "gather"):
             # G > 1: the kernel reads peer memory over NVLink (PEER*) -- its bound is the slower of
             # its HBM and NVLink bytes; achieved is measured against that resource
             hb, nv = costs[rank]["kinds"].get(kind, [0, 0])
@@ -922,6 +929,8 @@ def main():
              "avg_launch_us": round(us, 2), "timing": how, "avg_launch_us_event_pairs": round(ev_us, 2),
              "share_of_step": round(us * n_ / steps_profiled / 1e3 / ms, 3),
              "peak_source": peak_src if bound == "hbm" else "B200_PROFILING.md measured peer copy per direction",
+             **({"rehearsal": "all ranks on cuda:0: peer bytes counted as HBM bytes, ranks time-slice one GPU"}
+                if rehearse and costs is not None else {}),
              "frac_of_nominal": round(a / (HBM_NOMINAL_GBPS if bound == "hbm" else NVL_NOMINAL_GBPS), 4)}
         return r
 
@@ -974,6 +983,9 @@ def main():
               "stash_phase_ms": round(stash_ph, 4) if stash_ph is not None else None}
         if costs is not None:
             ar["roofline"] = plan_roofline(costs, ar_ph, peak)
+            if rehearse:   # what the plan would take on G GPUs; measured here on ONE shared GPU
+                ar["roofline"]["rehearsal"] = ("all ranks time-slice cuda:0 (separate processes, no MPS): "
+                                               "t_measured is not a G-GPU time; t_roof is the G-GPU model")
         elif not args.incremental:
             fold_bytes = (N + 1) * sum(n for n, _ in buckets) * esz          # (N+1) L b: SURVEY 8(d), G = 1
             a = fold_bytes / (ar_ph / 1e3) / 1e9
@@ -1176,16 +1188,18 @@ def main():
 
 
 def ring_crosscheck(args, name, N, G, rank, rehearse, dev, host):
-    """NEXT-3 (iii): with N == G (one EST per GPU) run ncclAllReduce(sum) with
-    NCCL_ALGO=Ring, NCCL_PROTO=Simple on a one-channel communicator (min/max CTAs = 1) over a
-    buffer whose per-rank ring chunk equals R1's chunk (L_x = N * 65536 fp32: C = L_x / N, one
-    NCCL loop), then compare its words, times fl32(1/N) (a power of two here: exact), with the
-    oracle's canonical fold of the same inputs.  Agreement 1.0 pins reading R2 to NCCL's ring;
-    anything less says the readings differ from NCCL's order.  Outside the timed region."""
+    """NEXT-3 (iii): one EST per GPU (N_x = G ring participants; rank k contributes
+    EST k's gradients of the workload, so any G >= 2 of a scaling run checks the reading, not only
+    N == G): run ncclAllReduce(sum) with NCCL_ALGO=Ring, NCCL_PROTO=Simple on a one-channel
+    communicator (min/max CTAs = 1) over a buffer whose per-rank ring chunk equals R1's chunk
+    (L_x = N_x * 65536 fp32: C = L_x / N_x, one NCCL loop), then compare its words, times
+    fl32(1/N_x) (a power of two here: exact), with the oracle's canonical fold of the same N_x
+    inputs.  Agreement 1.0 pins reading R2 to NCCL's ring; anything less says the readings differ
+    from NCCL's order.  Outside the timed region."""
     if args.no_ring_check:
         return {"skipped": "--no-ring-check"}
-    if N != G:
-        return {"skipped": f"needs N == G (here N={N}, G={G})"}
+    if G < 2:
+        return {"skipped": "needs G >= 2 ring participants"}
     if rehearse:
         return {"skipped": "rehearsal: NCCL refuses two ranks on one GPU"}
     import numpy as np
@@ -1195,10 +1209,11 @@ def ring_crosscheck(args, name, N, G, rank, rehearse, dev, host):
     cfg = workloads.config(name)
     b = max(range(len(cfg["buckets"])), key=lambda i: cfg["buckets"][i][0] if cfg["buckets"][i][1] == "f32" else -1)
     L_b, d = cfg["buckets"][b]
-    if d != "f32" or (N & (N - 1)):
-        return {"skipped": "needs an fp32 bucket and a power-of-two N (exact 1/N scale on both sides)"}
+    Nx = G                                      # one EST per GPU: ESTs 0..G-1 of the workload
+    if d != "f32" or (Nx & (Nx - 1)):
+        return {"skipped": "needs an fp32 bucket and a power-of-two G (exact 1/G scale on both sides)"}
     per = 65536
-    Lx = min(N * per, (L_b // (N * 16)) * N * 16)
+    Lx = min(Nx * per, (L_b // (Nx * 16)) * Nx * 16)
     saved = {k: os.environ.get(k) for k in ("NCCL_ALGO", "NCCL_PROTO")}
     os.environ["NCCL_ALGO"], os.environ["NCCL_PROTO"] = "Ring", "Simple"
     try:
@@ -1209,7 +1224,7 @@ def ring_crosscheck(args, name, N, G, rank, rehearse, dev, host):
         x = workloads.to_torch(workloads.est_bucket_np(name, rank, b, 0, Lx), dev)
         dist.all_reduce(x, group=pg)
         torch.cuda.synchronize()
-        got = (x * (1.0 / N)).cpu().numpy()
+        got = (x * (1.0 / Nx)).cpu().numpy()
         dist.destroy_process_group(pg)
     except Exception as e:
         return {"error": f"{type(e).__name__}: {e}"}
@@ -1222,13 +1237,14 @@ def ring_crosscheck(args, name, N, G, rank, rehearse, dev, host):
     if rank != 0:
         return None
     import oracle
-    miss = [k for k in range(N) if (k, b) not in host]
+    miss = [k for k in range(Nx) if (k, b) not in host]
     drawn = dict(zip(miss, workloads.window_np(name, b, miss, 0, Lx))) if miss else {}
-    xs = [host[(k, b)][:Lx] if (k, b) in host else drawn[k] for k in range(N)]
+    xs = [host[(k, b)][:Lx] if (k, b) in host else drawn[k] for k in range(Nx)]
     want = oracle.reduce(xs, "f32", L=Lx)
     eq = int((want.view(np.uint32) == got.view(np.uint32)).sum())
-    return {"bucket": b, "elements": Lx, "ring_chunk_elements": Lx // N, "words_equal": eq, "frac_equal": eq / Lx,
-            "nccl": "ncclAllReduce sum, NCCL_ALGO=Ring NCCL_PROTO=Simple, min/max CTAs 1, times fl32(1/N)",
+    return {"bucket": b, "ring_ranks": Nx, "ests": f"0..{Nx - 1} (one per GPU)", "elements": Lx,
+            "ring_chunk_elements": Lx // Nx, "words_equal": eq, "frac_equal": eq / Lx,
+            "nccl": "ncclAllReduce sum, NCCL_ALGO=Ring NCCL_PROTO=Simple, min/max CTAs 1, times fl32(1/G)",
             "nccl_sha256": hashlib.sha256(got.tobytes()).hexdigest(),
             "oracle_sha256": hashlib.sha256(want.tobytes()).hexdigest()}
 

@@ -88,7 +88,14 @@ typedef enum { ES_STASH_COPY = 0, ES_STASH_BORROW = 1, ES_STASH_INPLACE = 2 } es
  *           shards are all-gathered.
  *   CHAIN:  chunk c's unrounded fp32 partial walks the GPUs in canonical
  *           EST order; each GPU folds its consecutive local ESTs; the GPU of
- *           EST c scales, rounds and owns chunk c; then all-gather.
+ *           EST c scales, rounds and owns chunk c; then all-gather.  By
+ *           default the rounds are tile-pipelined: every chunk is cut into
+ *           the same number of tiles W (<= 8, ~2^20 elements each), the fold
+ *           of (round r, tile w) runs on the caller's stream and the transfer
+ *           of its partial on a library-owned side stream, ordered by events,
+ *           in (r + w) wavefront order, so transfers overlap later tiles'
+ *           folds; ES_OPT_PEER_ROUNDS keeps one fold launch + one transfer
+ *           group per round (same bits, same messages per peer pair).
  *   AUTO:   per bucket, the one with fewer max-per-GPU received bytes
  *           (ties -> DIRECT).  The choice is identical on every rank. */
 /*   PEER:   no transport library: rank g's fold kernel pulls the remote
@@ -164,8 +171,10 @@ typedef struct {
 /* ES_OPT_INCREMENTAL: reserve fp32 partials so that es_stash_fold_grads can
  * fold each EST into the running partials at its switch (NEXT-1, any G). */
 #define ES_OPT_INCREMENTAL 1u
-/* ES_OPT_PEER_ROUNDS: PEER_CHAIN without tile pipelining (a device barrier
- * between rounds).  Same bits; kept for comparison and as a fallback. */
+/* ES_OPT_PEER_ROUNDS: CHAIN and PEER_CHAIN without tile pipelining (PEER_CHAIN:
+ * a device barrier between rounds; CHAIN: one fold launch and one transfer
+ * group per round, one stream).  Same bits; kept for comparison and as a
+ * fallback. */
 #define ES_OPT_PEER_ROUNDS 2u
 /* ES_OPT_STASH_BACKGROUND: stash for overlap with the model's compute
  * (PAPER.md:599-606).  A one-shot stash grid of thousands of CTAs is

@@ -49,6 +49,215 @@ void inc_pieces(const es::Plan &p, const es::BucketPlan &b, bool inc, int64_t lo
   }
 }
 
+// ---- transport executor helpers ---------------------------------------------------
+
+// Pending fold segments of one dtype, launched together (multi-segment k_fold).
+struct FoldBatch {
+  std::vector<es::FoldSegDesc> segs;
+  std::vector<std::vector<const void *>> src;
+  es_dtype dt = ES_F32;
+  uint64_t bytes = 0;
+  bool empty() const { return segs.empty(); }
+  es_status flush(es_handle h, cudaStream_t cs, float r) {
+    if (segs.empty()) return ES_OK;
+    const es::Plan &p = h->plan;
+    for (size_t i = 0; i < segs.size(); ++i) segs[i].src = src[i].data();
+    es_status st = h->timed(ES_KERNEL_FOLD, bytes, cs, [&](int *nl) {
+      return es::launch_fold_multi(dt, p.N, r, p.compat, segs.data(), (int)segs.size(), cs, h->blocks_ov,
+                                   h->threads_ov, nl);
+    });
+    segs.clear();
+    src.clear();
+    bytes = 0;
+    return st;
+  }
+};
+
+// Where a bucket's operands live for the transport schedules (G == 1, DIRECT,
+// CHAIN): local contributions (slot or BORROWed buffer), DIRECT staging for
+// remote ones, CHAIN partial buffers, the caller's output.
+struct BucketAddr {
+  es_handle h;
+  const es::Plan &p;
+  int32_t bucket;
+  const es::BucketPlan &b;
+  uint32_t esz;
+  unsigned char *outp;
+  bool inc;   // NEXT-1: every local EST folded its prefix at its stash this step
+  BucketAddr(es_handle hh, int32_t bk, void *out)
+      : h(hh), p(hh->plan), bucket(bk), b(hh->plan.bp[bk]), esz(hh->plan.bp[bk].esize),
+        outp(reinterpret_cast<unsigned char *>(out)),
+        inc((hh->plan.options & ES_OPT_INCREMENTAL) && hh->inc_next[bk] == hh->n_local) {}
+  unsigned char *src_base(int32_t e) const {   // element 0 of local EST e's contribution
+    const int32_t li = p.local_index[e];
+    const void *bw = h->borrowed[(size_t)li * h->B + bucket];
+    if (bw) return reinterpret_cast<unsigned char *>(const_cast<void *>(bw));
+    return h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[bucket];
+  }
+  unsigned char *contrib_at(int32_t e, int64_t lo) const {
+    if (p.local_index[e] >= 0) return src_base(e) + (uint64_t)lo * esz;
+    return h->ws + p.stage_off + (uint64_t)b.stage_index[e] * b.stage_stride + (uint64_t)(lo - b.shard_lo) * esz;
+  }
+  unsigned char *part_at(int64_t id, int64_t lo) const {
+    const es::Part &pt = b.parts[id];
+    return h->ws + p.parts_off + pt.off + (uint64_t)(lo - pt.lo) * 4;
+  }
+  // The segments of FOLD op f restricted to [lo, hi) (a sub-range of the op's range).
+  void fold(const int64_t *f, int64_t lo, int64_t hi, FoldBatch *out) const {
+    if (hi <= lo) return;
+    std::vector<Piece> pcs;   // NEXT-1: pieces continuing from the incremental partials
+    inc_pieces(p, b, inc && f[5] == ES_BUF_NONE, lo, hi, f[3], (int32_t)f[4], &pcs);
+    for (const Piece &pc : pcs) {
+      const int64_t a = pc.lo;
+      es::FoldSegDesc d;
+      d.lo = a;
+      d.n = pc.hi - a;
+      d.C = (uint32_t)b.C;
+      std::vector<const void *> src;
+      if (pc.rot) {
+        d.rot = true;
+        for (int32_t e = 0; e < p.N; ++e) src.push_back(contrib_at(e, a));
+      } else {
+        d.rot = false;
+        d.m = pc.m;
+        for (int32_t t = 0; t < d.m; ++t) src.push_back(contrib_at((int32_t)((pc.e0 + t) % p.N), a));
+      }
+      if (f[5] == ES_BUF_PART) d.part_in = reinterpret_cast<const float *>(part_at(f[6], a));
+      else if (pc.part) d.part_in = reinterpret_cast<const float *>(h->ws + p.inc_off + p.inc_bucket_off[bucket]) + a;
+      d.out_partial = f[7] == ES_BUF_PART;
+      d.out = d.out_partial ? (void *)part_at(f[8], a) : (void *)(outp + (uint64_t)a * esz);
+      out->bytes += (uint64_t)d.n * ((uint64_t)src.size() * esz + (d.part_in ? 4 : 0) + (d.out_partial ? 4 : esz));
+      out->segs.push_back(d);
+      out->src.push_back(std::move(src));
+    }
+  }
+  // SEND / RECV op f restricted to [lo, hi), posted into the open transport group.
+  es_status xfer(const int64_t *f, int64_t lo, int64_t hi) const {
+    if (hi <= lo) return ES_OK;
+    unsigned char *ptr = nullptr;
+    uint64_t w = esz;
+    switch (f[4]) {
+      case ES_BUF_SRC:
+      case ES_BUF_STAGE: ptr = contrib_at((int32_t)f[5], lo); break;
+      case ES_BUF_PART: ptr = part_at(f[5], lo); w = 4; break;
+      case ES_BUF_OUT: ptr = outp + (uint64_t)lo * esz; break;
+      default: return h->poison(ES_ESTATE, "corrupt plan: bad buffer kind");
+    }
+    const size_t nbytes = (size_t)(hi - lo) * w;
+    es_status s = f[0] == ES_OP_SEND ? h->tp->send(ptr, nbytes, (int)f[3]) : h->tp->recv(ptr, nbytes, (int)f[3]);
+    return s == ES_OK ? ES_OK : h->poison(s, h->tp->err);
+  }
+};
+
+// CHAIN over a transport, tile-pipelined.  Every chunk is cut
+// into W tiles (W from the call's largest chunk, <= 8, ~2^20 elements; the
+// same on every rank).  Fold F(r, w) -- round r's segments restricted to tile
+// w -- runs on the caller's stream; transfer T(r, w) -- round r's outgoing
+// partials and round r+1's incoming ones, tile w -- is one transport group on
+// the handle's side stream, after F(r, w); F(r+1, w) waits for T(r, w).  Both
+// streams walk (r, w) in wavefront order (r + w ascending, r ascending), so
+// every rank posts the same group sequence and the per-peer message order of
+// the round executor is kept tile by tile; T(r, w) overlaps F(0, w+1),
+// F(1, w), ...  The all-gather follows as one group on the caller's stream.
+constexpr int64_t kChainTileElems = 1 << 20;
+constexpr int64_t kChainMaxTiles = 8;
+
+es_status chain_pipelined(es_handle h, const std::vector<int32_t> &bks, const std::vector<void *> &outs,
+                          cudaStream_t cs, float r) {
+  const es::Plan &p = h->plan;
+  es_status s;
+  if (!h->side && cudaStreamCreateWithFlags(&h->side, cudaStreamNonBlocking) != cudaSuccess)
+    return h->poison(ES_ECUDA, "cudaStreamCreateWithFlags failed");
+  uint64_t Cmax = 0;
+  int32_t R = 0;
+  for (int32_t bk : bks) {
+    Cmax = std::max(Cmax, p.bp[bk].C);
+    for (int32_t rr : p.bp[bk].op_round) R = std::max(R, rr + 1);
+  }
+  const int64_t W = std::max<int64_t>(1, std::min<int64_t>(kChainMaxTiles, ((int64_t)Cmax + kChainTileElems - 1) /
+                                                                             kChainTileElems));
+  auto tile = [&](int64_t lo, int64_t hi, int64_t w, int64_t *a, int64_t *z) {
+    const int64_t per = ((hi - lo + W - 1) / W + p.A - 1) / p.A * p.A;   // A-aligned: fold needs lo % 8 == 0
+    *a = std::min(hi, lo + w * per);
+    *z = std::min(hi, lo + (w + 1) * per);
+  };
+  const size_t nev = 2 * (size_t)R * (size_t)W + 2;
+  while (h->chain_ev.size() < nev) {
+    cudaEvent_t e = nullptr;
+    if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
+      return h->poison(ES_ECUDA, "cudaEventCreate failed");
+    h->chain_ev.push_back(e);
+  }
+  cudaEvent_t *FE = h->chain_ev.data(), *TE = FE + (size_t)R * W, *start = TE + (size_t)R * W, *join = start + 1;
+  std::vector<uint8_t> te_used((size_t)R * W, 0);
+  std::vector<BucketAddr> ad;
+  ad.reserve(bks.size());
+  for (size_t i = 0; i < bks.size(); ++i) ad.emplace_back(h, bks[i], outs[i]);
+  // the side stream starts after everything before this call on the caller's stream
+  if (cudaEventRecord(*start, cs) != cudaSuccess || cudaStreamWaitEvent(h->side, *start, 0) != cudaSuccess)
+    return h->poison(ES_ECUDA, "event record / wait failed");
+  for (int64_t d = 0; d < R + W - 1; ++d)
+    for (int32_t rr = 0; rr < R; ++rr) {
+      const int64_t w = d - rr;
+      if (w < 0 || w >= W) continue;
+      const size_t ix = (size_t)rr * W + w;
+      if (rr > 0 && te_used[ix - W] && cudaStreamWaitEvent(cs, TE[ix - W], 0) != cudaSuccess)
+        return h->poison(ES_ECUDA, "cudaStreamWaitEvent failed");
+      for (int dd = 0; dd < 2; ++dd) {           // F(rr, w)
+        FoldBatch fb;
+        fb.dt = (es_dtype)dd;
+        for (const BucketAddr &a : ad) {
+          if ((int)a.b.dtype != dd) continue;
+          for (size_t k = 0; k < a.b.ops.size(); ++k) {
+            const int64_t *f = a.b.ops[k].f;
+            if (f[0] != ES_OP_FOLD || a.b.op_round[k] != rr) continue;
+            int64_t lo, hi;
+            tile(f[1], f[2], w, &lo, &hi);
+            a.fold(f, lo, hi, &fb);
+          }
+        }
+        if ((s = fb.flush(h, cs, r)) != ES_OK) return s;
+      }
+      bool any = false;                          // T(rr, w)
+      for (const BucketAddr &a : ad)
+        for (size_t k = 0; k < a.b.ops.size() && !any; ++k) {
+          const int64_t *f = a.b.ops[k].f;
+          if ((f[0] == ES_OP_SEND || f[0] == ES_OP_RECV) && a.b.op_round[k] == rr) {
+            int64_t lo, hi;
+            tile(f[1], f[2], w, &lo, &hi);
+            any = hi > lo;
+          }
+        }
+      if (!any) continue;
+      if (cudaEventRecord(FE[ix], cs) != cudaSuccess || cudaStreamWaitEvent(h->side, FE[ix], 0) != cudaSuccess)
+        return h->poison(ES_ECUDA, "event record / wait failed");
+      if ((s = h->tp->group_begin()) != ES_OK) return h->poison(s, h->tp->err);
+      for (const BucketAddr &a : ad)
+        for (size_t k = 0; k < a.b.ops.size(); ++k) {
+          const int64_t *f = a.b.ops[k].f;
+          if ((f[0] != ES_OP_SEND && f[0] != ES_OP_RECV) || a.b.op_round[k] != rr) continue;
+          int64_t lo, hi;
+          tile(f[1], f[2], w, &lo, &hi);
+          if ((s = a.xfer(f, lo, hi)) != ES_OK) return s;
+        }
+      if ((s = h->tp->group_end(h->side)) != ES_OK) return h->poison(s, h->tp->err);
+      if (cudaEventRecord(TE[ix], h->side) != cudaSuccess) return h->poison(ES_ECUDA, "cudaEventRecord failed");
+      te_used[ix] = 1;
+    }
+  // join the side stream back, then the all-gather of every chain bucket as one group
+  if (cudaEventRecord(*join, h->side) != cudaSuccess || cudaStreamWaitEvent(cs, *join, 0) != cudaSuccess)
+    return h->poison(ES_ECUDA, "event record / wait failed");
+  if ((s = h->tp->group_begin()) != ES_OK) return h->poison(s, h->tp->err);
+  for (const BucketAddr &a : ad)
+    for (size_t k = 0; k < a.b.ops.size(); ++k) {
+      const int64_t *f = a.b.ops[k].f;
+      if ((f[0] == ES_OP_SEND || f[0] == ES_OP_RECV) && a.b.op_round[k] < 0 && (s = a.xfer(f, f[1], f[2])) != ES_OK)
+        return s;
+    }
+  if ((s = h->tp->group_end(cs)) != ES_OK) return h->poison(s, h->tp->err);
+  return ES_OK;
+}
+
 es_status peer_barrier(es_handle h, cudaStream_t cs) {
   const es::Plan &p = h->plan;
   std::vector<uint64_t *> pf(p.G);
@@ -301,108 +510,54 @@ es_status es_allreduce_many(es_handle h, int32_t n, const int32_t *buckets, void
   // Pending FOLD ops: consecutive folds (across buckets for G == 1, within a
   // chain round for G > 1) are independent and go out as one multi-segment
   // launch; a transport group flushes them first.
-  std::vector<es::FoldSegDesc> pend;
-  std::vector<std::vector<const void *>> pend_src;
-  es_dtype pend_dt = ES_F32;
-  uint64_t pend_bytes = 0;
-  auto flush = [&]() -> es_status {
-    if (pend.empty()) return ES_OK;
-    for (size_t i = 0; i < pend.size(); ++i) pend[i].src = pend_src[i].data();
-    es_status st = h->timed(ES_KERNEL_FOLD, pend_bytes, cs, [&](int *nl) {
-      return es::launch_fold_multi(pend_dt, p.N, r, p.compat, pend.data(), (int)pend.size(), cs, h->blocks_ov,
-                                   h->threads_ov, nl);
-    });
-    pend.clear();
-    pend_src.clear();
-    pend_bytes = 0;
-    return st;
-  };
+  FoldBatch pend;
+  // CHAIN buckets run tile-pipelined (chain_pipelined) unless ES_OPT_PEER_ROUNDS; every rank
+  // splits the call alike (the schedule per bucket is global), so messages still match.
+  const bool chain_pipe = p.G > 1 && !(p.options & ES_OPT_PEER_ROUNDS);
+  std::vector<int32_t> chain_i;
 
   for (int32_t i = 0; i < n; ++i) {
     const int32_t bucket = buckets[i];
     const es::BucketPlan &b = p.bp[bucket];
-    const uint32_t esz = b.esize;
-    auto src_base = [&](int32_t e) -> unsigned char * {   // element 0 of local EST e's contribution
-      const int32_t li = p.local_index[e];
-      const void *bw = h->borrowed[(size_t)li * h->B + bucket];
-      if (bw) return reinterpret_cast<unsigned char *>(const_cast<void *>(bw));
-      return h->ws + p.grad_off + (uint64_t)li * p.slot_block + p.slot_off[bucket];
-    };
-    auto contrib_at = [&](int32_t e, int64_t lo) -> unsigned char * {
-      if (p.local_index[e] >= 0) return src_base(e) + (uint64_t)lo * esz;
-      return h->ws + p.stage_off + (uint64_t)b.stage_index[e] * b.stage_stride + (uint64_t)(lo - b.shard_lo) * esz;
-    };
-    auto part_at = [&](int64_t id, int64_t lo) -> unsigned char * {
-      const es::Part &pt = b.parts[id];
-      return h->ws + p.parts_off + pt.off + (uint64_t)(lo - pt.lo) * 4;
-    };
-    unsigned char *outp = reinterpret_cast<unsigned char *>(outs[i]);
-    const bool inc = (p.options & ES_OPT_INCREMENTAL) && h->inc_next[bucket] == h->n_local;
+    if (chain_pipe && b.sched == ES_SCHED_CHAIN) {
+      if (b.L > 0) chain_i.push_back(i);
+      continue;
+    }
+    const BucketAddr ad(h, bucket, outs[i]);
     for (const es::Op &op : b.ops) {
       const int64_t *f = op.f;
       switch (f[0]) {
-        case ES_OP_FOLD: {
-          if (!pend.empty() && pend_dt != b.dtype && (s = flush()) != ES_OK) return s;
-          pend_dt = b.dtype;
-          std::vector<Piece> pcs;   // NEXT-1: pieces continuing from the incremental partials
-          inc_pieces(p, b, inc && f[5] == ES_BUF_NONE, f[1], f[2], f[3], (int32_t)f[4], &pcs);
-          for (const Piece &pc : pcs) {
-            const int64_t lo = pc.lo;
-            es::FoldSegDesc d;
-            d.lo = lo;
-            d.n = pc.hi - lo;
-            d.C = (uint32_t)b.C;
-            std::vector<const void *> src;
-            if (pc.rot) {
-              d.rot = true;
-              for (int32_t e = 0; e < p.N; ++e) src.push_back(contrib_at(e, lo));
-            } else {
-              d.rot = false;
-              d.m = pc.m;
-              for (int32_t t = 0; t < d.m; ++t) src.push_back(contrib_at((int32_t)((pc.e0 + t) % p.N), lo));
-            }
-            if (f[5] == ES_BUF_PART) d.part_in = reinterpret_cast<const float *>(part_at(f[6], lo));
-            else if (pc.part) d.part_in = reinterpret_cast<const float *>(h->ws + p.inc_off + p.inc_bucket_off[bucket]) + lo;
-            d.out_partial = f[7] == ES_BUF_PART;
-            d.out = d.out_partial ? (void *)part_at(f[8], lo) : (void *)(outp + (uint64_t)lo * esz);
-            pend_bytes +=
-                (uint64_t)d.n * ((uint64_t)src.size() * esz + (d.part_in ? 4 : 0) + (d.out_partial ? 4 : esz));
-            pend.push_back(d);
-            pend_src.push_back(std::move(src));
-          }
+        case ES_OP_FOLD:
+          if (!pend.empty() && pend.dt != b.dtype && (s = pend.flush(h, cs, r)) != ES_OK) return s;
+          pend.dt = b.dtype;
+          ad.fold(f, f[1], f[2], &pend);
           break;
-        }
         case ES_OP_GROUP_BEGIN:
-          if ((s = flush()) != ES_OK) return s;
+          if ((s = pend.flush(h, cs, r)) != ES_OK) return s;
           if ((s = h->tp->group_begin()) != ES_OK) return h->poison(s, h->tp->err);
           break;
         case ES_OP_GROUP_END:
           if ((s = h->tp->group_end(cs)) != ES_OK) return h->poison(s, h->tp->err);
           break;
         case ES_OP_SEND:
-        case ES_OP_RECV: {
-          const int64_t lo = f[1], hi = f[2];
-          const int peer = (int)f[3];
-          unsigned char *ptr = nullptr;
-          uint64_t w = esz;
-          switch (f[4]) {
-            case ES_BUF_SRC:
-            case ES_BUF_STAGE: ptr = contrib_at((int32_t)f[5], lo); break;
-            case ES_BUF_PART: ptr = part_at(f[5], lo); w = 4; break;
-            case ES_BUF_OUT: ptr = outp + (uint64_t)lo * esz; break;
-            default: return h->poison(ES_ESTATE, "corrupt plan: bad buffer kind");
-          }
-          const size_t nbytes = (size_t)(hi - lo) * w;
-          s = f[0] == ES_OP_SEND ? h->tp->send(ptr, nbytes, peer) : h->tp->recv(ptr, nbytes, peer);
-          if (s != ES_OK) return h->poison(s, h->tp->err);
+        case ES_OP_RECV:
+          if ((s = ad.xfer(f, f[1], f[2])) != ES_OK) return s;
           break;
-        }
         default:
           return h->poison(ES_ESTATE, "corrupt plan: bad opcode");
       }
     }
   }
-  if ((s = flush()) != ES_OK) return s;
+  if ((s = pend.flush(h, cs, r)) != ES_OK) return s;
+  if (!chain_i.empty()) {
+    std::vector<int32_t> cb;
+    std::vector<void *> co;
+    for (int32_t i : chain_i) {
+      cb.push_back(buckets[i]);
+      co.push_back(outs[i]);
+    }
+    if ((s = chain_pipelined(h, cb, co, cs, r)) != ES_OK) return s;
+  }
   return finish_allreduce(h, n, buckets, cs, cap);
 }
 

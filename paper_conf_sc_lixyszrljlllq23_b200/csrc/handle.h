@@ -103,6 +103,12 @@ struct es_ctx {
   bool peer_open = false;
   int32_t peer_share = 1;                 // ranks of this process sharing the device (loopback)
 
+  // CHAIN over a transport, tile-pipelined: the partials' transfers run on this
+  // library-owned stream (created on first use), ordered against the caller's
+  // stream with events, so they overlap later tiles' folds.
+  cudaStream_t side = nullptr;
+  std::vector<cudaEvent_t> chain_ev;      // ordering events of chain_pipelined (reused per call)
+
   // instrumentation
   bool prof = false;
   struct Rec {
@@ -135,6 +141,8 @@ struct es_ctx {
     for (auto e : pool) cudaEventDestroy(e);
     for (auto e : graph_events) cudaEventDestroy(e);
     for (void *p : ipc_mapped) cudaIpcCloseMemHandle(p);
+    for (auto e : chain_ev) cudaEventDestroy(e);
+    if (side) cudaStreamDestroy(side);
   }
   cudaEvent_t ev() {
     if (!pool.empty()) {

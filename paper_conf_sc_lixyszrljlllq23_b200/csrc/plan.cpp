@@ -225,7 +225,9 @@ void plan_chain(const Plan &p, BucketPlan *b) {
       b->ops.insert(b->ops.end(), xs.begin(), xs.end());
       b->ops.push_back(make_op(ES_OP_GROUP_END));
     }
+    b->op_round.resize(b->ops.size(), r);
   }
+  b->op_round.resize(b->ops.size(), R > 0 ? R - 1 : 0);   // last round's folds (the loop broke early)
   // All-gather: chunk c is finished (scaled, rounded) on the GPU of EST c,
   // the last EST of its sequence; it sends the chunk to every peer.
   b->ops.push_back(make_op(ES_OP_GROUP_BEGIN));
@@ -240,6 +242,7 @@ void plan_chain(const Plan &p, BucketPlan *b) {
     }
   }
   b->ops.push_back(make_op(ES_OP_GROUP_END));
+  b->op_round.resize(b->ops.size(), -1);
 }
 
 // ---- PEER_CHAIN ----------------------------------------------------------------

@@ -59,6 +59,8 @@ struct BucketPlan {
   uint64_t pipe_flag_base = 0;          // PEER_CHAIN: first tile flag (u64 words) of this bucket;
                                         //   chunk c, round r, tile t at base + (c*R + r)*tiles_per_chunk + t
   std::vector<Op> ops;
+  std::vector<int32_t> op_round;        // CHAIN: [ops] round of a fold / of the transfer group after
+                                        //   that round's folds; -1: the final all-gather group
   std::vector<IncChunk> inc;            // NEXT-1 (ES_OPT_INCREMENTAL): chunks with q >= 1, ascending c
   std::vector<int32_t> inc_q;           // NEXT-1: [N] q of chunk c on this rank (0: none)
 };

@@ -714,6 +714,26 @@ def test_peer_chain_pipelined_many_tiles(options, G, N, kind):
             assert_bits_equal(res[g][b], want[b], f"G={G} N={N} {kind} opt={options} rank={g} b={b}")
 
 
+@pytest.mark.parametrize("options", [0, es.ES_OPT_PEER_ROUNDS, es.ES_OPT_INCREMENTAL])
+@pytest.mark.parametrize("G,N,kind", [(2, 4, "contiguous"), (4, 4, "contiguous"), (3, 6, "random"),
+                                      (2, 8, "round_robin")])
+def test_chain_tile_pipelined_transport(options, G, N, kind):
+    """CHAIN over a transport (loopback here, NCCL on a multi-GPU box): chunks of
+    ~3 M elements are cut into W = 3 tiles whose folds (caller's stream) and
+    partial transfers (the handle's side stream) run in wavefront order; the
+    round executor (ES_OPT_PEER_ROUNDS) and NEXT-1 on top of the pipelined one
+    give the same bits.  Two steps reuse the events, side stream and partials."""
+    rng = np.random.default_rng(1400 + G * N + len(kind))
+    L = N * (3 << 20) + 13
+    xs = [_gauss(rng, N, L), _gauss(rng, N, N * (1 << 20) + 8, "bf16"), _gauss(rng, N, 100)]
+    want = [oracle.reduce(xs[0], "f32"), oracle.reduce(xs[1], "bf16"), oracle.reduce(xs[2], "f32")]
+    m = workloads.mapping(N, G, kind, seed=5)
+    res = reduce_loopback(xs, G, m, es.ES_SCHED_CHAIN, steps=2, batched=True, options=options)
+    for g in range(G):
+        for b in range(3):
+            assert_bits_equal(res[g][b], want[b], f"G={G} N={N} {kind} opt={options} rank={g} b={b}")
+
+
 def test_peer_auto_mixed_pipelined():
     """PEER_AUTO mixes PEER and PEER_CHAIN buckets in one batched call; both
     share the pipelined step's two barriers."""
