@@ -76,6 +76,7 @@ def parse(argv=None):
     p.add_argument("--no-ring-check", action="store_true", help="skip NEXT-3 (iii), the NCCL ring cross-check (N == G)")
     p.add_argument("--no-full-parity", action="store_true", help="check sampled windows only (not the whole output)")
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-next1", action="store_true", help="skip the NEXT-1 (incremental fold) leg after the timed region")
     p.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     p.add_argument("--cpu-seconds", type=float, default=10.0)
     return p.parse_args(argv)
@@ -621,12 +622,15 @@ def main():
 
     snb = workloads.state_nbytes()
     grads_host = {k: [host[(k, b)] for b in range(B)] for k in local}
-    opts_base = ((es.ES_OPT_INCREMENTAL if args.incremental else 0) |
+    fuse = not (args.per_bucket or args.no_fuse or args.incremental or args.inplace)
+    next1_leg = fuse and not args.no_graph and not args.no_next1
+    # NEXT-1 leg (after the timed region): the incremental step on the same handle -- the option
+    # only reserves the fp32 partials; the timed step never calls es_stash_fold_grads
+    opts_base = ((es.ES_OPT_INCREMENTAL if (args.incremental or next1_leg) else 0) |
                  (es.ES_OPT_STASH_BACKGROUND if args.stash_background else 0) |
                  (es.ES_OPT_PEER_PUSH if args.peer_push else 0))
     sched_ids = {"auto": es.ES_SCHED_AUTO, "direct": es.ES_SCHED_DIRECT, "chain": es.ES_SCHED_CHAIN,
                  "peer": es.ES_SCHED_PEER, "peer_chain": es.ES_SCHED_PEER_CHAIN, "peer_auto": es.ES_SCHED_PEER_AUTO}
-    fuse = not (args.per_bucket or args.no_fuse or args.incremental or args.inplace)
 
     def build(sched_name, extra, attempt):
         sched = sched_ids[sched_name]
@@ -842,7 +846,8 @@ def main():
                         flush_sink.copy_(flush_words.amax())
                     g_.replay()
             torch.cuda.synchronize()
-            phase_samples.append((marks[0].elapsed_time(marks[1]), marks[1].elapsed_time(marks[2])))
+            phase_samples.append((marks[0].elapsed_time(marks[1]), marks[1].elapsed_time(marks[2]),
+                                  marks[0].elapsed_time(marks[2])))
         with torch.cuda.stream(stream):
             for g_ in (graph, graph_prof):
                 if flush is not None:
@@ -851,7 +856,8 @@ def main():
                 g_.replay()
         torch.cuda.synchronize()
     elif args.steps >= 2:
-        phase_samples.append((marks[0].elapsed_time(marks[1]), marks[1].elapsed_time(marks[2])))
+        phase_samples.append((marks[0].elapsed_time(marks[1]), marks[1].elapsed_time(marks[2]),
+                              marks[0].elapsed_time(marks[2])))
     if world > 1:
         dist.barrier()
     clk = clocks.stop(t_start, t_end)
@@ -861,8 +867,10 @@ def main():
     # phase times of this rank (median of the samples), then max over ranks
     stash_ph = statistics.median(p[0] for p in phase_samples) if phase_samples else None
     ar_ph = statistics.median(p[1] for p in phase_samples) if phase_samples else None
+    # the same replays' stash-start -> allreduce-done span (the allreduce phase is part of it)
+    span_ph = statistics.median(p[2] for p in phase_samples) if phase_samples else None
     if world > 1 and ar_ph is not None:
-        stash_ph, ar_ph = max_over_ranks(stash_ph), max_over_ranks(ar_ph)
+        stash_ph, ar_ph, span_ph = max_over_ranks(stash_ph), max_over_ranks(ar_ph), max_over_ranks(span_ph)
 
     kinds = {"stash": es.ES_KERNEL_STASH, "fold": es.ES_KERNEL_FOLD, "swap": es.ES_KERNEL_SWAP,
              "gather": es.ES_KERNEL_GATHER, "barrier": es.ES_KERNEL_BARRIER}
@@ -898,6 +906,14 @@ def main():
     if ar_ph is not None and G == 1 and not args.incremental:
         phase_ms["fold"] = ar_ph
 
+    def steady_traffic(kname, us, pk):
+        # ncu --cache-control none over the graph replays: DRAM bytes per launch with the previous
+        # kernel's dirty L2 lines written back under this one (what the timed step sees)
+        b = traffic_all.get(f"{kname}_dram_bytes_per_launch_steady")
+        if not b:
+            return {}
+        return {"traffic_steady": b, "frac_steady": round(b / (us / 1e6) / 1e9 / pk, 4)}
+
     def roof(kind, kname):
         n_, ms_, bytes_ = prof[kind]
         if n_ == 0 or ms_ <= 0:
@@ -925,6 +941,7 @@ def main():
         a = bpl / (us / 1e6) / 1e9
         r = {"bound": bound, "kernel": kname, "achieved": round(a, 1), "peak": pk, "unit": "GB/s",
              "frac": round(a / pk, 4), "traffic": traffic_all.get(f"{kname}_dram_bytes_per_launch"),
+             **steady_traffic(kname, us, pk),
              "algorithmic_bytes_per_launch": int(bpl), "launches_per_step": int(n_ / steps_profiled),
              "avg_launch_us": round(us, 2), "timing": how, "avg_launch_us_event_pairs": round(ev_us, 2),
              "share_of_step": round(us * n_ / steps_profiled / 1e3 / ms, 3),
@@ -980,7 +997,8 @@ def main():
     if ar_ph is not None:
         ar = {"ms": round(ar_ph, 4), "GBps": round(payload / (ar_ph / 1e3) / 1e9, 1),
               "timing": f"phase events, median of {len(phase_samples)} replays, max over ranks",
-              "stash_phase_ms": round(stash_ph, 4) if stash_ph is not None else None}
+              "stash_phase_ms": round(stash_ph, 4) if stash_ph is not None else None,
+              "phase_step_ms": round(span_ph, 4) if span_ph is not None else None}
         if costs is not None:
             ar["roofline"] = plan_roofline(costs, ar_ph, peak)
             if rehearse:   # what the plan would take on G GPUs; measured here on ONE shared GPU
@@ -1041,8 +1059,67 @@ def main():
                           "timed": f"{10 * n_sw} back-to-back es_switch_context in a CUDA graph",
                           "share_of_step": round(us * len(local) / 1e3 / ms, 4)}
 
+    # ---- NEXT-1 on the measured path ----------------
+    # The same step with es_stash_fold_grads: each local EST folds its planned prefix into the
+    # fp32 partials at its switch.  What the paper's overlap shortens is the TAIL -- from the last
+    # local EST's stash (its backward done) to the aggregated gradients -- not the standalone
+    # step (which has no compute to hide the early folds behind).  Captured like the timed step,
+    # phase events, 5 replays, max over ranks; the outputs must equal the timed step's bits.
+    if next1_leg and G > 1 and sched not in es.PEER_SCHEDS:
+        line["next1"] = {"skipped": "NCCL transport rung: the incremental step is graph-tested on G = 1 and the "
+                                    "peer schedules only"}
+    elif next1_leg:
+        ref = [o.clone() for o in outs]
+        mk = [torch.cuda.Event(enable_timing=True, external=True) for _ in range(3)]
+
+        def inc_step():
+            mk[0].record(torch.cuda.current_stream())
+            for i, k in enumerate(local):
+                agg.switch(k)
+                agg.stash_fold(k, range(B), grads[k], es.ES_STASH_BORROW if i == len(local) - 1
+                               else es.ES_STASH_COPY)
+            mk[1].record(torch.cuda.current_stream())
+            agg.allreduce_many(range(B), outs)
+            mk[2].record(torch.cuda.current_stream())
+        for o in outs:
+            o.zero_()
+        with torch.cuda.stream(stream):
+            inc_step()                                   # eager once (lazy state), then captured
+        torch.cuda.synchronize()
+        g_inc = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g_inc, stream=stream):
+            inc_step()
+        samples = []
+        for _ in range(5):
+            with torch.cuda.stream(stream):
+                if flush is not None:
+                    flush.zero_()
+                    flush_sink.copy_(flush_words.amax())
+                g_inc.replay()
+            torch.cuda.synchronize()
+            samples.append((mk[0].elapsed_time(mk[2]), mk[1].elapsed_time(mk[2])))
+        same = all(torch.equal(a.view(torch.uint8) if a.dtype != torch.uint8 else a, b.view(torch.uint8))
+                   for a, b in zip(outs, ref))
+        same = bool(max_over_ranks(0 if same else 1) == 0)
+        inc_ms = max_over_ranks(statistics.median(x[0] for x in samples))
+        tail = max_over_ranks(statistics.median(x[1] for x in samples))
+        line["next1"] = {"step_ms": round(inc_ms, 4), "tail_ms": round(tail, 4),
+                         "copy_step_tail_ms": round(ar_ph, 4) if ar_ph is not None else None,
+                         "tail_ratio": round(tail / ar_ph, 4) if ar_ph else None,
+                         "bits_equal_timed_step": same,
+                         "what": "tail = last local EST's stash done -> es_allreduce_many done (phase events, "
+                                 "median of 5 replays, max over ranks); copy_step_tail_ms = the timed step's "
+                                 "allreduce phase"}
+        for o, r_ in zip(outs, ref):
+            o.copy_(r_)
+        torch.cuda.synchronize()
+        del ref, g_inc
+
     # ---- NEXT-3 (iii): ncclAllReduce (Ring, Simple, one channel) vs the canonical order --------
     line["ring_crosscheck"] = ring_crosscheck(args, name, N, G, rank, rehearse, dev, host)
+    # ---- the NVLink reference on this box -- ncclAllGather bus bandwidth --------
+    if G > 1 and not rehearse:
+        line["nvlink_busbw"] = allgather_busbw(G, dev, max_over_ranks)
 
     # ---- parity of the timed outputs against the oracle (+ cpu_baseline) ----
     if rank == 0:
@@ -1185,6 +1262,37 @@ def main():
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
+
+
+def allgather_busbw(G, dev, max_over_ranks, total_bytes=1 << 30, iters=10):
+    """ncclAllGather over the job's NCCL group of `total_bytes` (output size), bus bandwidth
+    (G-1)/G * bytes / t with t the max over ranks of the mean of `iters` CUDA-event-timed calls
+    after 3 warm-ups (nccl-tests' busBw definition).  Outside the timed region; the reference the
+    NVLink-bound fractions can be read against (B200_PROFILING.md quotes 725 GB/s all-reduce
+    busBW and a 770 GB/s peer copy per direction)."""
+    import torch
+    import torch.distributed as dist
+    try:
+        per = total_bytes // G // 4
+        x = torch.ones(per, dtype=torch.float32, device=dev)
+        y = torch.empty(per * G, dtype=torch.float32, device=dev)
+        for _ in range(3):
+            dist.all_gather_into_tensor(y, x)
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        dist.barrier()
+        a.record()
+        for _ in range(iters):
+            dist.all_gather_into_tensor(y, x)
+        b.record()
+        torch.cuda.synchronize()
+        ms = max_over_ranks(a.elapsed_time(b) / iters)
+        nbytes = per * G * 4
+        return {"op": "ncclAllGather (torch all_gather_into_tensor)", "bytes": nbytes, "ms": round(ms, 4),
+                "busbw_GBps": round((G - 1) / G * nbytes / (ms / 1e3) / 1e9, 1),
+                "algbw_GBps": round(nbytes / (ms / 1e3) / 1e9, 1), "timing": f"mean of {iters}, max over ranks"}
+    except Exception as e:   # a reference measurement; never fail the line over it
+        return {"error": f"{type(e).__name__}: {e}"}
 
 
 def ring_crosscheck(args, name, N, G, rank, rehearse, dev, host):

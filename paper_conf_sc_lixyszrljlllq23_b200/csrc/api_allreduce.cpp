@@ -100,7 +100,7 @@ struct BucketAddr {
   }
   unsigned char *part_at(int64_t id, int64_t lo) const {
     const es::Part &pt = b.parts[id];
-    return h->ws + p.parts_off + pt.off + (uint64_t)(lo - pt.lo) * 4;
+    return h->ws + p.parts_off + b.part_base + pt.off + (uint64_t)(lo - pt.lo) * 4;
   }
   // The segments of FOLD op f restricted to [lo, hi) (a sub-range of the op's range).
   void fold(const int64_t *f, int64_t lo, int64_t hi, FoldBatch *out) const {

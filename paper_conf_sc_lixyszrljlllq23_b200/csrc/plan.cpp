@@ -449,7 +449,10 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
   p->options = cfg->options;
 
   p->bp.resize(cfg->n_buckets);
-  uint64_t max_stage = 0, max_parts = 0, sum_peer_parts = 0, sum_pipe_flags = 0;
+  uint64_t max_stage = 0, max_parts = 0, sum_parts = 0, sum_peer_parts = 0, sum_pipe_flags = 0;
+  // CHAIN over a transport, tile-pipelined (chain_pipelined): all chain buckets of one
+  // es_allreduce_many are in flight together, so each owns its partial buffers
+  const bool chain_pipe = cfg->G > 1 && !(cfg->options & ES_OPT_PEER_ROUNDS);
   for (int32_t bi = 0; bi < cfg->n_buckets; ++bi) {
     BucketPlan &b = p->bp[bi];
     b.L = p->buckets[bi].numel;
@@ -478,6 +481,8 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
     if (p->options & ES_OPT_INCREMENTAL) plan_incremental(*p, &b);
     max_stage = std::max(max_stage, b.stage_bytes);
     max_parts = std::max(max_parts, b.part_bytes);
+    b.part_base = chain_pipe ? sum_parts : 0;
+    sum_parts += chain_pipe ? align256(b.part_bytes) : 0;
     b.peer_part_base = sum_peer_parts;   // buckets of one batched call run their rounds together
     sum_peer_parts += align256(b.peer_part_bytes);
     if (b.sched == ES_SCHED_PEER_CHAIN) {
@@ -528,7 +533,7 @@ es_status build_plan(const es_config *cfg, Plan *p, std::string *err, bool need_
   p->stage_off = total;
   total += max_stage;
   p->parts_off = total;
-  total += max_parts;
+  total += chain_pipe ? sum_parts : max_parts;
   if (p->options & ES_OPT_INCREMENTAL) {
     p->inc_off = align256(total);
     uint64_t o = 0;

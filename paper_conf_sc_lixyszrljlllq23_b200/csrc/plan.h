@@ -52,6 +52,8 @@ struct BucketPlan {
   uint64_t stage_bytes = 0;
   std::vector<Part> parts;
   uint64_t part_bytes = 0;
+  uint64_t part_base = 0;               // CHAIN: this bucket's base in the partials area (0 when the
+                                        //   round executor reuses one area bucket after bucket)
   uint64_t peer_part_bytes = 0;         // PEER_CHAIN: max over ranks of their outgoing partials
   uint64_t peer_part_base = 0;          // PEER_CHAIN: this bucket's base in the peer partials area
   int32_t chain_rounds = 0;             // PEER_CHAIN: R, the most segments of any chunk (all ranks)
@@ -92,7 +94,8 @@ struct Plan {
   uint64_t table_off = 0;               // swap table (n_state entries)
   uint64_t scratch_off = 0;             // 256 B of zeroed scratch (dropout grid counter)
   uint64_t stage_off = 0;               // exchange staging (max over buckets)
-  uint64_t parts_off = 0;               // chain partials (max over buckets)
+  uint64_t parts_off = 0;               // chain partials: max over buckets (round executor), or the
+                                        //   sum (tile-pipelined: every bucket of a call in flight at once)
   uint64_t flags_off = 0;               // PEER: G barrier flags (u64) written by peers + epoch counter
   uint64_t result_off = 0;              // PEER: per-bucket shard results (slot-block layout)
   uint64_t peer_parts_off = 0;          // PEER_CHAIN: partials read by the next GPU (uniform offset)

@@ -12,11 +12,19 @@ bytes read/written, DRAM throughput, occupancy, registers, stall summary).
 gpurun_out/full_{fold,stash}_<config>.ncu-rep and writes
 profiles/traffic_<config>_g<G>.json (dram read + write bytes per launch), which
 bench.py reports as roofline.traffic.
+`steady`: python scripts/ncu_summary.py steady <csv> <config> [G]  reads an
+`ncu --cache-control none --metrics gpu__time_duration.sum,dram__bytes_read.sum,
+dram__bytes_write.sum` list of the default command's graph replays and merges the
+per-launch mean DRAM bytes (dirty L2 lines of the previous kernel written back
+under this one, as in the timed step) into profiles/traffic_<config>_g<G>.json
+as <kernel>_dram_bytes_per_launch_steady; bench.py reports roofline.traffic_steady
+and frac_steady from them.
 """
 import collections
 import csv
 import io
 import json
+import os
 import subprocess
 import sys
 
@@ -108,5 +116,41 @@ def traffic(config, G="1"):
     print(path, d)
 
 
+def steady(path, config, G="1"):
+    rows = _csv_after_header(open(path).read())
+    per = collections.defaultdict(lambda: collections.defaultdict(float))   # (kernel, launch id) -> metric
+    for r in rows:
+        name = r["Kernel Name"]
+        k = next((k for k in ("k_fold", "k_stash") if k in name), None)
+        if k is None:
+            continue
+        m, v, u = r["Metric Name"], float(r["Metric Value"].replace(",", "")), r.get("Metric Unit", "")
+        if m.startswith("dram__bytes"):
+            v *= {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(u, 1)
+        elif u == "us":
+            v *= 1e3
+        elif u == "ms":
+            v *= 1e6
+        per[(k, r["ID"])][m] += v
+    tfile = f"profiles/traffic_{config}_g{G}.json"
+    d = json.load(open(tfile)) if os.path.exists(tfile) else {}
+    for k in ("k_fold", "k_stash"):
+        ls = [v for (kk, _), v in per.items() if kk == k]
+        if not ls:
+            continue
+        byt = sum(v["dram__bytes_read.sum"] + v["dram__bytes_write.sum"] for v in ls) / len(ls)
+        ns = sum(v["gpu__time_duration.sum"] for v in ls) / len(ls)
+        d[f"{k}_dram_bytes_per_launch_steady"] = int(round(byt))
+        d[f"{k}_steady_launches"] = len(ls)
+        d[f"{k}_steady_mean_us"] = round(ns / 1e3, 2)
+    d["source_steady"] = (f"{path}: ncu --cache-control none over the default command's CUDA-graph replays "
+                          "(after the eager warm-up), mean dram__bytes_read + write per launch: dirty L2 lines a "
+                          "kernel leaves are written back (and counted) under the next, as in the timed step")
+    with open(tfile, "w") as f:
+        json.dump(d, f, indent=1)
+        f.write("\n")
+    print(tfile, d)
+
+
 if __name__ == "__main__":
-    {"launches": launches, "full": full, "traffic": traffic}[sys.argv[1]](*sys.argv[2:])
+    {"launches": launches, "full": full, "traffic": traffic, "steady": steady}[sys.argv[1]](*sys.argv[2:])

@@ -6,8 +6,11 @@ the C ABI (es_plan_ops) and count, per rank: bytes received over NVLink
 shards) and HBM bytes (fold reads/writes, staging writes, gathers).  The step
 time bound is the slowest rank's max(HBM / 6.54 TB/s, NVLink / 0.77 TB/s);
 chain rounds are separated by barriers, so for CHAIN / PEER_CHAIN the bound
-is summed over rounds.  Stash bytes are excluded (allreduce
-only).  Writes profiles/r01_plan_roofline.md.
+is summed over rounds; the "pipelined" columns are the default executors
+(PEER_CHAIN: k_fold_pipe's per-tile flags; CHAIN over NCCL: chain_pipelined's
+tile wavefront on two streams), where every fold round and transfer overlaps
+and only the all-gather follows.  Stash bytes are excluded (SURVEY 8(d):
+allreduce only).  Writes profiles/r02_plan_roofline.md.
 
   python scripts/plan_roofline.py [out.md]
 """
@@ -19,7 +22,7 @@ sys.path.insert(0, ROOT)
 
 from paper_conf_sc_lixyszrljlllq23_b200 import es, workloads  # noqa: E402
 
-HBM = 6541.5e9          # MEASURED_PEAKS hbm_gbs (copy)
+HBM = 6455.6e9          # MEASURED_PEAKS hbm_gbs (copy), round 2
 NVL = 770e9             # B200_PROFILING.md measured peer copy per direction
 SCHEDS = {"direct": es.ES_SCHED_DIRECT, "chain": es.ES_SCHED_CHAIN, "peer": es.ES_SCHED_PEER,
           "peer_chain": es.ES_SCHED_PEER_CHAIN}
@@ -103,16 +106,18 @@ def bound_ms_pipelined(costs):
 
 
 def main(path):
-    rows = ["# Multi-GPU roofline of the exported plans (allreduce only; HBM 6.54 TB/s, NVLink 0.77 TB/s)\n",
+    rows = ["# Multi-GPU roofline of the exported plans (allreduce only; HBM 6.46 TB/s, NVLink 0.77 TB/s)\n",
             "Per phase (between groups / barriers), the slowest rank's max(HBM, NVLink) time, summed.\n",
             "peer_chain = rounds separated by barriers (ES_OPT_PEER_ROUNDS); pipelined = the default k_fold_pipe step "
             "(all rounds overlapped through per-tile flags, then the gather).\n",
             "peer push = ES_OPT_PEER_PUSH (the gather fused into the fold as NVLink stores): the same ingress bytes "
             "per rank move into the fold phase, so the bandwidth bound does not drop; what it removes is the "
             "gather's remote loads and one phase boundary (not modelled here).\n",
-            "| config | G | mapping | direct ms | chain ms | peer ms | peer push ms | peer_chain ms | "
-            "peer_chain pipelined ms | AUTO picks | max NVLink in / rank MB (direct, chain) |",
-            "|---|---|---|---|---|---|---|---|---|---|---|"]
+            "chain pipelined = CHAIN over NCCL as chain_pipelined runs it (tile wavefront: every round's folds "
+            "and transfers overlapped, then the all-gather group).\n",
+            "| config | G | mapping | direct ms | chain ms (rounds) | chain pipelined ms | peer ms | peer push ms | "
+            "peer_chain ms | peer_chain pipelined ms | AUTO picks | max NVLink in / rank MB (direct, chain) |",
+            "|---|---|---|---|---|---|---|---|---|---|---|---|"]
     cases = [("resnet50", G, "contiguous") for G in (2, 4, 8)] + [("vgg19", G, "contiguous") for G in (2, 4, 8)] + \
         [("bert_base", 8, "contiguous"), ("bert_base", 8, "round_robin")] + \
         [("swin_b", G, "contiguous") for G in (2, 4, 8)]
@@ -127,6 +132,7 @@ def main(path):
         nvd = max(sum(ph[1] for ph in r.values()) for r in res["direct"]) / 1e6
         nvc = max(sum(ph[1] for ph in r.values()) for r in res["chain"]) / 1e6
         rows.append(f"| {name} | {G} | {kind} | {bound_ms(res['direct']):.3f} | {bound_ms(res['chain']):.3f} | "
+                    f"{bound_ms_pipelined(res['chain']):.3f} | "
                     f"{bound_ms(res['peer']):.3f} | {bound_ms(res['peer_push']):.3f} | {bound_ms(res['peer_chain']):.3f} | "
                     f"{bound_ms_pipelined(res['peer_chain']):.3f} | {pick} | {nvd:.0f}, {nvc:.0f} |")
     text = "\n".join(rows) + "\n"
@@ -136,4 +142,4 @@ def main(path):
 
 
 if __name__ == "__main__":
-    main(sys.argv[1] if len(sys.argv) > 1 else os.path.join(ROOT, "profiles", "r01_plan_roofline.md"))
+    main(sys.argv[1] if len(sys.argv) > 1 else os.path.join(ROOT, "profiles", "r02_plan_roofline.md"))

@@ -10,12 +10,13 @@
 #    g1_bg's count is recorded separately.
 mkdir -p gpurun_out
 out=gpurun_out/sanitizer.txt; : > $out
-ALL="g1 g1_bg direct chain peer peer_chain_rounds peer_push"
+ALL="g1 g1_bg direct chain peer peer_chain_rounds peer_push chain_rounds chain_tiles direct_inc chain_inc peer_inc peer_chain_rounds_inc"
+INIT="g1 direct chain peer peer_chain_rounds peer_push chain_rounds chain_tiles direct_inc chain_inc peer_inc peer_chain_rounds_inc"
 for t in memcheck racecheck synccheck; do
   echo "== compute-sanitizer --tool $t python scripts/sanitize_step.py $ALL" >> $out
-  timeout 900 compute-sanitizer --tool $t python scripts/sanitize_step.py $ALL >> $out 2>&1
+  timeout 1500 compute-sanitizer --tool $t python scripts/sanitize_step.py $ALL >> $out 2>&1
 done
-echo "== compute-sanitizer --tool initcheck python scripts/sanitize_step.py g1 direct chain peer peer_chain_rounds peer_push" >> $out
-timeout 900 compute-sanitizer --tool initcheck python scripts/sanitize_step.py g1 direct chain peer peer_chain_rounds peer_push >> $out 2>&1
+echo "== compute-sanitizer --tool initcheck python scripts/sanitize_step.py $INIT" >> $out
+timeout 1500 compute-sanitizer --tool initcheck python scripts/sanitize_step.py $INIT >> $out 2>&1
 echo "== compute-sanitizer --tool initcheck python scripts/sanitize_step.py g1_bg   (TMA writes invisible to initcheck)" >> $out
-timeout 900 compute-sanitizer --tool initcheck python scripts/sanitize_step.py g1_bg 2>&1 | grep "ok\|SUMMARY" >> $out
+timeout 1500 compute-sanitizer --tool initcheck python scripts/sanitize_step.py g1_bg 2>&1 | grep "ok\|SUMMARY" >> $out

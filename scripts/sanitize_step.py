@@ -65,9 +65,12 @@ def g1(rng, options=0):
     inc.close()
 
 
-def multi(rng, sched, options=0):
+def multi(rng, sched, options=0, big=False):
     N, G, m = 6, 3, [0, 1, 2, 2, 0, 1]
     Ls, dts = [1003, 40, 9], ["f32", "bf16", "f32"]
+    if big:   # chunks above 2^20 elements: the tile-pipelined CHAIN cuts them into W = 2 tiles
+        N, G, m = 4, 2, [0, 0, 1, 1]
+        Ls, dts = [4 * (1 << 20) + 4 * 4096 + 3, 40], ["f32", "bf16"]
     xs = data(rng, N, Ls, dts)
     world = es.es_loopback_create(G)
     aggs = [Aggregator(N, G, g, m, list(zip(Ls, dts)), transport=es.ES_TRANSPORT_LOOPBACK, comm=world.value,
@@ -87,8 +90,11 @@ def multi(rng, sched, options=0):
             with torch.cuda.stream(streams[g]):
                 loc = aggs[g].local_ests
                 for i, k in enumerate(loc):
-                    aggs[g].stash_many(k, range(len(Ls)), devs[k],
-                                       es.ES_STASH_BORROW if i == len(loc) - 1 else es.ES_STASH_COPY)
+                    mode = es.ES_STASH_BORROW if i == len(loc) - 1 else es.ES_STASH_COPY
+                    if options & es.ES_OPT_INCREMENTAL:     # NEXT-1 at G > 1
+                        aggs[g].stash_fold(k, range(len(Ls)), devs[k], mode)
+                    else:
+                        aggs[g].stash_many(k, range(len(Ls)), devs[k], mode)
                 aggs[g].allreduce_many(range(len(Ls)), outs[g])
         except Exception as e:
             errs.append(e)
@@ -109,10 +115,16 @@ def multi(rng, sched, options=0):
 SCHEDS = {"direct": (es.ES_SCHED_DIRECT, 0), "chain": (es.ES_SCHED_CHAIN, 0), "peer": (es.ES_SCHED_PEER, 0),
           "peer_chain": (es.ES_SCHED_PEER_CHAIN, 0),
           "peer_chain_rounds": (es.ES_SCHED_PEER_CHAIN, es.ES_OPT_PEER_ROUNDS),
-          "peer_push": (es.ES_SCHED_PEER, es.ES_OPT_PEER_PUSH)}
+          "peer_push": (es.ES_SCHED_PEER, es.ES_OPT_PEER_PUSH),
+          "chain_rounds": (es.ES_SCHED_CHAIN, es.ES_OPT_PEER_ROUNDS),
+          "chain_tiles": (es.ES_SCHED_CHAIN, 0, True),
+          "direct_inc": (es.ES_SCHED_DIRECT, es.ES_OPT_INCREMENTAL),
+          "chain_inc": (es.ES_SCHED_CHAIN, es.ES_OPT_INCREMENTAL),
+          "peer_inc": (es.ES_SCHED_PEER, es.ES_OPT_INCREMENTAL),
+          "peer_chain_rounds_inc": (es.ES_SCHED_PEER_CHAIN, es.ES_OPT_PEER_ROUNDS | es.ES_OPT_INCREMENTAL)}
 
 if __name__ == "__main__":
-    # argv: which parts to run (default: all): g1 g1_bg direct chain peer peer_chain peer_chain_rounds peer_push
+    # argv: which parts to run (default: all): g1 g1_bg and the SCHEDS keys
     parts = sys.argv[1:] or ["g1", "g1_bg"] + list(SCHEDS)
     rng = np.random.default_rng(0)
     for part in parts:

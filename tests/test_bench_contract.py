@@ -60,3 +60,7 @@ def test_main_arm_line_keys():
     assert d["gpu_launches"] > 0 and {"sm_mhz", "sm_max_mhz", "reasons"} <= set(d["clocks"])
     assert d["parity"]["mismatched_words"] == 0 and d["parity"]["full_output_mismatched_words"] == 0
     assert d["parity"]["sha256_equal"] is True and d["switch"]["us_per_switch"] > 0
+    ar = d["allreduce_only"]
+    assert 0 < ar["ms"] <= ar["phase_step_ms"] and ar["ms"] <= d["ms_per_step"]
+    n1 = d["next1"]                       # NEXT-1 leg: same bits, tail measured beside the copy step's
+    assert n1["bits_equal_timed_step"] is True and n1["tail_ms"] > 0 and n1["copy_step_tail_ms"] > 0

@@ -39,3 +39,5 @@ def test_bench_two_ranks_same_gpu_matches_g1():
         assert g2["parity"]["mismatched_words"] == 0
         assert g2["output_sha256"] == g1["output_sha256"], sched
         assert g2["e2e"]["value"] > 0
+        assert g2["next1"]["bits_equal_timed_step"] is True          # NEXT-1 at G = 2 on the bench path
+        assert 0 < g2["allreduce_only"]["ms"] <= g2["ms_per_step"]

@@ -22,30 +22,32 @@ pytestmark = pytest.mark.gpu
 
 
 def test_export_refuses_partially_folded_slot():
+    """NEXT-1 (es_stash_fold_grads) at G = 1, N = 4: EST 0 opens chunk 3's partial (its
+    sequence 0, 1, 2, 3 starts there), EST 1 folds into chunks 3 and 0, EST 2 into 3, 0, 1;
+    EST 3, the last local EST, folds nothing and its COPY slot holds its whole gradient."""
     N, L = 4, 100003
     agg = Aggregator(N, 1, 0, [0] * N, [(L, "f32")], options=es.ES_OPT_INCREMENTAL)
     rng = np.random.default_rng(5)
     xs = [(rng.standard_normal(L) * 1e-2).astype(np.float32) for _ in range(N)]
     d = [to_dev(x) for x in xs]
-    agg.stash_fold(0, [0], [d[0]], es.ES_STASH_COPY)          # EST 0: whole gradient stashed
-    agg.stash_fold(1, [0], [d[1]], es.ES_STASH_COPY)          # EST 1: chunk 0 folded, rest stashed
-    blob0 = agg.export_context(0)
-    with pytest.raises(es.EsError) as ei:
-        agg.export_context(1)
-    assert ei.value.status == es.ES_ESTATE
-    with pytest.raises(es.EsError) as ei:                     # importing would bypass the partials
-        agg.import_context(0, blob0)
-    assert ei.value.status == es.ES_ESTATE
+    agg.stash_fold(0, [0], [d[0]], es.ES_STASH_COPY)
+    agg.stash_fold(1, [0], [d[1]], es.ES_STASH_COPY)
+    for e in (0, 1):                                          # partly folded: the slot is not the gradient
+        with pytest.raises(es.EsError) as ei:
+            agg.export_context(e)
+        assert ei.value.status == es.ES_ESTATE
     agg.stash_fold(2, [0], [d[2]], es.ES_STASH_COPY)
-    agg.stash_fold(3, [0], [d[3]], es.ES_STASH_BORROW)        # BORROW: the live buffer is whole
-    agg.export_context(3)
+    agg.stash_fold(3, [0], [d[3]], es.ES_STASH_COPY)
+    blob3 = agg.export_context(3)                             # nothing folded: exportable
+    with pytest.raises(es.EsError) as ei:                     # importing would bypass the partials
+        agg.import_context(3, blob3)
+    assert ei.value.status == es.ES_ESTATE
     out = agg.new_out(0)
     agg.allreduce(0, out)                                     # the refused calls changed nothing
     torch.cuda.synchronize()
     assert_bits_equal(from_dev(out), oracle.reduce(xs, "f32"), "incremental after refused export")
-    # the exported EST 0 context is its gradient
-    blob = np.frombuffer(blob0, dtype=np.uint8)
-    assert blob[-L * 4:].tobytes() == xs[0].tobytes()        # no context buffers: the bucket ends the blob
+    blob = np.frombuffer(blob3, dtype=np.uint8)
+    assert blob[-L * 4:].tobytes() == xs[3].tobytes()        # no context buffers: the bucket ends the blob
     agg.close()
 
 
