@@ -1,4 +1,4 @@
-"""The committed G = 1 bench lines (profiles/r01_bench_<config>_g1.json) keep the bench contract:
+"""The committed G = 1 bench lines (profiles/r02_bench_<config>_g1.json) keep the bench contract:
 BASELINE's metric, the roofline / cpu_baseline / e2e / clocks objects, bit-exact parity, and the
 tables in DESIGN.md and README.md are the ones scripts/bench_table.py generates from them."""
 import json
@@ -13,7 +13,7 @@ CONFIGS = ["tiny", "resnet50", "vgg19", "bert_base", "swin_b"]
 
 
 def _line(name):
-    with open(os.path.join(ROOT, "profiles", f"r01_bench_{name}_g1.json")) as f:
+    with open(os.path.join(ROOT, "profiles", f"r02_bench_{name}_g1.json")) as f:
         return json.load(f)
 
 
@@ -39,8 +39,11 @@ def test_committed_line_keeps_the_contract(name):
     assert not set(c["reasons"]) & {"hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown"}
     p = d["parity"]
     assert p["mismatched_words"] == 0 and p["checked_elements"] > 0
-    if p.get("full_output_checked"):
-        assert p["full_output_mismatched_words"] == 0 and p["sha256_equal"] is True
+    assert p["full_output_checked"] and p["full_output_mismatched_words"] == 0 and p["sha256_equal"] is True
+    ar = d["allreduce_only"]
+    assert 0 < ar["ms"] <= ar["phase_step_ms"] and ar["ms"] <= d["ms_per_step"]
+    n1 = d["next1"]
+    assert n1["bits_equal_timed_step"] is True and 0 < n1["tail_ms"] and 0 < n1["copy_step_tail_ms"]
 
 
 def test_output_hash_is_the_oracles_where_checked_whole():
