@@ -174,12 +174,14 @@ class Clocks:
 
 class NvLink:
     """Per-GPU NVLink facts and data counters through NVML (nvidia_ml_py).
-    Data counters: NVML_FI_DEV_NVLINK_THROUGHPUT_DATA_TX/RX (KiB, per link,
-    payload only), summed over the active links."""
-    FI_TX, FI_RX = 138, 139
+    Data counters, summed over the active links: NVML_FI_DEV_NVLINK_COUNT_XMIT/RCV_BYTES
+    (fields 202/204, bytes, NVLink 5 / Blackwell) if the driver supports them, else
+    NVML_FI_DEV_NVLINK_THROUGHPUT_DATA_TX/RX (fields 138/139, KiB of payload)."""
+    SOURCES = (((202, 204), 1, "NVML NVLINK_COUNT_XMIT/RCV_BYTES (bytes), active links"),
+               ((138, 139), 1024, "NVML NVLINK_THROUGHPUT_DATA_TX/RX (KiB, payload), active links"))
 
     def __init__(self, uuid):
-        self.ok, self.why, self.links = False, None, []
+        self.ok, self.why, self.links, self.source = False, None, [], None
         try:
             import pynvml
             pynvml.nvmlInit()
@@ -197,26 +199,26 @@ class NvLink:
             self.why = f"NVML unavailable: {e}"
 
     def read(self):
-        """(tx_bytes, rx_bytes) summed over active links, or None."""
+        """(tx_bytes, rx_bytes) summed over active links, or None (self.why says why)."""
         if not self.ok or not self.links:
             return None
-        try:
-            fields = [(self.FI_TX, l) for l in self.links] + [(self.FI_RX, l) for l in self.links]
-            vals = self.nv.nvmlDeviceGetFieldValues(self.h, fields)
-            tx = rx = 0
-            for i, v in enumerate(vals):
-                if v.nvmlReturn != 0:
-                    self.why = f"NVML field {fields[i]} returned {v.nvmlReturn}"
-                    return None
-                kib = int(v.value.ullVal)
-                if i < len(self.links):
-                    tx += kib
-                else:
-                    rx += kib
-            return tx * 1024, rx * 1024
-        except Exception as e:
-            self.why = f"NVML field read failed: {e}"
-            return None
+        errs = []
+        for (ftx, frx), scale, name in self.SOURCES:
+            try:
+                fields = [(ftx, l) for l in self.links] + [(frx, l) for l in self.links]
+                vals = self.nv.nvmlDeviceGetFieldValues(self.h, fields)
+                bad = [(fields[i], v.nvmlReturn) for i, v in enumerate(vals) if v.nvmlReturn != 0]
+                if bad:
+                    errs.append(f"field {bad[0][0]} returned {bad[0][1]}")
+                    continue
+                tx = sum(int(v.value.ullVal) for v in vals[:len(self.links)])
+                rx = sum(int(v.value.ullVal) for v in vals[len(self.links):])
+                self.source = name
+                return tx * scale, rx * scale
+            except Exception as e:
+                errs.append(f"read failed: {e}")
+        self.why = "NVML NVLink data counters unavailable: " + "; ".join(errs)
+        return None
 
 
 # ---- the multi-GPU roofline of the exported plan (SURVEY 8(d)) ---------------------------------
@@ -1028,7 +1030,7 @@ def main():
         per_rank = gather_objects(mine)
         plan_nv = [{"in_bytes": c["nvl_in"], "out_bytes": c["nvl_out"]} for c in costs]
         line["nvlink_counters"] = {"per_rank": per_rank, "plan_per_rank": plan_nv,
-                                   "source": "NVML NVLINK_THROUGHPUT_DATA_TX/RX (KiB, payload), active links",
+                                   "source": nvl.source or nvl.why,
                                    **({"note": "rehearsal: every rank on one GPU, peer traffic stays in HBM"}
                                       if rehearse else {})}
 

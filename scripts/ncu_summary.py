@@ -98,18 +98,18 @@ def _bytes(v, unit):
     return int(round(float(v.replace(",", "")) * scale))
 
 
-def traffic(config, G="1"):
-    d = {}
+def traffic(config, G="1", rnd="r01"):
+    path = f"profiles/traffic_{config}_g{G}.json"
+    d = json.load(open(path)) if os.path.exists(path) else {}     # keeps the *_steady entries
     for kname, tag in (("k_fold", "fold"), ("k_stash", "stash")):
         rep = f"gpurun_out/full_{tag}_{config}.ncu-rep"
         hdr, units, rows = _raw(rep)
         r = rows[0]
         rd, wr = hdr.index("dram__bytes_read.sum"), hdr.index("dram__bytes_write.sum")
         d[f"{kname}_dram_bytes_per_launch"] = _bytes(r[rd], units[rd]) + _bytes(r[wr], units[wr])
-    d["source"] = (f"ncu --set full (profiles/r01_k_fold_full_{config}.md, r01_k_stash_full_{config}.md): "
+    d["source"] = (f"ncu --set full (profiles/{rnd}_k_fold_full_{config}.md, {rnd}_k_stash_full_{config}.md): "
                    "dram__bytes_read.sum + dram__bytes_write.sum per launch, cold cache; writes still dirty "
                    "in L2 at kernel end are not counted")
-    path = f"profiles/traffic_{config}_g{G}.json"
     with open(path, "w") as f:
         json.dump(d, f, indent=1)
         f.write("\n")
