@@ -24,7 +24,7 @@ def _port():
     return p
 
 
-def _worker(rank, G, port, sched_name, q):
+def _worker(rank, G, port, sched_name, q, options=0):
     import sys
     sys.path.insert(0, ROOT)
     sys.path.insert(0, os.path.join(ROOT, "tests"))
@@ -45,7 +45,7 @@ def _worker(rank, G, port, sched_name, q):
         m = workloads.mapping(N, G, "contiguous")
         Ls, dts = [200003, 4099, 17], ["f32", "bf16", "f32"]
         agg = Aggregator(N, G, rank, m, list(zip(Ls, dts)), transport=es.ES_TRANSPORT_NCCL, comm=nccl_comm_ptr(),
-                         sched=sched, device=dev)
+                         sched=sched, device=dev, options=options)
         if sched in es.PEER_SCHEDS:
             agg.peer_connect()
         ok = True
@@ -57,8 +57,11 @@ def _worker(rank, G, port, sched_name, q):
                 xs.append(row if d == "f32" else [oracle.f32_to_bf16_bits(x) for x in row])
             devs = {k: [to_dev(xs[b][k]).to(dev) for b in range(3)] for k in agg.local_ests}
             for i, k in enumerate(agg.local_ests):
-                agg.stash_many(k, range(3), devs[k],
-                               es.ES_STASH_BORROW if i == len(agg.local_ests) - 1 else es.ES_STASH_COPY)
+                mode = es.ES_STASH_BORROW if i == len(agg.local_ests) - 1 else es.ES_STASH_COPY
+                if options & es.ES_OPT_INCREMENTAL:          # NEXT-1 across real GPUs
+                    agg.stash_fold(k, range(3), devs[k], mode)
+                else:
+                    agg.stash_many(k, range(3), devs[k], mode)
             outs = [agg.new_out(b) for b in range(3)]
             agg.allreduce_many(range(3), outs)
             torch.cuda.synchronize()
@@ -75,11 +78,14 @@ def _worker(rank, G, port, sched_name, q):
 @pytest.mark.parametrize("G", [g for g in (2, 4, 8) if g <= NGPU] or [2])
 @pytest.mark.parametrize("sched_name", ["ES_SCHED_DIRECT", "ES_SCHED_CHAIN", "ES_SCHED_AUTO", "ES_SCHED_PEER",
                                         "ES_SCHED_PEER_CHAIN"])
-def test_nccl_and_peer_paths_on_real_gpus(G, sched_name):
+@pytest.mark.parametrize("options", [0, 1, 2], ids=["default", "incremental", "rounds"])
+def test_nccl_and_peer_paths_on_real_gpus(G, sched_name, options):
+    """options: 0 (tile-pipelined CHAIN / PEER_CHAIN), 1 = ES_OPT_INCREMENTAL (NEXT-1),
+    2 = ES_OPT_PEER_ROUNDS (the round executors)."""
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _port()
-    ps = [ctx.Process(target=_worker, args=(r, G, port, sched_name, q)) for r in range(G)]
+    ps = [ctx.Process(target=_worker, args=(r, G, port, sched_name, q, options)) for r in range(G)]
     for p in ps:
         p.start()
     for p in ps:

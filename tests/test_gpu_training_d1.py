@@ -65,12 +65,14 @@ def flat_grad(params):
 class Rank:
     """One rank (GPU) of the job: a parameter replica and an aggregator."""
 
-    def __init__(self, G, r, mapping, world, chunk_align=16):
+    def __init__(self, G, r, mapping, world, chunk_align=16, incremental=False):
         self.params = make_model()
         self.n = sum(p.numel() for p in self.params)
+        self.incremental = incremental
         self.agg = Aggregator(N, G, r, mapping, [(self.n, "f32")], state_nbytes=[16], chunk_align=chunk_align,
                               transport=es.ES_TRANSPORT_LOOPBACK if G > 1 else es.ES_TRANSPORT_NONE,
-                              comm=world.value if G > 1 else None)
+                              comm=world.value if G > 1 else None,
+                              options=es.ES_OPT_INCREMENTAL if incremental else 0)
         self.live = [torch.zeros(16, dtype=torch.uint8, device="cuda")]
         self.agg.register_state(self.live)
         self.stream = torch.cuda.Stream()
@@ -95,7 +97,11 @@ class Rank:
             loss.backward()
             g = flat_grad(self.params).contiguous()
             bufs.append(g)
-            self.agg.stash(k, 0, g, es.ES_STASH_BORROW if i == len(loc) - 1 else es.ES_STASH_COPY)
+            mode = es.ES_STASH_BORROW if i == len(loc) - 1 else es.ES_STASH_COPY
+            if self.incremental:                                 # NEXT-1: fold at the switch
+                self.agg.stash_fold(k, [0], [g], mode)
+            else:
+                self.agg.stash(k, 0, g, mode)
         avg = torch.empty(self.n, device="cuda")
         self.agg.allreduce(0, avg)
         with torch.no_grad():                                    # replicated SGD update
@@ -126,14 +132,14 @@ def run_stage(ranks, steps):
         raise errs[0]
 
 
-def new_stage(G, mapping, chunk_align=16):
+def new_stage(G, mapping, chunk_align=16, incremental=False):
     world = es.es_loopback_create(G) if G > 1 else None
-    ranks = [Rank(G, r, mapping, world, chunk_align) for r in range(G)]
+    ranks = [Rank(G, r, mapping, world, chunk_align, incremental) for r in range(G)]
     return world, ranks
 
 
-def train(G, mapping, steps, chunk_align=16):
-    world, ranks = new_stage(G, mapping, chunk_align)
+def train(G, mapping, steps, chunk_align=16, incremental=False):
+    world, ranks = new_stage(G, mapping, chunk_align, incremental)
     for r in ranks:
         r.init_contexts()
     run_stage(ranks, steps)
@@ -178,6 +184,10 @@ def test_training_is_bitwise_identical_across_g_and_elastic_change():
         assert all(torch.equal(a, b) for a, b in zip(bits(r.params), ref)), "elastic run diverged"
         r.close()
     es.es_loopback_destroy(world)
+    # NEXT-1 (incremental fold at every switch) trains to the same bits on G = 1 and G = 2
+    for G, mapping in [(1, [0, 0, 0, 0]), (2, [0, 0, 1, 1]), (2, [1, 0, 1, 0])]:
+        for rank_params in train(G, mapping, steps, incremental=True):
+            assert all(torch.equal(a, b) for a, b in zip(bits(rank_params), ref)), ("incremental", G, mapping)
     # negative control (R8): another persisted layout -- here the chunk
     # alignment -- changes the aggregation order and therefore the trained bits
     other = bits(train(1, [0, 0, 0, 0], steps, chunk_align=1024)[0])
