@@ -114,6 +114,12 @@ es_status es_init(const es_config *cfg, void *workspace, size_t workspace_bytes,
     if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
       return set_err(ES_ECUDA, "cudaEventCreate failed");
   for (uint64_t n : h->plan.state_nbytes) h->max_state = std::max<uint64_t>(h->max_state, n);
+  // The tile-pipelined CHAIN's side stream, created here rather than at its first use, which may
+  // be inside a CUDA-graph capture.
+  for (const es::BucketPlan &b : h->plan.bp)
+    if (b.sched == ES_SCHED_CHAIN && !(h->plan.options & ES_OPT_PEER_ROUNDS) && !h->side &&
+        cudaStreamCreateWithFlags(&h->side, cudaStreamNonBlocking) != cudaSuccess)
+      return set_err(ES_ECUDA, "cudaStreamCreate failed");
   {
     // Zero the scratch words and the peer flags + epoch counter on a private
     // stream and wait for it: peers may write these flags as soon as they hold

@@ -154,3 +154,25 @@ def reduce_loopback(xs_per_bucket, G, mapping, sched=es.ES_SCHED_AUTO, A=16, bor
         a.close()
     es.es_loopback_destroy(world)
     return res
+
+
+def check_whole_output(what, outs, fetch, buckets, N, win=1 << 21):
+    """The WHOLE reduced bucket set against the oracle (plain definition, windows of `win`
+    elements on a thread pool: the C oracle releases the GIL), bit-exact.  fetch(k, b) -> EST
+    k's bucket b as a host array."""
+    import concurrent.futures as cf
+    import os
+
+    import oracle
+    host = [[fetch(k, b) for k in range(N)] for b in range(len(buckets))]
+    got = [from_dev(o) for o in outs]
+    jobs = [(b, s, min(win, L - s)) for b, (L, _) in enumerate(buckets) for s in range(0, L, win)]
+
+    def run(j):
+        b, s, n = j
+        L, d = buckets[b]
+        want = oracle.reduce([host[b][k][s:s + n] for k in range(N)], d, L=L, first=s)
+        assert_bits_equal(got[b][s:s + n], want, f"{what} b={b} s={s}")
+        return n
+    with cf.ThreadPoolExecutor(max_workers=len(os.sched_getaffinity(0))) as ex:
+        assert sum(ex.map(run, jobs)) == sum(L for L, _ in buckets)

@@ -308,10 +308,17 @@ def test_loopback_multi_step_reuse(sched, batched):
 
 # ---- full size, in the bench launch configuration: sampled windows -----------------------------
 
-def _bench_step(agg, local, grads, outs):
+def _bench_step(agg, local, grads, outs, incremental=False):
     """Exactly bench.py's step: switch-in, fused stash+switch per EST, the last
-    local EST borrowed, one batched allreduce."""
+    local EST borrowed, one batched allreduce (incremental: bench.py's NEXT-1
+    leg -- switch, es_stash_fold_grads per EST)."""
     B = len(outs)
+    if incremental:
+        for i, k in enumerate(local):
+            agg.switch(k)
+            agg.stash_fold(k, range(B), grads[k], es.ES_STASH_BORROW if i == len(local) - 1 else es.ES_STASH_COPY)
+        agg.allreduce_many(range(B), outs)
+        return
     agg.switch(local[0])
     for i, k in enumerate(local):
         if i == len(local) - 1:
@@ -336,10 +343,12 @@ def _check_sampled(name, outs, fetch, buckets, N, seed=0):
 
 
 @pytest.mark.parametrize("name", ["tiny", "resnet50", "vgg19", "bert_base", "swin_b"])
-def test_full_size_sampled_parity(name):
+def test_full_size_whole_output_parity(name):
     """BASELINE.json's full sizes at G=1, in bench.py's launch configuration
-    (CUDA graph of the fused step, replayed), checked on sampled windows that
-    include chunk boundaries and the ragged end, plus a property at any size."""
+    (CUDA graph of the fused step, replayed): the WHOLE output against the
+    oracle (all host cores), plus sampled windows at chunk boundaries and the
+    ragged end, plus a property at any size."""
+    from gpu_util import check_whole_output
     cfg = workloads.config(name)
     N = cfg["N"]
     from gpu_util import Aggregator, from_dev
@@ -366,6 +375,7 @@ def test_full_size_sampled_parity(name):
     torch.cuda.synchronize()
     agg.sync()
     _check_sampled(name, outs, lambda k, b, st, n: from_dev(grads[k][b][st:st + n]), buckets, N)
+    check_whole_output(name, outs, lambda k, b: from_dev(grads[k][b]), buckets, N)
     for b in range(len(buckets)):         # property at any size: finite, |out| <= max_k |x_k| (+ rounding)
         o = outs[b].float()
         mx = grads[0][b].float().abs()
@@ -375,12 +385,15 @@ def test_full_size_sampled_parity(name):
     agg.close()
 
 
-@pytest.mark.parametrize("name,G,kind", [("resnet50", 8, "contiguous"), ("resnet50", 2, "contiguous"),
-                                         ("bert_base", 8, "contiguous"), ("bert_base", 8, "round_robin"),
-                                         ("vgg19", 4, "contiguous")])
-def test_full_size_multi_rank_loopback(name, G, kind):
+@pytest.mark.parametrize("name,G,kind,inc", [("resnet50", 8, "contiguous", False), ("resnet50", 2, "contiguous", False),
+                                             ("bert_base", 8, "contiguous", False),
+                                             ("bert_base", 8, "round_robin", False),
+                                             ("vgg19", 4, "contiguous", False), ("swin_b", 4, "contiguous", True),
+                                             ("bert_base", 8, "contiguous", True)])
+def test_full_size_multi_rank_loopback(name, G, kind, inc):
     """The configs' G > 1 shapes at full size over the loopback transport
-    (all G ranks on this GPU): every rank holds the oracle's bits."""
+    (all G ranks on this GPU; AUTO: tile-pipelined CHAIN / DIRECT): every rank
+    holds the oracle's bits (rank 0's whole output checked).  inc: NEXT-1."""
     import threading
     cfg = workloads.config(name)
     N = cfg["N"]
@@ -389,7 +402,8 @@ def test_full_size_multi_rank_loopback(name, G, kind):
     m = workloads.mapping(N, G, kind)
     world = es.es_loopback_create(G)
     aggs = [Aggregator(N, G, r, m, buckets, state_nbytes=workloads.state_nbytes(),
-                       transport=es.ES_TRANSPORT_LOOPBACK, comm=world.value) for r in range(G)]
+                       transport=es.ES_TRANSPORT_LOOPBACK, comm=world.value,
+                       options=es.ES_OPT_INCREMENTAL if inc else 0) for r in range(G)]
     lives = []
     for r, a in enumerate(aggs):
         live = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in workloads.state_nbytes()]
@@ -407,7 +421,7 @@ def test_full_size_multi_rank_loopback(name, G, kind):
     def run(r):
         try:
             with torch.cuda.stream(streams[r]):
-                _bench_step(aggs[r], aggs[r].local_ests, grads, outs[r])
+                _bench_step(aggs[r], aggs[r].local_ests, grads, outs[r], incremental=inc)
         except Exception as e:
             errs.append(e)
     ts = [threading.Thread(target=run, args=(r,)) for r in range(G)]
@@ -419,6 +433,8 @@ def test_full_size_multi_rank_loopback(name, G, kind):
     fetch = lambda k, b, st, n: from_dev(grads[k][b][st:st + n])  # noqa: E731
     for r in (0, G - 1):
         _check_sampled(f"{name} G={G} {kind} rank {r}", outs[r], fetch, buckets, N, seed=r)
+    from gpu_util import check_whole_output
+    check_whole_output(f"{name} G={G} {kind} rank 0", outs[0], lambda k, b: from_dev(grads[k][b]), buckets, N)
     for r in range(1, G):                 # every rank holds the same bits
         for b in range(len(buckets)):
             iv = torch.int16 if outs[r][b].dtype == torch.bfloat16 else torch.int32
