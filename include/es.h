@@ -222,8 +222,9 @@ es_status es_workspace_bytes(const es_config *cfg, size_t *bytes);
 /* Creates a handle.  `workspace` is caller-owned device memory of at least
  * es_workspace_bytes() bytes, 256-byte aligned, outliving the handle; the
  * library never calls cudaMalloc (PyTorch stays the only device allocator)
- * and owns only host metadata, CUDA events and, for G > 1, its planner
- * tables.  The bucket plan (chunk table, shards, schedule, exchange ops) is
+ * and owns only host metadata, CUDA events, for G > 1 its planner tables
+ * and, when a CHAIN bucket runs tile-pipelined over a transport, one
+ * non-blocking side stream (created here, destroyed by es_destroy).  The bucket plan (chunk table, shards, schedule, exchange ops) is
  * computed here once and never rebuilt (D1).  Elastic change of
  * G or of the mapping = es_destroy + es_init with the same N, layout and A
  * (P:619-624).  cfg and its arrays are copied. */
