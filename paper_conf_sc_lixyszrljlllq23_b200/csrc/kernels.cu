@@ -295,8 +295,12 @@ __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const 
     cnt = g.m;
   }
   const int64_t boff = t * T::kSize;
-  int done = 0;
-  if (g.part_in) {                                            // R14: continue a chain partial
+  // R3 / R14: the accumulator opens with the first contribution, or continues a chain partial.
+  // The opening contribution is loaded in the first batch together with the next ones (one memory
+  // round trip for up to kBatch sources, not an extra dependent one first); the adds keep the
+  // canonical order.
+  bool open = g.part_in == nullptr;
+  if (!open) {
     const float *pp = g.part_in + t;
 #pragma unroll
     for (int q = 0; q < V / 4; ++q) {
@@ -304,14 +308,8 @@ __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const 
       acc[4 * q + 0] = __int_as_float(w.x); acc[4 * q + 1] = __int_as_float(w.y);
       acc[4 * q + 2] = __int_as_float(w.z); acc[4 * q + 3] = __int_as_float(w.w);
     }
-  } else {                                                    // R3: start from the first contribution
-    int4 w = ld_stream(reinterpret_cast<const char *>(src[idx]) + boff);
-    T::widen(w, acc);
-#pragma unroll
-    for (int e = 0; e < V; ++e) acc[e] = prep<COMPAT>(acc[e], compat, r, fN);
-    idx = (idx + 1 == cnt) ? 0 : idx + 1;
-    done = 1;
   }
+  int done = 0;
   while (done < cnt) {
     const int nb = min(kBatch, cnt - done);
     int4 buf[kBatch];
@@ -328,10 +326,16 @@ __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const 
       if (b < nb) {
         float x[V];
         T::widen(buf[b], x);
+        if (b == 0 && open) {                                 // R3: start from the first contribution
 #pragma unroll
-        for (int e = 0; e < V; ++e) acc[e] = add_step<COMPAT>(acc[e], prep<COMPAT>(x[e], compat, r, fN), compat);
+          for (int e = 0; e < V; ++e) acc[e] = prep<COMPAT>(x[e], compat, r, fN);
+        } else {
+#pragma unroll
+          for (int e = 0; e < V; ++e) acc[e] = add_step<COMPAT>(acc[e], prep<COMPAT>(x[e], compat, r, fN), compat);
+        }
       }
     }
+    open = false;
     idx = k;
     done += nb;
   }
@@ -366,8 +370,18 @@ __device__ __forceinline__ float fold_scalar(const FoldSeg &g, const void *const
   return s;
 }
 
+// Build-time register bound of k_fold (ES_FOLD_MINB resident 256-thread blocks per SM; 0 = none).
+#ifndef ES_FOLD_MINB
+#define ES_FOLD_MINB 0
+#endif
+#if ES_FOLD_MINB > 0
+#define ES_FOLD_LB __launch_bounds__(256, ES_FOLD_MINB)
+#else
+#define ES_FOLD_LB __launch_bounds__(256)
+#endif
+
 template <typename T, int MAXSEG, int MAXSRC, bool COMPAT>
-__global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams<MAXSEG, MAXSRC> p) {
+__global__ void ES_FOLD_LB k_fold(const __grid_constant__ FoldParams<MAXSEG, MAXSRC> p) {
   constexpr int V = T::kVec;
   // post-scale unless a pre-scale variant already applied 1/N (R5 vs NEXT-3)
   const bool post = !COMPAT || !(p.compat & (kPreDiv | kPreMul));
