@@ -296,10 +296,13 @@ __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const 
   }
   const int64_t boff = t * T::kSize;
   // R3 / R14: the accumulator opens with the first contribution, or continues a chain partial.
-  // The opening contribution is loaded in the first batch together with the next ones (one memory
-  // round trip for up to kBatch sources, not an extra dependent one first); the adds keep the
-  // canonical order.
+  // bf16 (MERGE): the opening contribution is loaded in the first batch together with the next
+  // ones -- one memory round trip for up to kBatch sources instead of a dependent one first;
+  // measured +2.8 % on BERT's fold (profiles/r02_fold_variants.md).  fp32 keeps the separate
+  // opening load, which measured 1.9-2.1 % faster there (Swin-B, VGG-19).  Same adds, same order.
+  constexpr bool MERGE = T::kSize == 2;
   bool open = g.part_in == nullptr;
+  int done = 0;
   if (!open) {
     const float *pp = g.part_in + t;
 #pragma unroll
@@ -308,8 +311,15 @@ __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const 
       acc[4 * q + 0] = __int_as_float(w.x); acc[4 * q + 1] = __int_as_float(w.y);
       acc[4 * q + 2] = __int_as_float(w.z); acc[4 * q + 3] = __int_as_float(w.w);
     }
+  } else if (!MERGE) {
+    int4 w = ld_stream(reinterpret_cast<const char *>(src[idx]) + boff);
+    T::widen(w, acc);
+#pragma unroll
+    for (int e = 0; e < V; ++e) acc[e] = prep<COMPAT>(acc[e], compat, r, fN);
+    idx = (idx + 1 == cnt) ? 0 : idx + 1;
+    done = 1;
+    open = false;
   }
-  int done = 0;
   while (done < cnt) {
     const int nb = min(kBatch, cnt - done);
     int4 buf[kBatch];
@@ -326,7 +336,7 @@ __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const 
       if (b < nb) {
         float x[V];
         T::widen(buf[b], x);
-        if (b == 0 && open) {                                 // R3: start from the first contribution
+        if (MERGE && b == 0 && open) {                        // R3: start from the first contribution
 #pragma unroll
           for (int e = 0; e < V; ++e) acc[e] = prep<COMPAT>(x[e], compat, r, fN);
         } else {
@@ -370,18 +380,8 @@ __device__ __forceinline__ float fold_scalar(const FoldSeg &g, const void *const
   return s;
 }
 
-// Build-time register bound of k_fold (ES_FOLD_MINB resident 256-thread blocks per SM; 0 = none).
-#ifndef ES_FOLD_MINB
-#define ES_FOLD_MINB 0
-#endif
-#if ES_FOLD_MINB > 0
-#define ES_FOLD_LB __launch_bounds__(256, ES_FOLD_MINB)
-#else
-#define ES_FOLD_LB __launch_bounds__(256)
-#endif
-
 template <typename T, int MAXSEG, int MAXSRC, bool COMPAT>
-__global__ void ES_FOLD_LB k_fold(const __grid_constant__ FoldParams<MAXSEG, MAXSRC> p) {
+__device__ __forceinline__ void fold_body(const FoldParams<MAXSEG, MAXSRC> &p) {
   constexpr int V = T::kVec;
   // post-scale unless a pre-scale variant already applied 1/N (R5 vs NEXT-3)
   const bool post = !COMPAT || !(p.compat & (kPreDiv | kPreMul));
@@ -429,6 +429,18 @@ __global__ void ES_FOLD_LB k_fold(const __grid_constant__ FoldParams<MAXSEG, MAX
       for (int j = 0; j < g.npush; ++j) T::store1(const_cast<void *>(src[cnt_src + j]), t, o);
     }
   }
+}
+
+// fp32: compiled as in round 1 (62 registers, no bound).  bf16 (k_fold_b): at most 64 registers
+// (4 resident 256-thread blocks per SM) -- the merged first batch otherwise takes 79 and drops to
+// 3 (profiles/r02_fold_variants.md).
+template <typename T, int MAXSEG, int MAXSRC, bool COMPAT>
+__global__ void __launch_bounds__(256) k_fold(const __grid_constant__ FoldParams<MAXSEG, MAXSRC> p) {
+  fold_body<T, MAXSEG, MAXSRC, COMPAT>(p);
+}
+template <typename T, int MAXSEG, int MAXSRC, bool COMPAT>
+__global__ void __launch_bounds__(256, 4) k_fold_b(const __grid_constant__ FoldParams<MAXSEG, MAXSRC> p) {
+  fold_body<T, MAXSEG, MAXSRC, COMPAT>(p);
 }
 
 // ---- k_fold_pipe: the PEER_CHAIN rounds as one tile-pipelined kernel ----------------
@@ -705,8 +717,13 @@ cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSeg
     (void)KernelReg<k_fold_tma<T, MAXSEG, MAXSRC, kS>>::token;
     return cudaLaunchKernelEx(&cfg, k_fold_tma<T, MAXSEG, MAXSRC, kS>, p);
   }
-  if (compat) return launch_k<k_fold<T, MAXSEG, MAXSRC, true>>(dim3(p.nblocks), dim3(threads), s, p);
-  return launch_k<k_fold<T, MAXSEG, MAXSRC, false>>(dim3(p.nblocks), dim3(threads), s, p);
+  if constexpr (T::kSize == 2) {
+    if (compat) return launch_k<k_fold_b<T, MAXSEG, MAXSRC, true>>(dim3(p.nblocks), dim3(threads), s, p);
+    return launch_k<k_fold_b<T, MAXSEG, MAXSRC, false>>(dim3(p.nblocks), dim3(threads), s, p);
+  } else {
+    if (compat) return launch_k<k_fold<T, MAXSEG, MAXSRC, true>>(dim3(p.nblocks), dim3(threads), s, p);
+    return launch_k<k_fold<T, MAXSEG, MAXSRC, false>>(dim3(p.nblocks), dim3(threads), s, p);
+  }
 }
 
 template <typename T>
