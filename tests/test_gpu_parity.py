@@ -783,6 +783,8 @@ def test_random_schedules_mappings_layouts(seed):
     rng.shuffle(m)
     nb = int(rng.integers(1, 5))
     sizes = [int(rng.choice([0, 1, 7, 15, 16, 17, 1000, 8191, 8193, 65537, 300_001])) for _ in range(nb)]
+    if seed % 5 == 3:                     # chunks above 2^20 elements: the pipelined CHAIN cuts W >= 2 tiles
+        sizes[0] = int(N * (1 << 20) + rng.integers(1, 3 * (1 << 20)))
     sizes[0] = max(sizes[0], 1)                                   # at least one non-empty bucket
     dts = [str(rng.choice(["f32", "bf16"])) for _ in range(nb)]
     A = int(rng.choice([8, 16, 64, 1024]))
