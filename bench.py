@@ -564,6 +564,11 @@ def main():
     buckets = cfg["buckets"]
     B = len(buckets)
     rehearse = args.rehearse_same_gpu and world > 1
+    # how the rehearsal's ranks share the one GPU: CUDA MPS runs them concurrently (each limited to
+    # CUDA_MPS_ACTIVE_THREAD_PERCENTAGE of the SMs); otherwise separate processes time-slice it
+    mps = os.environ.get("CUDA_MPS_PIPE_DIRECTORY") or os.environ.get("CUDA_MPS_ACTIVE_THREAD_PERCENTAGE")
+    share_mode = (f"concurrently under CUDA MPS, each rank <= {os.environ.get('CUDA_MPS_ACTIVE_THREAD_PERCENTAGE', '100')} "
+                  f"% of the SMs" if mps else "separate processes time-slicing the GPU (no MPS)")
     # Host inputs BEFORE CUDA is initialised (forked workers draw them on this rank's share of the
     # cores).  Rank 0 also draws the remote ESTs: it checks the whole output against the oracle.
     need = list(range(N)) if rank == 0 and not args.no_full_parity else local
@@ -948,7 +953,7 @@ def main():
              "avg_launch_us": round(us, 2), "timing": how, "avg_launch_us_event_pairs": round(ev_us, 2),
              "share_of_step": round(us * n_ / steps_profiled / 1e3 / ms, 3),
              "peak_source": peak_src if bound == "hbm" else "B200_PROFILING.md measured peer copy per direction",
-             **({"rehearsal": "all ranks on cuda:0: peer bytes counted as HBM bytes, ranks time-slice one GPU"}
+             **({"rehearsal": f"all ranks on cuda:0: peer bytes counted as HBM bytes; {share_mode}"}
                 if rehearse and costs is not None else {}),
              "frac_of_nominal": round(a / (HBM_NOMINAL_GBPS if bound == "hbm" else NVL_NOMINAL_GBPS), 4)}
         return r
@@ -962,7 +967,8 @@ def main():
         "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": cfg["dtype"], "data": "synthetic",
         "config": {**workload_config(args, cfg, G), "graph": graph is not None,
-                   **({"rehearsal": "all ranks on cuda:0 (functional check of the N>1 path, not a scaling number)"}
+                   **({"rehearsal": f"all ranks on cuda:0 ({share_mode}; functional check of the N>1 path, "
+                                    "not a scaling number)"}
                       if rehearse else {}),
                    "api": "per-bucket" if args.per_bucket else ("incremental" if args.incremental else
                                                                ("zero-copy-inplace" if args.inplace else
@@ -1004,7 +1010,7 @@ def main():
         if costs is not None:
             ar["roofline"] = plan_roofline(costs, ar_ph, peak)
             if rehearse:   # what the plan would take on G GPUs; measured here on ONE shared GPU
-                ar["roofline"]["rehearsal"] = ("all ranks time-slice cuda:0 (separate processes, no MPS): "
+                ar["roofline"]["rehearsal"] = (f"all ranks share cuda:0 ({share_mode}): "
                                                "t_measured is not a G-GPU time; t_roof is the G-GPU model")
         elif not args.incremental:
             fold_bytes = (N + 1) * sum(n for n, _ in buckets) * esz          # (N+1) L b: SURVEY 8(d), G = 1
