@@ -11,18 +11,31 @@ import os
 import pytest
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-G1_SHA = {  # whole-output oracle SHA-256 of the G = 1 lines of the same workloads
-    "resnet50": "aba86c1309381f1c144e4941229a8e3f6ef08c38e753851f61e8133f81ed161f",
-    "swin_b": "9d346f3ce5f85666fff141cefda48fe0757fdcffccbebfa9daa6be85c8018a27",
-}
+def _g1_sha():
+    """whole-output oracle SHA-256 of the committed G = 1 line of each workload"""
+    out = {}
+    for name in ("tiny", "resnet50", "vgg19", "bert_base", "swin_b"):
+        with open(os.path.join(ROOT, "profiles", f"r02_bench_{name}_g1.json")) as f:
+            d = json.load(f)
+        assert d["parity"]["sha256_equal"]
+        out[name] = d["output_sha256"]
+    return out
 
 
-def _lines():
-    with open(os.path.join(ROOT, "profiles", "r02_rehearsal_same_gpu.jsonl")) as f:
+G1_SHA = _g1_sha()
+
+
+def _lines(name="r02_rehearsal_same_gpu.jsonl"):
+    with open(os.path.join(ROOT, "profiles", name)) as f:
         return [json.loads(l) for l in f if l.strip()]
 
 
-@pytest.mark.parametrize("d", _lines(), ids=lambda d: d["run"])
+def _all_lines():
+    # time-sliced processes, and the same under CUDA MPS (ranks running concurrently)
+    return _lines() + _lines("r02_rehearsal_mps.jsonl")
+
+
+@pytest.mark.parametrize("d", _all_lines(), ids=lambda d: d["run"])
 def test_rehearsal_line_contract(d):
     with open(os.path.join(ROOT, "BASELINE.json")) as f:
         assert d["metric"] == json.load(f)["metric"]
@@ -52,7 +65,7 @@ def test_rehearsal_line_contract(d):
             assert k["bound"] == "hbm"       # peer bytes never cross NVLink on one GPU
     p = d["parity"]
     assert p["mismatched_words"] == 0 and p["full_output_checked"] and p["full_output_mismatched_words"] == 0
-    assert p["sha256_equal"] and d["output_sha256"] == G1_SHA.get(d["config"]["workload"], d["output_sha256"])
+    assert p["sha256_equal"] and d["output_sha256"] == G1_SHA[d["config"]["workload"]]
     assert "ring_crosscheck" in d
 
 
@@ -67,7 +80,7 @@ def test_fallback_ladder_recorded():
 
 def test_every_g_prints_the_same_hash():
     by = {}
-    for d in _lines():
+    for d in _all_lines():
         by.setdefault(d["config"]["workload"], set()).add(d["output_sha256"])
     for w, hs in by.items():
         assert len(hs) == 1, w
