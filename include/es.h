@@ -300,7 +300,8 @@ es_status es_stash_and_switch(es_handle h, int32_t est, int32_t n, const int32_t
  * chunks with EST c+1 local, for CHAIN / PEER_CHAIN a chain's first segment --
  * has a prefix of local ESTs c+1, c+2, ... (ascending, up to the wrap
  * N-1 -> 0, never the rank's last local EST, leaving the segment at least one
- * EST).  At the stash of a prefix EST its contribution is folded straight into
+ * EST, and only if its q contributions outweigh the fp32 partial that replaces
+ * them: q·b > 4 bytes, i.e. q >= 2 for fp32 and q >= 3 for bf16).  At the stash of a prefix EST its contribution is folded straight into
  * the running unrounded fp32 partial of that chunk (the first prefix EST opens
  * it); everything else of its gradient -- ranges peers or the exchange read,
  * chunks after the wrap -- is copied to the slot (COPY) or kept (BORROW).

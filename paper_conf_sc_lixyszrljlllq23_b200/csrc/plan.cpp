@@ -334,7 +334,8 @@ void plan_peer_chain(const Plan &p, BucketPlan *b) {
 // Local ESTs stash in ascending order, so the prefix stops at the wrap
 // N-1 -> 0; it never takes the last local EST (nothing is left to overlap
 // with after its stash, and the end fold reads it straight from its stash)
-// and leaves the segment's end fold at least one source.
+// and leaves the segment's end fold at least one source.  A prefix is taken only if its q
+// contributions outweigh the fp32 partial that replaces them in the end fold (q·b > 4 bytes).
 void plan_incremental(const Plan &p, BucketPlan *b) {
   b->inc.clear();
   b->inc_q.assign(p.N, 0);
@@ -362,7 +363,9 @@ void plan_incremental(const Plan &p, BucketPlan *b) {
       if (e >= p.N || p.est_to_gpu[e] != g || e == last_local) break;
       ++q;
     }
-    if (q == 0) continue;
+    // worth it only if the end fold then reads fewer bytes: q contributions (q*b) become one
+    // fp32 partial (4 B) -- fp32 needs q >= 2, bf16 q >= 3
+    if ((uint64_t)q * b->esize <= 4) continue;
     b->inc_q[c] = q;
     b->inc.push_back({c, first, q, r.lo, r.hi});
   }

@@ -34,7 +34,8 @@ struct Part {
 // shard); first = (c+1) mod N.  q >= 1 only; q ends before the wrap N-1 -> 0
 // (ESTs run in ascending order), never takes this rank's last local EST (its
 // contribution joins the end fold straight from its stash) and leaves at least
-// one source of the segment to the end fold.
+// one source of the segment to the end fold; only prefixes with q·b > 4 (they must save more
+// end-fold reads than the 4-byte partial costs) are kept.
 struct IncChunk {
   int32_t c, first, q;
   int64_t lo, hi;

@@ -105,6 +105,31 @@ def bound_ms_pipelined(costs):
     return bound_ms(merged)
 
 
+def next1_tail_saving(name, G, kind, sched):
+    """NEXT-1 (es_plan_incremental): per rank, the end-of-step fold reads that move to the stashes
+    -- q contributions per element of each row, less the fp32 partial read instead -- as a share of
+    that rank's end-of-step fold reads; returns the slowest rank's (max fold bytes) saving."""
+    c = workloads.config(name)
+    N = c["N"]
+    m = workloads.mapping(N, G, kind)
+    buckets = [(n, es.ES_F32 if d == "f32" else es.ES_BF16) for n, d in c["buckets"]]
+    worst = None
+    for g in range(G):
+        cfg = es.Config(N, G, g, m, buckets, sched=sched, options=es.ES_OPT_INCREMENTAL)
+        fold = saved = 0
+        for b, (L, dt) in enumerate(buckets):
+            esz = 2 if dt == es.ES_BF16 else 4
+            ops, _ = es.es_plan_ops(cfg, b)
+            for f in ops:
+                if int(f[0]) == es.ES_OP_FOLD:
+                    fold += (int(f[2]) - int(f[1])) * esz * (N if int(f[3]) < 0 else int(f[4]))
+            for _c, _first, q, lo, hi in es.es_plan_incremental(cfg, b).tolist():
+                saved += (hi - lo) * (q * esz - 4)
+        if worst is None or fold > worst[0]:
+            worst = (fold, saved)
+    return worst[1] / worst[0] if worst and worst[0] else 0.0
+
+
 def main(path):
     rows = ["# Multi-GPU roofline of the exported plans (allreduce only; HBM 6.46 TB/s, NVLink 0.77 TB/s)\n",
             "Per phase (between groups / barriers), the slowest rank's max(HBM, NVLink) time, summed.\n",
@@ -115,9 +140,13 @@ def main(path):
             "gather's remote loads and one phase boundary (not modelled here).\n",
             "chain pipelined = CHAIN over NCCL as chain_pipelined runs it (tile wavefront: every round's folds "
             "and transfers overlapped, then the all-gather group).\n",
+            "NEXT-1 = the share of the slowest rank's end-of-step fold reads that es_stash_fold_grads moves to the "
+            "stashes (es_plan_incremental rows: q contributions per element, less the fp32 partial read), under "
+            "the AUTO schedule.\n",
             "| config | G | mapping | direct ms | chain ms (rounds) | chain pipelined ms | peer ms | peer push ms | "
-            "peer_chain ms | peer_chain pipelined ms | AUTO picks | max NVLink in / rank MB (direct, chain) |",
-            "|---|---|---|---|---|---|---|---|---|---|---|---|"]
+            "peer_chain ms | peer_chain pipelined ms | AUTO picks | max NVLink in / rank MB (direct, chain) | "
+            "NEXT-1 tail reads moved |",
+            "|---|---|---|---|---|---|---|---|---|---|---|---|---|"]
     cases = [("resnet50", G, "contiguous") for G in (2, 4, 8)] + [("vgg19", G, "contiguous") for G in (2, 4, 8)] + \
         [("bert_base", 8, "contiguous"), ("bert_base", 8, "round_robin")] + \
         [("swin_b", G, "contiguous") for G in (2, 4, 8)]
@@ -134,7 +163,11 @@ def main(path):
         rows.append(f"| {name} | {G} | {kind} | {bound_ms(res['direct']):.3f} | {bound_ms(res['chain']):.3f} | "
                     f"{bound_ms_pipelined(res['chain']):.3f} | "
                     f"{bound_ms(res['peer']):.3f} | {bound_ms(res['peer_push']):.3f} | {bound_ms(res['peer_chain']):.3f} | "
-                    f"{bound_ms_pipelined(res['peer_chain']):.3f} | {pick} | {nvd:.0f}, {nvc:.0f} |")
+                    f"{bound_ms_pipelined(res['peer_chain']):.3f} | {pick} | {nvd:.0f}, {nvc:.0f} | "
+                    f"{100 * next1_tail_saving(name, G, kind, es.ES_SCHED_AUTO):.0f} % |")
+    g1 = ", ".join(f"{n} {100 * next1_tail_saving(n, 1, 'contiguous', es.ES_SCHED_AUTO):.0f} %"
+                   for n in ("resnet50", "vgg19", "bert_base", "swin_b"))
+    rows.append(f"\nNEXT-1 tail reads moved at G = 1 (same measure): {g1}.")
     text = "\n".join(rows) + "\n"
     with open(path, "w") as f:
         f.write(text)

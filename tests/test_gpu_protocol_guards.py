@@ -23,8 +23,9 @@ pytestmark = pytest.mark.gpu
 
 def test_export_refuses_partially_folded_slot():
     """NEXT-1 (es_stash_fold_grads) at G = 1, N = 4: EST 0 opens chunk 3's partial (its
-    sequence 0, 1, 2, 3 starts there), EST 1 folds into chunks 3 and 0, EST 2 into 3, 0, 1;
-    EST 3, the last local EST, folds nothing and its COPY slot holds its whole gradient."""
+    sequence 0, 1, 2, 3 starts there), EST 1 folds into chunk 3 and opens chunk 0's, EST 2 folds
+    into both (chunk 1's one-EST prefix is not worth a partial); EST 3, the last local EST, folds
+    nothing and its COPY slot holds its whole gradient."""
     N, L = 4, 100003
     agg = Aggregator(N, 1, 0, [0] * N, [(L, "f32")], options=es.ES_OPT_INCREMENTAL)
     rng = np.random.default_rng(5)

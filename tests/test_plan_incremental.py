@@ -32,22 +32,23 @@ def _shard(L, G, h, A=16):
     return min(L, S * h), min(L, S * (h + 1))
 
 
-def _rows(N, G, rank, m, L, sched):
-    cfg = es.Config(N, G, rank, m, [(L, es.ES_F32)], sched=sched, options=es.ES_OPT_INCREMENTAL)
+def _rows(N, G, rank, m, L, sched, esz=4):
+    cfg = es.Config(N, G, rank, m, [(L, es.ES_F32 if esz == 4 else es.ES_BF16)], sched=sched,
+                    options=es.ES_OPT_INCREMENTAL)
     ops, sch = es.es_plan_ops(cfg, 0)
     return es.es_plan_incremental(cfg, 0), sch
 
 
-def _check_rank(N, G, g, m, L, sched):
-    rows, sch = _rows(N, G, g, m, L, sched)
+def _check_rank(N, G, g, m, L, sched, esz=4):
+    rows, sch = _rows(N, G, g, m, L, sched, esz)
     C = _chunk(L, N)
     local = [e for e in range(N) if m[e] == g]
     last_local = local[-1]
-    seen = set()
+    seen, seen_q = set(), {}
     for c, first, q, lo, hi in rows.tolist():
         assert c not in seen and (not seen or c > max(seen)), "rows ascend in c"
         seen.add(c)
-        assert first == (c + 1) % N and q >= 1
+        assert first == (c + 1) % N and q * esz > 4, "a prefix must save more than the partial costs"
         pre = list(range(first, first + q))
         assert pre[-1] <= N - 1, "the prefix never wraps N-1 -> 0"
         assert all(m[e] == g for e in pre) and last_local not in pre
@@ -66,6 +67,7 @@ def _check_rank(N, G, g, m, L, sched):
         assert q <= seg_len - 1, "the end fold keeps at least one source"
         nxt = first + q        # maximal: the prefix stops only where the rule says
         assert nxt >= N or m[nxt] != g or nxt == last_local or q == seg_len - 1
+        seen_q[c] = q
     # completeness: every chunk whose sequence starts here with a foldable EST has a row
     for c in range(N):
         first = (c + 1) % N
@@ -77,19 +79,25 @@ def _check_rank(N, G, g, m, L, sched):
         while run < N and m[(first + run) % N] == g:
             run += 1
         seg_len = run if sch in (es.ES_SCHED_CHAIN, es.ES_SCHED_PEER_CHAIN) else N
-        can = m[first] == g and first != last_local and seg_len >= 2 and chi > clo
+        q = 0                  # the rule, restated: local, ascending, not the last local EST
+        while q < seg_len - 1 and first + q < N and m[first + q] == g and first + q != last_local:
+            q += 1
+        can = m[first] == g and chi > clo and q * esz > 4
         assert (c in seen) == can, f"chunk {c}"
+        if can:
+            assert seen_q[c] == q
     return rows
 
 
+@pytest.mark.parametrize("esz", [4, 2])
 @pytest.mark.parametrize("N,G", [(4, 1), (4, 2), (4, 3), (4, 4), (6, 3), (5, 2)])
-def test_incremental_prefixes_follow_the_rule(N, G):
+def test_incremental_prefixes_follow_the_rule(N, G, esz):
     for sched in (SCHEDS if G > 1 else [es.ES_SCHED_AUTO]):
         for m in _surjections(N, G):
             for L in (N * 16 * 3 + 5, 40):        # ragged tail; 40 < N*C leaves chunks empty
                 owners = {}
                 for g in range(G):
-                    for c, first, q, lo, hi in _check_rank(N, G, g, m, L, sched).tolist():
+                    for c, first, q, lo, hi in _check_rank(N, G, g, m, L, sched, esz).tolist():
                         for i in range(lo, hi):   # every element's partial belongs to one rank
                             assert i not in owners
                             owners[i] = g
