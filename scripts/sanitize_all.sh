@@ -6,7 +6,7 @@
 #    schedule (peer_chain_rounds) is covered.
 #  * initcheck does not see cp.async.bulk (TMA) global writes, so the TMA-ring stash of
 #    ES_OPT_STASH_BACKGROUND (g1_bg) reports reads of slot memory as uninitialised although the
-#    results are bit-exact (ES_STASH_TMA=1 shows the same); initcheck runs without g1_bg, and
+#    results are bit-exact (round 1's TMA stash variant showed the same); initcheck runs without g1_bg, and
 #    g1_bg's count is recorded separately.
 mkdir -p gpurun_out
 out=gpurun_out/sanitizer.txt; : > $out
