@@ -1312,6 +1312,27 @@ def allgather_busbw(G, dev, max_over_ranks, total_bytes=1 << 30, iters=10):
         return {"error": f"{type(e).__name__}: {e}"}
 
 
+def ring_start_offsets(xs, got):
+    """Diagnostic of the ring cross-check ("which rotation matched"): xs = the Nx
+    ranks' fp32 inputs (Nx * C elements, C = one ring chunk), got = an all-reduced result scaled by
+    fl32(1/Nx).  The oracle on the inputs rotated by d folds chunk c starting at rank c+1+d; returns,
+    per chunk, the d whose words equal `got` (0 = reading R2; None = no rotation of the rank order
+    matches -- the ring is then another permutation of the ranks).  With Nx = 2 every rotation is
+    the same commutative add, so the offsets read 0."""
+    import numpy as np
+    import oracle
+    Nx, Lx = len(xs), len(xs[0])
+    C = Lx // Nx
+    g = np.asarray(got, dtype=np.float32).view(np.uint32)
+    offs = [None] * Nx
+    for d in range(Nx):
+        want_d = oracle.reduce([xs[(k + d) % Nx] for k in range(Nx)], "f32", L=Lx).view(np.uint32)
+        for c in range(Nx):
+            if offs[c] is None and np.array_equal(want_d[c * C:(c + 1) * C], g[c * C:(c + 1) * C]):
+                offs[c] = d
+    return offs
+
+
 def ring_crosscheck(args, name, N, G, rank, rehearse, dev, host):
     """NEXT-3 (iii): one EST per GPU (N_x = G ring participants; rank k contributes
     EST k's gradients of the workload, so any G >= 2 of a scaling run checks the reading, not only
@@ -1367,8 +1388,10 @@ def ring_crosscheck(args, name, N, G, rank, rehearse, dev, host):
     xs = [host[(k, b)][:Lx] if (k, b) in host else drawn[k] for k in range(Nx)]
     want = oracle.reduce(xs, "f32", L=Lx)
     eq = int((want.view(np.uint32) == got.view(np.uint32)).sum())
+    offs = ring_start_offsets(xs, got)
     return {"bucket": b, "ring_ranks": Nx, "ests": f"0..{Nx - 1} (one per GPU)", "elements": Lx,
             "ring_chunk_elements": Lx // Nx, "words_equal": eq, "frac_equal": eq / Lx,
+            "start_offset_per_chunk": offs,
             "nccl": "ncclAllReduce sum, NCCL_ALGO=Ring NCCL_PROTO=Simple, min/max CTAs 1, times fl32(1/G)",
             "nccl_sha256": hashlib.sha256(got.tobytes()).hexdigest(),
             "oracle_sha256": hashlib.sha256(want.tobytes()).hexdigest()}

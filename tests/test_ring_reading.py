@@ -57,3 +57,30 @@ def test_ring_simulation_distinguishes_start_ranks():
     out = ring_allreduce(xs)
     assert out[0] == 0.5 and out[16] == 0.5 and out[32] == 0.0 and out[48] == 0.25
     assert np.array_equal(out.view(np.uint32), oracle.reduce(xs, "f32").view(np.uint32))
+
+
+def ring_allreduce_started(xs, shift):
+    """The same ring, but every chunk's reduce-scatter starts `shift` ranks later (rank r sends
+    chunk (r - 1 - shift - s) mod N at step s): chunk c is folded from rank c+1+shift on."""
+    N = len(xs)
+    rot = [xs[(k + shift) % N] for k in range(N)]
+    out = ring_allreduce(rot)           # ring over the relabelled ranks
+    return out
+
+
+@pytest.mark.parametrize("N", [2, 4, 8])
+def test_bench_ring_diagnostic_names_the_start_rank(N):
+    """bench.py's ring_crosscheck diagnostic (ring_start_offsets) reports, per chunk, how far the
+    ring's start rank is from reading R2's c+1: 0 for the R2 ring, `shift` for a shifted one.
+    With two ranks every rotation is the same single (commutative) add: offsets read 0."""
+    import os
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import bench
+    rng = np.random.default_rng(50 + N)
+    L = N * 4096
+    xs = [(rng.standard_normal(L) * 10.0 ** rng.uniform(-3, 3, L)).astype(np.float32) for _ in range(N)]
+    assert bench.ring_start_offsets(xs, ring_allreduce(xs)) == [0] * N
+    for shift in range(1, N):
+        want = [0] * N if N == 2 else [shift] * N
+        assert bench.ring_start_offsets(xs, ring_allreduce_started(xs, shift)) == want
