@@ -1388,7 +1388,10 @@ def ring_crosscheck(args, name, N, G, rank, rehearse, dev, host):
     xs = [host[(k, b)][:Lx] if (k, b) in host else drawn[k] for k in range(Nx)]
     want = oracle.reduce(xs, "f32", L=Lx)
     eq = int((want.view(np.uint32) == got.view(np.uint32)).sum())
-    offs = ring_start_offsets(xs, got)
+    try:
+        offs = ring_start_offsets(xs, got)
+    except Exception as e:     # a diagnostic: never fail the line over it
+        offs = f"{type(e).__name__}: {e}"
     return {"bucket": b, "ring_ranks": Nx, "ests": f"0..{Nx - 1} (one per GPU)", "elements": Lx,
             "ring_chunk_elements": Lx // Nx, "words_equal": eq, "frac_equal": eq / Lx,
             "start_offset_per_chunk": offs,
