@@ -39,7 +39,6 @@ namespace es {
 namespace {
 
 constexpr int kSMs = 148;        // B200
-constexpr int kBatch = 8;        // sources loaded per batch in k_fold
 // Grid cap: measured on B200 (scripts/sweep_launch.py, profiles/), near
 // one-shot grids (each thread ~1 vector per segment) stream better than
 // persistent grid-stride ones; 148 x 64 blocks covers every bucket this build
@@ -103,6 +102,24 @@ __device__ __forceinline__ float ld_cg1(const float *p) {
   float r;
   asm volatile("ld.global.cg.f32 %0, [%1];" : "=f"(r) : "l"(p) : "memory");
   return r;
+}
+
+// 32-byte accesses (LDG.E.256 / STG.E.256 on sm_100a), used by the small-fold type F32WT.
+struct V32 {
+  int4 a, b;
+};
+__device__ __forceinline__ V32 ld_stream(const V32 *p) {
+  V32 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v8.s32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+               : "=r"(r.a.x), "=r"(r.a.y), "=r"(r.a.z), "=r"(r.a.w), "=r"(r.b.x), "=r"(r.b.y), "=r"(r.b.z),
+                 "=r"(r.b.w)
+               : "l"(p));
+  return r;
+}
+__device__ __forceinline__ void st_stream(V32 *p, const V32 &v) {
+  asm volatile("st.global.L1::no_allocate.v8.s32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(p), "r"(v.a.x),
+               "r"(v.a.y), "r"(v.a.z), "r"(v.a.w), "r"(v.b.x), "r"(v.b.y), "r"(v.b.z), "r"(v.b.w)
+               : "memory");
 }
 
 __device__ __forceinline__ void st_stream(void *p, const int4 &v) {
@@ -188,6 +205,9 @@ void split_blocks(const std::vector<int64_t> &work, int total, std::vector<int32
 struct F32T {
   static constexpr int kVec = 4;
   static constexpr int kSize = 4;
+  static constexpr int kBatch = 8;      // sources per load batch in k_fold
+  static constexpr bool kMerge = false; // opening contribution loaded alone (profiles/r02_fold_variants.md)
+  using Load = int4;
   __device__ static __forceinline__ void widen(const int4 &v, float *a) {
     a[0] = __int_as_float(v.x); a[1] = __int_as_float(v.y);
     a[2] = __int_as_float(v.z); a[3] = __int_as_float(v.w);
@@ -207,6 +227,9 @@ struct F32T {
 struct BF16T {
   static constexpr int kVec = 8;
   static constexpr int kSize = 2;
+  static constexpr int kBatch = 8;
+  static constexpr bool kMerge = true;  // opening contribution in the first batch (+2.4 % BERT fold)
+  using Load = int4;
   // bf16 is the high half of an fp32: widening is exact (R4).
   __device__ static __forceinline__ void widen2(uint32_t w, float *a) {
     a[0] = __uint_as_float(w << 16);
@@ -232,6 +255,26 @@ struct BF16T {
     reinterpret_cast<unsigned short *>(p)[i] = __bfloat16_as_ushort(__float2bfloat16_rn(v));
   }
 };
+
+// fp32, 8 elements (32 bytes) per thread and source: the small-fold type.  A fold of at most
+// kWideMaxElems elements is latency-bound (1M fp32 = 1.7 waves of one-vector threads); F32WT
+// halves the threads to one wave and, with the opening contribution in the first batch, needs
+// one memory round trip per thread (launch_fold_multi picks it; same per-element arithmetic).
+struct F32WT {
+  static constexpr int kVec = 8;
+  static constexpr int kSize = 4;
+  static constexpr int kBatch = 4;      // 4 x 32 B in flight: the registers of F32T's 8 x 16 B
+  static constexpr bool kMerge = true;
+  using Load = V32;
+  __device__ static __forceinline__ void widen(const V32 &v, float *a) {
+    F32T::widen(v.a, a);
+    F32T::widen(v.b, a + 4);
+  }
+  __device__ static __forceinline__ V32 narrow(const float *a) { return V32{F32T::narrow(a), F32T::narrow(a + 4)}; }
+  __device__ static __forceinline__ float load1(const void *p, int64_t i) { return F32T::load1(p, i); }
+  __device__ static __forceinline__ void store1(void *p, int64_t i, float v) { F32T::store1(p, i, v); }
+};
+constexpr int64_t kWideMaxElems = 1 << 21;
 
 // ---- k_fold ---------------------------------------------------------------
 
@@ -300,7 +343,9 @@ __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const 
   // ones -- one memory round trip for up to kBatch sources instead of a dependent one first;
   // measured +2.8 % on BERT's fold (profiles/r02_fold_variants.md).  fp32 keeps the separate
   // opening load, which measured 1.9-2.1 % faster there (Swin-B, VGG-19).  Same adds, same order.
-  constexpr bool MERGE = T::kSize == 2;
+  constexpr bool MERGE = T::kMerge;
+  constexpr int KB = T::kBatch;
+  using LD = typename T::Load;
   bool open = g.part_in == nullptr;
   int done = 0;
   if (!open) {
@@ -312,7 +357,7 @@ __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const 
       acc[4 * q + 2] = __int_as_float(w.z); acc[4 * q + 3] = __int_as_float(w.w);
     }
   } else if (!MERGE) {
-    int4 w = ld_stream(reinterpret_cast<const char *>(src[idx]) + boff);
+    LD w = ld_stream(reinterpret_cast<const LD *>(reinterpret_cast<const char *>(src[idx]) + boff));
     T::widen(w, acc);
 #pragma unroll
     for (int e = 0; e < V; ++e) acc[e] = prep<COMPAT>(acc[e], compat, r, fN);
@@ -321,18 +366,18 @@ __device__ __forceinline__ void fold_vector(const FoldSeg &g, const void *const 
     open = false;
   }
   while (done < cnt) {
-    const int nb = min(kBatch, cnt - done);
-    int4 buf[kBatch];
+    const int nb = min(KB, cnt - done);
+    LD buf[KB];
     int k = idx;
 #pragma unroll
-    for (int b = 0; b < kBatch; ++b) {                        // all loads of the batch first ...
+    for (int b = 0; b < KB; ++b) {                            // all loads of the batch first ...
       if (b < nb) {
-        buf[b] = ld_stream(reinterpret_cast<const char *>(src[k]) + boff);
+        buf[b] = ld_stream(reinterpret_cast<const LD *>(reinterpret_cast<const char *>(src[k]) + boff));
         k = (k + 1 == cnt) ? 0 : k + 1;
       }
     }
 #pragma unroll
-    for (int b = 0; b < kBatch; ++b) {                        // ... then the adds, in canonical order
+    for (int b = 0; b < KB; ++b) {                            // ... then the adds, in canonical order
       if (b < nb) {
         float x[V];
         T::widen(buf[b], x);
@@ -409,12 +454,13 @@ __device__ __forceinline__ void fold_body(const FoldParams<MAXSEG, MAXSRC> &p) {
 #pragma unroll
         for (int e = 0; e < V; ++e) acc[e] = __fmul_rn(acc[e], p.r);   // R5: one rounding
       }
-      const int4 w = T::narrow(acc);                                   // R13
-      st_stream(reinterpret_cast<char *>(g.out) + t * T::kSize, w);
+      using LD = typename T::Load;
+      const LD w = T::narrow(acc);                                     // R13
+      st_stream(reinterpret_cast<LD *>(reinterpret_cast<char *>(g.out) + t * T::kSize), w);
       // ES_OPT_PEER_PUSH: the same words into every peer's RESULT area over NVLink (posted
       // stores), so the all-gather's traffic rides the fold's otherwise idle egress
       for (int j = 0; j < g.npush; ++j)
-        st_stream(reinterpret_cast<char *>(const_cast<void *>(src[cnt_src + j])) + t * T::kSize, w);
+        st_stream(reinterpret_cast<LD *>(reinterpret_cast<char *>(const_cast<void *>(src[cnt_src + j])) + t * T::kSize), w);
     }
   }
   const int64_t tail0 = nvec * V;                                    // ragged tail (< V elements)
@@ -687,6 +733,9 @@ cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSeg
   std::vector<int32_t> block0;
   split_blocks(work, total, &block0, &p.nblocks);
   for (int i = 0; i < nseg; ++i) p.seg[i].block0 = block0[i];
+  if constexpr (std::is_same<T, F32WT>::value) {   // small canonical folds only (launch_fold_multi)
+    return launch_k<k_fold<T, MAXSEG, MAXSRC, false>>(dim3(p.nblocks), dim3(threads), s, p);
+  } else {
   bool tma_ok = g_fold_tma > 0 && !compat && N <= 16 && bo == 0 && to == 0;
   for (int i = 0; i < nseg && tma_ok; ++i) tma_ok = d[i].rot && !d[i].part_in && !d[i].out_partial && !d[i].npush;
   if (tma_ok) {
@@ -723,6 +772,7 @@ cudaError_t launch_fold_group(int32_t N, float r, uint32_t compat, const FoldSeg
   } else {
     if (compat) return launch_k<k_fold<T, MAXSEG, MAXSRC, true>>(dim3(p.nblocks), dim3(threads), s, p);
     return launch_k<k_fold<T, MAXSEG, MAXSRC, false>>(dim3(p.nblocks), dim3(threads), s, p);
+  }
   }
 }
 
@@ -1308,6 +1358,18 @@ cudaError_t launch_fold_multi(es_dtype dtype, int32_t N, float r, uint32_t compa
   if (live.empty()) return cudaSuccess;
   if (dtype == ES_BF16)
     return launch_fold_t<BF16T>(N, r, compat, live.data(), (int)live.size(), s, blocks_override, threads_override,
+                                launches);
+  // small fp32 folds: 8 elements per thread (F32WT) when every pointer allows 32-byte accesses
+  int64_t elems = 0;
+  bool wide = compat == 0 && blocks_override <= 0;
+  auto a32 = [](const void *q) { return (reinterpret_cast<uintptr_t>(q) & 31) == 0; };
+  for (const FoldSegDesc &d : live) {
+    elems += d.n;
+    wide = wide && a32(d.out) && (!d.part_in || a32(d.part_in));
+    for (int j = 0; wide && j < (d.rot ? N : d.m) + d.npush; ++j) wide = a32(d.src[j]);
+  }
+  if (wide && elems <= kWideMaxElems)
+    return launch_fold_t<F32WT>(N, r, compat, live.data(), (int)live.size(), s, blocks_override, threads_override,
                                 launches);
   return launch_fold_t<F32T>(N, r, compat, live.data(), (int)live.size(), s, blocks_override, threads_override,
                              launches);
