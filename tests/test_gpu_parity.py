@@ -829,3 +829,32 @@ def test_stash_background_grid_bit_exact(incremental):
     for b, d in enumerate(dts):
         assert_bits_equal(from_dev(outs[b]), oracle.reduce(xs[b], d), f"b={b}")
     agg.close()
+
+
+# ---- small-fold kernel selection (k_fold<F32WT>) ------------------------------------------------
+
+@pytest.mark.parametrize("L", [8, 17, 10007, 1 << 20, (1 << 21) + 16])
+def test_small_fold_wide_and_narrow_paths(L):
+    """fp32 folds of <= 2^21 elements with 32-byte aligned pointers run 8 elements per thread
+    (k_fold<F32WT>); a BORROWed gradient and an output that are only 16-byte aligned take the
+    F32T kernel; above 2^21 elements F32T as well.  Every path gives the oracle's bits."""
+    from gpu_util import Aggregator, from_dev, to_dev
+    N = 4
+    rng = np.random.default_rng(2100 + L % 97)
+    xs = _gauss(rng, N, L)
+    want = oracle.reduce(xs, "f32")
+    for offset in (0, 4):                  # 4 floats = 16 bytes: breaks 32-byte alignment only
+        agg = Aggregator(N, 1, 0, [0] * N, [(L, "f32")])
+        base = [torch.zeros(L + 8, dtype=torch.float32, device="cuda") for _ in range(N)]
+        devs = []
+        for k in range(N):
+            base[k][offset:offset + L].copy_(to_dev(xs[k]))
+            devs.append(base[k][offset:offset + L])
+        out_base = torch.zeros(L + 8, dtype=torch.float32, device="cuda")
+        out = out_base[offset:offset + L]
+        for k in range(N):
+            agg.stash(k, 0, devs[k], es.ES_STASH_BORROW if k == N - 1 else es.ES_STASH_COPY)
+        agg.allreduce(0, out)
+        torch.cuda.synchronize()
+        assert_bits_equal(from_dev(out), want, f"L={L} offset={offset}")
+        agg.close()
