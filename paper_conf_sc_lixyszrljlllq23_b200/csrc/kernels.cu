@@ -6,8 +6,11 @@
 //
 // All three are HBM-streaming kernels (no data reuse, no contraction), so
 // they use 128-bit vector loads on the non-coherent path with L1
-// no-allocate, many independent loads in flight per thread, coalesced lanes,
-// and grids sized in multiples of the 148 SMs.
+// no-allocate (256-bit for small fp32 folds, k_fold<F32WT>), many independent
+// loads in flight per thread, coalesced lanes, and grids sized in multiples
+// of the 148 SMs.  Element types: F32T (4 fp32 per
+// thread and source), BF16T (8 bf16; k_fold_b), F32WT (8 fp32, folds of at
+// most 2^21 elements with 32-byte aligned operands).
 //
 // Fold and stash are MULTI-SEGMENT kernels: one launch covers many buckets
 // (or many chain segments), each segment owning a contiguous range of
